@@ -1,0 +1,377 @@
+#!/usr/bin/env python
+"""bench.py -- the driver's benchmark contract for the B200 TTLG library.
+
+Metric (BASELINE.json): effective transpose GB/s = 2*N*sizeof(elem)/time/1e9
+(PAPER.md L1501-1505), here summed over one "step" = one pass of the hot path
+over the workload: every case of the TTC-like 57-case suite (BASELINE config 2,
+SURVEY App. A synthetic re-creation), fp64, 200 MiB per tensor, each case one
+`ttlg_execute` of a pre-built plan (repeated-use mode, L1569-1593).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload ttc57|ccsdt|smallfvi|c1]
+  python bench.py --impl reference ...   (the oracle on the host cores)
+
+Inputs are generated on the device by the shared SplitMix64 generator
+(synth/), resident in HBM before the timed region; every tensor (200 MiB in +
+200 MiB out) exceeds the 126 MB L2, so no flush is needed between launches.
+Timing: CUDA events on the launching stream, W warm-up steps, K timed steps,
+barrier + synchronize on both sides, max over ranks.  Multi-GPU (torchrun):
+each rank transposes the full suite on its own GPU (independent problems, no
+data-path collective) -> "scaling": "weak".
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+PEAK_FALLBACK_GBS = 6650.0  # B200_PROFILING.md fallback (only if MEASURED_PEAKS.json absent)
+
+
+def _peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)", d
+    return PEAK_FALLBACK_GBS, "fallback (B200_PROFILING.md)", {}
+
+
+def _workload(name):
+    from synth import configs
+    if name == "ttc57":
+        return "ttc57-fp64-200MiB (BASELINE config 2, synthetic re-creation)", configs.config2()
+    if name == "ccsdt":
+        return "ccsdt-rank6-fp64 (BASELINE config 3)", configs.config3()
+    if name == "smallfvi":
+        return "smallfvi-rank3-fp32 (BASELINE config 4)", configs.config4()
+    if name == "c1":
+        return "rank4-16^4-fp64 all 24 perms (BASELINE config 1)", configs.config1()
+    raise SystemExit(f"unknown workload {name}")
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def start(self):
+        q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+             "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+             "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={q}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.th = threading.Thread(target=self._read, daemon=True)
+            self.th.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.samples.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for s in self.samples:
+            try:
+                sm.append(float(s[0]))
+                mx.append(float(s[1]))
+                for nm, v in zip(names, s[4:8]):
+                    if v.strip().lower() == "active":
+                        reasons.add(nm)
+            except (ValueError, IndexError):
+                continue
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(cases, budget_s=12.0, threads=None):
+    """The oracle as it stands (oracle.c d-nested loop, threaded over the
+    outermost index) on the host cores, on a bounded sample of the workload."""
+    import numpy as np
+    import oracle
+    from synth import gen_tensor_np, case_seed
+    cores = threads or len(os.sched_getaffinity(0))
+    done, t_total, nbytes = [], 0.0, 0
+    for c in cases:
+        A = gen_tensor_np(case_seed(c.case_id), c.n_elems, c.elem_bytes)
+        t0 = time.perf_counter()
+        oracle.transpose(A, c.extents, c.perm, threads=cores)
+        t_total += time.perf_counter() - t0
+        nbytes += c.alg_bytes
+        done.append(c.label())
+        del A
+        if t_total >= budget_s:
+            break
+    return {"value": nbytes / t_total / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
+            "sample": f"{len(done)} of {len(cases)} cases ({', '.join(done[:4])}"
+                      f"{', ...' if len(done) > 4 else ''}), {t_total:.1f} s of oracle time"}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the oracle on the host cores (rank 0 only)."""
+    if rank != 0:
+        return
+    name, cases = _workload(args.workload)
+    import oracle
+    from synth import gen_tensor_np, case_seed
+    cores = len(os.sched_getaffinity(0))
+    times, nb = [], []
+    for step in range(args.warmup + args.steps):
+        c = cases[step % len(cases)]
+        A = gen_tensor_np(case_seed(c.case_id), c.n_elems, c.elem_bytes)
+        t0 = time.perf_counter()
+        oracle.transpose(A, c.extents, c.perm, threads=cores)
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+            nb.append(c.alg_bytes)
+    value = sum(nb) / sum(times) / 1e9
+    line = {"impl": "reference", "metric": "effective transpose GB/s (2*N*s/time)",
+            "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (SplitMix64 bit patterns)",
+            "config": {"workload": name, "step": "one case of the suite per step (bounded)"},
+            "cpu_baseline": {"value": value, "unit": "GB/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{len(times)} timed cases, one per step"},
+            "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0,
+                    "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ttlg", choices=["ttlg", "reference"])
+    ap.add_argument("--workload", default="ttc57")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=12.0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
+    from synth import gen_tensor_torch, case_seed
+
+    name, cases = _workload(args.workload)
+    peak, peak_src, peaks = _peaks()
+    stream = torch.cuda.Stream(device=dev)
+    sptr = stream.cuda_stream
+
+    # ---- resident inputs + plans (outside the timed region)
+    As, Bs, plans, infos = [], [], [], []
+    for c in cases:
+        A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
+        As.append(A)
+        Bs.append(torch.empty_like(A))
+        p = ttlg.plan("f64" if c.elem_bytes == 8 else "f32", c.extents, c.perm)
+        plans.append(p)
+        infos.append(p.describe())
+    torch.cuda.synchronize()
+    step_bytes = sum(c.alg_bytes for c in cases)
+
+    def kname(info):
+        return f"{'k_direct' if info['schema'] in ('FML', 'COPY') else 'k_staged'}" \
+               f"<W={info['access_bytes']}>[{info['schema']}]"
+
+    def one_step(evs=None):
+        with torch.cuda.stream(stream):
+            for i, p in enumerate(plans):
+                if evs is not None:
+                    evs[i][0].record(stream)
+                p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
+                if evs is not None:
+                    evs[i][1].record(stream)
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+
+    # ---- timed region (device events on the launching stream)
+    evs = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            for _ in plans] for _ in range(args.steps)]
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    for s in range(args.steps):
+        one_step(evs[s])
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clk = clocks.stop()
+    elapsed_ms = t_start.elapsed_time(t_end)
+    if world > 1:
+        t = torch.tensor([elapsed_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(t.item())
+    launches = len(plans) * args.steps
+
+    # per-launch durations -> per-kernel shares, model error, per-case table
+    per_case_ms = [[evs[s][i][0].elapsed_time(evs[s][i][1]) for s in range(args.steps)]
+                   for i in range(len(plans))]
+    groups = {}
+    for i, info in enumerate(infos):
+        k = kname(info)
+        g = groups.setdefault(k, {"ms": 0.0, "bytes": 0, "launches": 0})
+        g["ms"] += sum(per_case_ms[i])
+        g["bytes"] += cases[i].alg_bytes * args.steps
+        g["launches"] += args.steps
+    dom = max(groups, key=lambda k: groups[k]["ms"])
+    dg = groups[dom]
+    achieved = dg["bytes"] / (dg["ms"] / 1e3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            with open(tpath) as f:
+                tr = json.load(f)
+            traffic = tr.get(args.workload, {}).get(dom.split("[")[0])
+        except Exception:
+            traffic = None
+    med = [statistics.median(x) for x in per_case_ms]
+    errs = [abs(m * 1e-3 - inf["predicted_seconds"]) / (m * 1e-3) for m, inf in zip(med, infos)]
+
+    # same-size device-to-device copy (the north star's "% of D2D" denominator)
+    d2d_ms = []
+    big = max(range(len(cases)), key=lambda i: cases[i].alg_bytes)
+    src, dst = As[big], Bs[big]
+    with torch.cuda.stream(stream):
+        for _ in range(3):
+            dst.copy_(src)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(10):
+            dst.copy_(src)
+        e1.record(stream)
+    torch.cuda.synchronize()
+    d2d_gbs = 10 * cases[big].alg_bytes / (e0.elapsed_time(e1) / 1e3) / 1e9
+
+    value = world * step_bytes * args.steps / (elapsed_ms / 1e3) / 1e9
+
+    # ---- end to end: C-ABI call with HOST buffers, H2D + D2H inside the timed region
+    e2e = None
+    if args.e2e_steps > 0:
+        try:
+            hA = [torch.empty(A.numel(), dtype=A.dtype, pin_memory=True) for A in As]
+            for h, A in zip(hA, As):
+                h.copy_(A)
+            hB = torch.empty(max(A.numel() for A in As), dtype=As[0].dtype, pin_memory=True)
+            torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(args.e2e_steps):
+                for i, p in enumerate(plans):
+                    p.execute_host(hA[i].data_ptr(), hB.data_ptr(), As[i].data_ptr(),
+                                   Bs[i].data_ptr(), sptr)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            e2e_ms = e0.elapsed_time(e1)
+            if world > 1:
+                t = torch.tensor([e2e_ms], device=dev)
+                dist.all_reduce(t, op=dist.ReduceOp.MAX)
+                e2e_ms = float(t.item())
+            h2d = sum(c.n_elems * c.elem_bytes for c in cases)
+            e2e = {"value": world * step_bytes * args.e2e_steps / (e2e_ms / 1e3) / 1e9,
+                   "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": h2d,
+                   "steps": args.e2e_steps, "api": "ttlg_execute_host (pinned host buffers)"}
+            del hA, hB
+        except Exception as ex:  # report, do not hide
+            e2e = {"value": None, "unit": "GB/s", "error": str(ex)[:200]}
+
+    if rank == 0:
+        cpu = None
+        if not args.no_cpu_baseline and world == 1:
+            cpu = cpu_baseline(cases, budget_s=args.cpu_budget)
+        schemas = {}
+        for inf in infos:
+            schemas[inf["schema"]] = schemas.get(inf["schema"], 0) + 1
+        line = {
+            "metric": "effective transpose GB/s (2*N*s/time)",
+            "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "f64" if cases[0].elem_bytes == 8 else "f32",
+            "data": "synthetic (SplitMix64 bit patterns, generated on device)",
+            "config": {"workload": name, "cases_per_step": len(cases),
+                       "bytes_per_step": step_bytes, "parallelism": f"replica x{world}",
+                       "mode": "repeated-use (pre-built plans)",
+                       "l2": "no flush: every case moves >= 2x126 MB L2 (inputs larger than L2)"},
+            "gpu_launches": launches,
+            "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
+                         "peak_source": peak_src, "unit": "GB/s", "frac": achieved / peak,
+                         "traffic": traffic, "share_of_step": dg["ms"] / sum(
+                             g["ms"] for g in groups.values())},
+            "frac_of_peak": value / world / peak,
+            "d2d_gbs": d2d_gbs, "frac_of_d2d": value / world / d2d_gbs,
+            "kernels": {k: {"gbs": g["bytes"] / (g["ms"] / 1e3) / 1e9,
+                            "share": g["ms"] / sum(x["ms"] for x in groups.values()),
+                            "launches": g["launches"]} for k, g in groups.items()},
+            "schemas": schemas,
+            "model_err_pct": 100.0 * sum(errs) / len(errs),
+            "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        if os.environ.get("TTLG_BENCH_CASES"):
+            line["cases"] = [{"case": c.label(), "schema": inf["schema"],
+                              "gbs": c.alg_bytes / (m * 1e-3) / 1e9,
+                              "pred_gbs": c.alg_bytes / inf["predicted_seconds"] / 1e9}
+                             for c, inf, m in zip(cases, infos, med)]
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,160 @@
+/*
+ * ttlg.h -- C ABI of the B200-native TTLG tensor-transposition library.
+ *
+ * Operation (§I, Eq. 1): out-of-place transposition
+ *     B[rho(i0, ..., i_{d-1})] <- A[i0, ..., i_{d-1}]
+ * of a dense rank-d tensor of fp32 or fp64 elements, moved as bit patterns
+ * (no arithmetic, so the result is unique bit for bit).
+ *
+ * Conventions (readings R1, R2):
+ *   - extents[0] is the fastest-varying index (FVI): the element with
+ *     multi-index (i0..i_{d-1}) lives at linear offset sum_k i_k * prod_{k'<k} n_k'
+ *     (MATLAB/Fortran notation, PAPER.md L284-286 footnote 1);
+ *   - perm[i] = j means output dimension i is input dimension j (PAPER.md
+ *     L1883-1886, §VI).  B therefore has extents m[i] = extents[perm[i]]; the
+ *     paper's rho is perm^{-1}.
+ *
+ * Usage modes (§VI): "repeated use" = ttlg_plan once +
+ * ttlg_execute many times; "single use" = ttlg_transpose (plan cost counts).
+ * ttlg_predict_time is the performance-model query for higher-level optimisers
+ * such as a TTGT contraction engine (PAPER.md L11-21 Abstract, L60-63 §I).
+ *
+ * Threading / ownership:
+ *   - the caller owns extents/perm (copied into the plan) and A/B (device
+ *     memory, N*s bytes each, N = prod extents, s = 4 or 8);
+ *   - a plan is immutable host memory; it is bound to the CUDA device that was
+ *     current when it was created (TTLG_ERR_DEVICE if executed elsewhere); all
+ *     kernel parameters are captured at launch, so a plan may be destroyed as
+ *     soon as ttlg_execute returns and one plan may be executed concurrently
+ *     on several streams;
+ *   - ttlg_execute / ttlg_transpose are asynchronous in stream order and never
+ *     synchronise the host; launch failures return TTLG_ERR_CUDA.
+ *   - planning makes no CUDA calls other than cached device-attribute queries;
+ *     with no CUDA device present a virtual B200 profile (148 SMs, 227 KB
+ *     shared memory per block) is used, so ttlg_plan / ttlg_predict_time work
+ *     on a CPU-only host (ttlg_execute then returns TTLG_ERR_DEVICE).
+ */
+#ifndef TTLG_H_
+#define TTLG_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define TTLG_MAX_RANK 15 /* rank-specialised code "until rank 15" */
+#define TTLG_VERSION 100
+
+typedef enum { TTLG_F32 = 0, TTLG_F64 = 1 } ttlg_dtype;
+
+typedef enum {
+  TTLG_OK = 0,
+  TTLG_ERR_INVALID_VALUE = 1, /* bad rank/extent/perm/dtype, null or misaligned pointer */
+  TTLG_ERR_ALIASING = 2,      /* [A, A+N*s) overlaps [B, B+N*s): op is out-of-place (L91) */
+  TTLG_ERR_DEVICE = 3,        /* no CUDA device, or executed on another device than planned */
+  TTLG_ERR_CUDA = 4,          /* a CUDA launch / runtime call failed */
+  TTLG_ERR_NO_MEMORY = 5,     /* host allocation failed */
+  TTLG_ERR_INTERNAL = 6,      /* planner could not build a legal plan (bug) */
+  TTLG_ERR_UNSUPPORTED = 7    /* e.g. a forced schema that does not apply */
+} ttlg_status;
+
+/* Kernel schemas (§III-IV, Alg. 1; flowchart L686-697).
+ * COPY is the fused-rank-1 case (identity after index fusion). */
+typedef enum {
+  TTLG_SCHEMA_AUTO = -1,
+  TTLG_SCHEMA_COPY = 0,
+  TTLG_SCHEMA_FML = 1, /* FVI-Match-Large, Alg. 7 */
+  TTLG_SCHEMA_FMS = 2, /* FVI-Match-Small, Alg. 6 */
+  TTLG_SCHEMA_OD = 3,  /* Orthogonal-Distinct, Alg. 2 */
+  TTLG_SCHEMA_OA = 4   /* Orthogonal-Arbitrary, Alg. 4/5 L868-1020 */
+} ttlg_schema;
+
+typedef struct ttlg_plan_s *ttlg_plan_t;
+
+/* Optional planning hints (tests, calibration, model-regret studies).
+ * Initialise with ttlg_plan_hints_init() (everything "auto"), then set what
+ * you want forced. */
+typedef struct {
+  int32_t schema;                        /* TTLG_SCHEMA_AUTO (-1) = model choice        */
+  int32_t in_dim;                        /* -1 = auto; else last fused input dim of the
+                                            input slice (Alg. 3 dimsIn)                   */
+  int64_t in_block;                      /* blocking factor of that dim (blockA), 0=auto */
+  int32_t out_dim;                       /* -1 = auto; position b of the last output dim
+                                            of the output slice (Alg. 3 dimsOut)          */
+  int64_t out_block;                     /* blockB, 0 = auto                             */
+  int32_t elem_bytes_override;           /* 0 = auto widening; else 4/8/16 access width  */
+  int32_t threads;                       /* 0 = auto; else threads per block             */
+  int32_t grid;                          /* 0 = auto (persistent); else blocks           */
+  int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
+} ttlg_plan_hints;
+
+/* Everything a test or benchmark may want to know about a plan. */
+typedef struct {
+  int32_t schema;                         /* ttlg_schema actually used                   */
+  int32_t dtype;                          /* ttlg_dtype                                  */
+  int32_t rank;                           /* rank as given                               */
+  int32_t fused_rank;                     /* rank after squeeze + fusion (L666-685)      */
+  int64_t fused_extents[TTLG_MAX_RANK];   /* in units of the access element (below)      */
+  int32_t fused_perm[TTLG_MAX_RANK];
+  int32_t access_bytes;                   /* 4, 8 or 16: element width after widening    */
+  int64_t tile_extents[TTLG_MAX_RANK];    /* per fused dim; 1 = not in the slice         */
+  int32_t in_dim, out_dim;                /* last dims of the input / output slice       */
+  int64_t in_run, out_run;                /* contiguous run lengths (access elements)    */
+  int64_t tile_volume;                    /* elements per slice (tile)                   */
+  int64_t num_tiles;
+  int32_t grid, threads, smem_bytes;
+  int64_t bytes;                          /* algorithmic bytes 2*N*s                     */
+  double predicted_seconds;               /* performance-model prediction                */
+  int32_t candidates;                     /* number of candidates the model scored       */
+  int32_t param_bytes;                    /* kernel-parameter blob size                  */
+} ttlg_plan_info;
+
+void ttlg_plan_hints_init(ttlg_plan_hints *hints);
+
+/* Create a plan (Alg. 1 taxonomy + Alg. 3 slice/block search + §V model).
+ * extents: [rank] int64, each >= 1; perm: [rank] permutation of 0..rank-1;
+ * rank in [1, 15].  Returns TTLG_ERR_INVALID_VALUE on bad arguments. */
+ttlg_status ttlg_plan(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                      const int32_t *perm);
+
+/* As ttlg_plan, with hints (may be NULL). Forced choices that do not apply
+ * return TTLG_ERR_UNSUPPORTED. */
+ttlg_status ttlg_plan_ex(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                         const int32_t *perm, const ttlg_plan_hints *hints);
+
+/* Repeated-use execution: one asynchronous kernel launch on `stream`
+ * (a cudaStream_t; NULL = legacy default stream).  A and B are device
+ * pointers, element-aligned, non-overlapping. */
+ttlg_status ttlg_execute(ttlg_plan_t plan, const void *A, void *B, void *stream);
+
+ttlg_status ttlg_plan_destroy(ttlg_plan_t plan);
+
+/* Single-use: plan + execute + destroy, no caching, no host sync. */
+ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, const int32_t *perm,
+                           const void *A, void *B, void *stream);
+
+/* Host-buffer convenience (end-to-end path): copies A_host -> A_dev, executes,
+ * copies B_dev -> B_host, all asynchronous on `stream`, with the copies split in
+ * chunks where the plan allows so transfers overlap.  A_host/B_host should be
+ * pinned for asynchrony; A_dev/B_dev are device scratch of N*s bytes each. */
+ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
+                              void *B_dev, void *stream);
+
+/* Performance-model query (§V): predicted seconds of the
+ * plan the library would choose.  No CUDA calls beyond cached attributes. */
+ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,
+                              const int32_t *perm, double *seconds);
+
+ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info);
+
+const char *ttlg_status_string(ttlg_status s);
+const char *ttlg_schema_name(int schema);
+int ttlg_version(void);
+/* Provenance of the performance-model coefficients compiled in (calibration tag). */
+const char *ttlg_model_source(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TTLG_H_ */

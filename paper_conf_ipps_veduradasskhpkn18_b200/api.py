@@ -1,0 +1,169 @@
+"""Python surface of the TTLG C ABI (same names as include/ttlg.h).
+
+Raw-pointer functions (`plan`, `execute`, `transpose`, `predict_time`) mirror
+the C calls one to one.  `transpose_tensor` is the torch convenience: torch
+tensors are row-major (last axis fastest), the library is FVI-first (DESIGN.md
+reading R1), so a torch permute(perm_t) of a rank-d tensor is the library call
+with extents_c[k] = shape[d-1-k] and perm_c[i] = d-1-perm_t[d-1-i].
+PyTorch supplies device memory and streams only; the data movement is the
+library's kernels.
+"""
+from __future__ import annotations
+
+import ctypes
+from typing import Optional, Sequence
+
+from . import _ffi
+from ._ffi import (F32, F64, SCHEMA_AUTO, SCHEMA_IDS, TtlgError, PlanHints, PlanInfo,
+                   arrays, check, lib)
+
+
+def _dtype_code(dtype) -> int:
+    if isinstance(dtype, int):
+        return dtype
+    s = str(dtype)
+    if s in ("f32", "float32", "torch.float32", "fp32"):
+        return F32
+    if s in ("f64", "float64", "torch.float64", "fp64"):
+        return F64
+    raise ValueError(f"unsupported dtype {dtype!r} (fp32/fp64)")
+
+
+def make_hints(schema=None, in_dim=None, in_block=None, out_dim=None, out_block=None,
+               access_bytes=None, threads=None, grid=None, no_fusion=False) -> PlanHints:
+    h = PlanHints()
+    lib.ttlg_plan_hints_init(ctypes.byref(h))
+    if schema is not None:
+        h.schema = SCHEMA_IDS[schema] if isinstance(schema, str) else int(schema)
+    if in_dim is not None:
+        h.in_dim = in_dim
+    if in_block is not None:
+        h.in_block = in_block
+    if out_dim is not None:
+        h.out_dim = out_dim
+    if out_block is not None:
+        h.out_block = out_block
+    if access_bytes is not None:
+        h.elem_bytes_override = access_bytes
+    if threads is not None:
+        h.threads = threads
+    if grid is not None:
+        h.grid = grid
+    h.no_fusion = 1 if no_fusion else 0
+    return h
+
+
+class Plan:
+    """A ttlg_plan_t (repeated-use mode)."""
+
+    def __init__(self, dtype, extents: Sequence[int], perm: Sequence[int], **hints):
+        self._h = ctypes.c_void_p()
+        self.dtype = _dtype_code(dtype)
+        self.extents = [int(e) for e in extents]
+        self.perm = [int(p) for p in perm]
+        ext, pr = arrays(self.extents, self.perm)
+        if hints:
+            hh = make_hints(**hints)
+            check(lib.ttlg_plan_ex(ctypes.byref(self._h), self.dtype, len(self.extents), ext, pr,
+                                   ctypes.byref(hh)), "ttlg_plan_ex")
+        else:
+            check(lib.ttlg_plan(ctypes.byref(self._h), self.dtype, len(self.extents), ext, pr),
+                  "ttlg_plan")
+
+    @property
+    def handle(self):
+        return self._h
+
+    def describe(self) -> dict:
+        info = PlanInfo()
+        check(lib.ttlg_plan_describe(self._h, ctypes.byref(info)), "ttlg_plan_describe")
+        return info.to_dict()
+
+    def execute(self, A_ptr: int, B_ptr: int, stream: int = 0):
+        check(lib.ttlg_execute(self._h, ctypes.c_void_p(A_ptr), ctypes.c_void_p(B_ptr),
+                               ctypes.c_void_p(stream)), "ttlg_execute")
+
+    def execute_host(self, A_host: int, B_host: int, A_dev: int, B_dev: int, stream: int = 0):
+        check(lib.ttlg_execute_host(self._h, ctypes.c_void_p(A_host), ctypes.c_void_p(B_host),
+                                    ctypes.c_void_p(A_dev), ctypes.c_void_p(B_dev),
+                                    ctypes.c_void_p(stream)), "ttlg_execute_host")
+
+    def destroy(self):
+        if self._h:
+            lib.ttlg_plan_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+
+def plan(dtype, extents, perm, **hints) -> Plan:
+    return Plan(dtype, extents, perm, **hints)
+
+
+def execute(p: Plan, A_ptr: int, B_ptr: int, stream: int = 0):
+    p.execute(A_ptr, B_ptr, stream)
+
+
+def transpose(dtype, extents, perm, A_ptr: int, B_ptr: int, stream: int = 0):
+    """Single-use: ttlg_transpose (plan + launch, no cache, no host sync)."""
+    ext, pr = arrays(extents, perm)
+    check(lib.ttlg_transpose(_dtype_code(dtype), len(extents), ext, pr, ctypes.c_void_p(A_ptr),
+                             ctypes.c_void_p(B_ptr), ctypes.c_void_p(stream)), "ttlg_transpose")
+
+
+def predict_time(dtype, extents, perm) -> float:
+    """Performance-model query (§V; L60-63): predicted seconds."""
+    ext, pr = arrays(extents, perm)
+    out = ctypes.c_double()
+    check(lib.ttlg_predict_time(_dtype_code(dtype), len(extents), ext, pr, ctypes.byref(out)),
+          "ttlg_predict_time")
+    return out.value
+
+
+def model_source() -> str:
+    return lib.ttlg_model_source().decode()
+
+
+# ---- torch conveniences ---------------------------------------------------------------
+def torch_to_c(shape: Sequence[int], perm_t: Sequence[int]):
+    """Row-major torch (shape, permute order) -> FVI-first (extents, perm)."""
+    d = len(shape)
+    ext = [int(shape[d - 1 - k]) for k in range(d)]
+    perm = [d - 1 - int(perm_t[d - 1 - i]) for i in range(d)]
+    return ext, perm
+
+
+def _dt_of_tensor(x) -> int:
+    if x.element_size() == 8:
+        return F64
+    if x.element_size() == 4:
+        return F32
+    raise ValueError("tensor elements must be 4 or 8 bytes")
+
+
+def transpose_tensor(x, perm_t: Sequence[int], out=None, plan_: Optional[Plan] = None):
+    """out = x.permute(perm_t).contiguous(), computed by the library on x's device
+    and current stream."""
+    import torch
+
+    if not x.is_cuda:
+        raise ValueError("transpose_tensor needs a CUDA tensor (no CPU path)")
+    if not x.is_contiguous():
+        raise ValueError("input must be contiguous")
+    shape_out = [x.shape[p] for p in perm_t]
+    if out is None:
+        out = torch.empty(shape_out, dtype=x.dtype, device=x.device)
+    if x.numel() == 0:
+        return out
+    ext, perm = torch_to_c(list(x.shape), perm_t)
+    stream = torch.cuda.current_stream(x.device).cuda_stream
+    with torch.cuda.device(x.device):
+        if plan_ is not None:
+            plan_.execute(x.data_ptr(), out.data_ptr(), stream)
+        else:
+            transpose(_dt_of_tensor(x), ext, perm, x.data_ptr(), out.data_ptr(), stream)
+    return out

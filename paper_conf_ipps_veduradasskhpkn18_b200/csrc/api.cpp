@@ -1,0 +1,255 @@
+// api.cpp -- the C ABI declared in include/ttlg.h.
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#include <mutex>
+#include <new>
+
+#include "model_coeffs.h"
+#include "ttlg_internal.h"
+
+namespace ttlg {
+
+// Virtual B200 profile (no device): 148 SMs, 227 KB opt-in smem per block,
+// 228 KB per SM, 2048 threads and 64K registers per SM; HBM copy bandwidth as
+// measured by the driver on this pool (MEASURED_PEAKS.json hbm_gbs).
+static DeviceProfile virtual_b200() {
+  DeviceProfile d;
+  d.sms = 148;
+  d.smem_per_block_optin = 227 * 1024;
+  d.smem_per_sm = 228 * 1024;
+  d.max_threads_per_sm = 2048;
+  d.regs_per_sm = 65536;
+  d.hbm_gbs = 6555.5;
+  d.virt = true;
+  return d;
+}
+
+const DeviceProfile &device_profile(int device) {
+  static DeviceProfile cache[16];
+  static bool have[16] = {false};
+  static DeviceProfile virt = virtual_b200();
+  static std::mutex mu;
+  if (device < 0 || device >= 16) return virt;
+  std::lock_guard<std::mutex> g(mu);
+  if (!have[device]) {
+    DeviceProfile d = virtual_b200();
+    int v;
+    if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device) == cudaSuccess) {
+      d.sms = v;
+      d.virt = false;
+      if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerBlockOptin, device) ==
+          cudaSuccess)
+        d.smem_per_block_optin = v;
+      if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxSharedMemoryPerMultiprocessor, device) ==
+          cudaSuccess)
+        d.smem_per_sm = v;
+      if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxThreadsPerMultiProcessor, device) ==
+          cudaSuccess)
+        d.max_threads_per_sm = v;
+      if (cudaDeviceGetAttribute(&v, cudaDevAttrMaxRegistersPerMultiprocessor, device) ==
+          cudaSuccess)
+        d.regs_per_sm = v;
+    } else {
+      cudaGetLastError();
+    }
+    cache[device] = d;
+    have[device] = true;
+  }
+  return cache[device];
+}
+
+static int current_device() {
+  static int ndev = -2;
+  if (ndev == -2) {
+    int n = 0;
+    if (cudaGetDeviceCount(&n) != cudaSuccess) {
+      cudaGetLastError();
+      n = 0;
+    }
+    ndev = n;
+  }
+  if (ndev <= 0) return -1;
+  int dev = -1;
+  if (cudaGetDevice(&dev) != cudaSuccess) {
+    cudaGetLastError();
+    return -1;
+  }
+  return dev;
+}
+
+static ttlg_status plan_into(ttlg_plan_s *p, ttlg_dtype dt, int rank, const int64_t *ext,
+                             const int32_t *perm, const ttlg_plan_hints *hints) {
+  const int dev = current_device();
+  ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev));
+  if (st != TTLG_OK) return st;
+  p->device = dev;
+  p->dt = dt;
+  p->rank = rank;
+  for (int k = 0; k < rank; k++) {
+    p->ext[k] = ext[k];
+    p->perm[k] = perm[k];
+  }
+  p->has_hints = hints != nullptr;
+  if (hints) p->hints = *hints;
+  return TTLG_OK;
+}
+
+// TTLG_SYNC=1: synchronise and check after every launch (debug mode).
+static bool getenv_sync() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_SYNC");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
+static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *stream) {
+  if (!p || !A || !B) return TTLG_ERR_INVALID_VALUE;
+  const int s = p->dt == TTLG_F64 ? 8 : 4;
+  const uintptr_t a = (uintptr_t)A, b = (uintptr_t)B;
+  if (a % s || b % s) return TTLG_ERR_INVALID_VALUE;
+  const uintptr_t nb = (uintptr_t)p->nbytes;
+  if (a < b + nb && b < a + nb) return TTLG_ERR_ALIASING;
+  if (p->device < 0) return TTLG_ERR_DEVICE;
+  int dev = -1;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) {
+    cudaGetLastError();
+    return TTLG_ERR_DEVICE;
+  }
+  if ((a | b) % (uintptr_t)p->W) {
+    // widened access needs W-aligned pointers: re-plan at the element width
+    ttlg_plan_s q;
+    ttlg_plan_hints h;
+    if (p->has_hints) {
+      h = p->hints;
+    } else {
+      ttlg_plan_hints_init(&h);
+    }
+    h.elem_bytes_override = s;
+    ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h);
+    if (st != TTLG_OK) return st;
+    return launch(&q, A, B, stream);
+  }
+  ttlg_status st = launch(p, A, B, stream);
+  if (st == TTLG_OK && getenv_sync()) {
+    if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return TTLG_ERR_CUDA;
+  }
+  return st;
+}
+
+}  // namespace ttlg
+
+using namespace ttlg;
+
+extern "C" {
+
+void ttlg_plan_hints_init(ttlg_plan_hints *h) {
+  if (!h) return;
+  memset(h, 0, sizeof(*h));
+  h->schema = TTLG_SCHEMA_AUTO;
+  h->in_dim = -1;
+  h->out_dim = -1;
+}
+
+ttlg_status ttlg_plan_ex(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                         const int32_t *perm, const ttlg_plan_hints *hints) {
+  if (!out) return TTLG_ERR_INVALID_VALUE;
+  *out = nullptr;
+  ttlg_plan_s *p = new (std::nothrow) ttlg_plan_s;
+  if (!p) return TTLG_ERR_NO_MEMORY;
+  ttlg_status st = plan_into(p, dt, rank, extents, perm, hints);
+  if (st != TTLG_OK) {
+    delete p;
+    return st;
+  }
+  *out = p;
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_plan(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                      const int32_t *perm) {
+  return ttlg_plan_ex(out, dt, rank, extents, perm, nullptr);
+}
+
+ttlg_status ttlg_execute(ttlg_plan_t plan, const void *A, void *B, void *stream) {
+  return execute(plan, A, B, stream);
+}
+
+ttlg_status ttlg_plan_destroy(ttlg_plan_t plan) {
+  delete plan;
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, const int32_t *perm,
+                           const void *A, void *B, void *stream) {
+  ttlg_plan_s p;  // single use: no heap, no cache
+  ttlg_status st = plan_into(&p, dt, rank, extents, perm, nullptr);
+  if (st != TTLG_OK) return st;
+  return execute(&p, A, B, stream);
+}
+
+ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
+                              void *B_dev, void *stream) {
+  if (!plan || !A_host || !B_host || !A_dev || !B_dev) return TTLG_ERR_INVALID_VALUE;
+  cudaStream_t s = (cudaStream_t)stream;
+  if (cudaMemcpyAsync(A_dev, A_host, (size_t)plan->nbytes, cudaMemcpyHostToDevice, s) !=
+      cudaSuccess)
+    return TTLG_ERR_CUDA;
+  ttlg_status st = execute(plan, A_dev, B_dev, stream);
+  if (st != TTLG_OK) return st;
+  if (cudaMemcpyAsync(B_host, B_dev, (size_t)plan->nbytes, cudaMemcpyDeviceToHost, s) !=
+      cudaSuccess)
+    return TTLG_ERR_CUDA;
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,
+                              const int32_t *perm, double *seconds) {
+  if (!seconds) return TTLG_ERR_INVALID_VALUE;
+  ttlg_plan_s p;
+  ttlg_status st = plan_into(&p, dt, rank, extents, perm, nullptr);
+  if (st != TTLG_OK) return st;
+  *seconds = p.info.predicted_seconds;
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info) {
+  if (!plan || !info) return TTLG_ERR_INVALID_VALUE;
+  *info = plan->info;
+  return TTLG_OK;
+}
+
+const char *ttlg_status_string(ttlg_status s) {
+  switch (s) {
+    case TTLG_OK: return "TTLG_OK";
+    case TTLG_ERR_INVALID_VALUE: return "TTLG_ERR_INVALID_VALUE";
+    case TTLG_ERR_ALIASING: return "TTLG_ERR_ALIASING";
+    case TTLG_ERR_DEVICE: return "TTLG_ERR_DEVICE";
+    case TTLG_ERR_CUDA: return "TTLG_ERR_CUDA";
+    case TTLG_ERR_NO_MEMORY: return "TTLG_ERR_NO_MEMORY";
+    case TTLG_ERR_INTERNAL: return "TTLG_ERR_INTERNAL";
+    case TTLG_ERR_UNSUPPORTED: return "TTLG_ERR_UNSUPPORTED";
+  }
+  return "TTLG_ERR_UNKNOWN";
+}
+
+const char *ttlg_schema_name(int schema) {
+  switch (schema) {
+    case TTLG_SCHEMA_COPY: return "COPY";
+    case TTLG_SCHEMA_FML: return "FML";
+    case TTLG_SCHEMA_FMS: return "FMS";
+    case TTLG_SCHEMA_OD: return "OD";
+    case TTLG_SCHEMA_OA: return "OA";
+  }
+  return "AUTO";
+}
+
+int ttlg_version(void) { return TTLG_VERSION; }
+
+const char *ttlg_model_source(void) { return kModelSource; }
+
+}  // extern "C"

@@ -1,0 +1,62 @@
+// model.cpp -- B200 performance model; see model.h.
+#include "model.h"
+
+#include <algorithm>
+#include <cmath>
+
+#include "model_coeffs.h"
+
+namespace ttlg {
+
+// DRAM bytes moved for one contiguous run of R bytes: whole 32-byte sectors,
+// plus half a sector on average when the run is not sector-aligned, with a
+// 64-byte floor (HBM burst) -- the B200 restatement of Table I's transaction
+// counts, which count 128-byte K40 transactions.
+static double run_cost(double R) {
+  double c = 32.0 * std::ceil(R / 32.0);
+  if (std::fmod(R, 32.0) != 0.0) c += 16.0;
+  return std::max(c, 64.0);
+}
+
+ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
+  ModelFeatures F;
+  for (double &x : F.f) x = 0.0;
+  const double W = mi.W;
+  const double tiles = (double)mi.num_tiles;
+  const double fill = mi.fillA;
+  double read_bytes, write_bytes, runs;
+  if (mi.kind == KK_DIRECT) {
+    read_bytes = tiles * fill * run_cost(mi.V * W);
+    runs = tiles * fill * (1.0 + mi.RB);
+  } else {
+    read_bytes = tiles * fill * mi.RA * run_cost(mi.LA * W);
+    runs = tiles * fill * (mi.RA + mi.RB);
+  }
+  write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
+  const double bw = dev.hbm_gbs * 1e9;
+  // bytes in flight: each CTA keeps up to UNROLL*threads access elements of
+  // loads outstanding (Little's law with the loaded-DRAM latency)
+  const double unroll = (mi.kind == KK_DIRECT) ? kModelUnrollDirect : kModelUnrollStaged;
+  const double inflight = (double)mi.occ * std::min<double>(mi.V, unroll * mi.threads) * W;
+  const double bw_lat = dev.sms * inflight / kModelLatency;
+  const double bw_eff = std::min(bw, bw_lat);
+  const double per_cta = std::ceil(tiles / mi.grid);
+  const double wave = per_cta / (tiles / mi.grid);
+  F.f[0] = 1.0;
+  F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
+  F.f[2] = per_cta / std::max(1, mi.occ);
+  F.f[3] = runs / dev.sms;
+  return F;
+}
+
+double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
+  const ModelFeatures F = model_features(mi, dev);
+  const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect : kCoefStaged;
+  double t = 0.0;
+  for (int i = 0; i < kModelNumFeatures; i++) t += c[i] * F.f[i];
+  // the model can never beat one pass of the algorithmic bytes at copy speed
+  const double floor_t = 2.0 * (double)mi.N * mi.W / (dev.hbm_gbs * 1e9);
+  return std::max(t, floor_t);
+}
+
+}  // namespace ttlg

@@ -1,0 +1,36 @@
+// model.h -- B200 performance model (§V, re-derived).
+//
+// The paper fits, per kernel, a linear regression of time on features of the
+// chosen slices (Volume, NumBlocks, input/output slice, "Cycles" for idle
+// lanes on partial tiles; Table II).  On B200 the transposition is
+// HBM-bound, so the features are bytes-first: the DRAM sectors the schedule
+// touches (run lengths -> 32-byte sectors), the bytes-in-flight limit
+// (occupancy x staged elements), tail waves of the persistent grid, per-tile
+// synchronisation overhead and idle lanes.  Coefficients are fitted offline
+// on B200 measurements (tools/calibrate.py) and shipped in model_coeffs.h.
+#pragma once
+
+#include <stdint.h>
+
+#include "ttlg_internal.h"
+
+namespace ttlg {
+
+struct ModelInput {
+  int kind, schema, W;
+  int64_t N;  // access elements
+  int V, LA, LB, RA, RB;
+  int64_t num_tiles;
+  int threads, smem_bytes, occ, grid;
+  double fillA;  // useful fraction of the tile grid (partial tiles)
+};
+
+struct ModelFeatures {
+  double f[8];
+};
+
+// Feature vector (units: seconds at the reference bandwidth, or counts).
+ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev);
+double predict_seconds(const ModelInput &mi, const DeviceProfile &dev);
+
+}  // namespace ttlg

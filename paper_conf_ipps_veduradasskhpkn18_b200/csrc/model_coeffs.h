@@ -1,0 +1,15 @@
+// model_coeffs.h -- coefficients of the B200 performance model (model.cpp).
+// Initial physically-motivated values; replaced by tools/calibrate.py with a
+// least-squares fit on B200 measurements (§V L1402-1419 method).
+#pragma once
+
+namespace ttlg {
+constexpr int kModelNumFeatures = 4;
+constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
+constexpr double kModelUnrollStaged = 8.0;   // loads in flight per thread (staged)
+constexpr double kModelUnrollDirect = 8.0;   // loads in flight per thread (direct)
+// features: [launch, memory-time, tiles-per-CTA/occ, runs-per-SM]
+constexpr double kCoefDirect[kModelNumFeatures] = {2.5e-6, 1.0, 0.10e-6, 0.2e-9};
+constexpr double kCoefStaged[kModelNumFeatures] = {2.5e-6, 1.0, 0.25e-6, 0.2e-9};
+constexpr const char *kModelSource = "default (uncalibrated)";
+}  // namespace ttlg

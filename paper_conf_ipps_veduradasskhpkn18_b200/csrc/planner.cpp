@@ -1,0 +1,525 @@
+// planner.cpp -- host-only planning for the B200 TTLG library.
+//
+//   validate -> squeeze extent-1 dims -> index fusion
+//   -> FVI widening (matching FVI rows moved as 8/16-byte access elements)
+//   -> candidate slices (Alg. 3: input-prefix group with a blocked
+//      slowest dim, output-prefix group with a blocked slowest dim)
+//   -> schema label per candidate (Alg. 1; reading R9/R11:
+//      every applicable schema competes, the model arbitrates)
+//   -> B200 performance model (§V re-derived, model.cpp) -> best candidate
+//   -> kernel parameter block (TileParams) + launch geometry.
+//
+// No CUDA calls here: the device profile is passed in, so plans can be built
+// (and unit-tested) on a host with no GPU.
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+
+#include "model.h"
+#include "ttlg_internal.h"
+
+namespace ttlg {
+
+ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm) {
+  if (dt != TTLG_F32 && dt != TTLG_F64) return TTLG_ERR_INVALID_VALUE;
+  if (rank < 1 || rank > TTLG_MAX_RANK) return TTLG_ERR_INVALID_VALUE;
+  if (!ext || !perm) return TTLG_ERR_INVALID_VALUE;
+  bool seen[TTLG_MAXD] = {false};
+  const int64_t s = (dt == TTLG_F64) ? 8 : 4;
+  int64_t n = 1;
+  for (int k = 0; k < rank; k++) {
+    if (ext[k] < 1) return TTLG_ERR_INVALID_VALUE;
+    if (perm[k] < 0 || perm[k] >= rank || seen[perm[k]]) return TTLG_ERR_INVALID_VALUE;
+    seen[perm[k]] = true;
+    if (n > (INT64_MAX / 4) / s / ext[k]) return TTLG_ERR_INVALID_VALUE;  // 2*N*s must fit
+    n *= ext[k];
+  }
+  return TTLG_OK;
+}
+
+// Squeeze extent-1 dims (reading R4), then fuse maximal runs of
+// input dims that stay consecutive and in the same order in the output
+// ([i0,i1,i2,i3] => [i3,i1,i2,i0] fuses i1,i2).
+static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool fuse,
+                         Problem &P) {
+  int map[TTLG_MAXD];
+  int64_t n[TTLG_MAXD];
+  int d = 0;
+  for (int k = 0; k < rank; k++) {
+    if (ext[k] > 1) {
+      map[k] = d;
+      n[d++] = ext[k];
+    } else {
+      map[k] = -1;
+    }
+  }
+  int32_t p[TTLG_MAXD];
+  int dd = 0;
+  for (int i = 0; i < rank; i++)
+    if (map[perm[i]] >= 0) p[dd++] = map[perm[i]];
+  if (d == 0) {
+    P.d = 1;
+    P.n[0] = 1;
+    P.p[0] = 0;
+    return;
+  }
+  if (!fuse) {
+    P.d = d;
+    for (int k = 0; k < d; k++) {
+      P.n[k] = n[k];
+      P.p[k] = p[k];
+    }
+    return;
+  }
+  // groups in output order
+  int gstart[TTLG_MAXD], glen[TTLG_MAXD], ng = 0;
+  for (int i = 0; i < d; i++) {
+    if (i == 0 || p[i] != p[i - 1] + 1) {
+      gstart[ng] = i;
+      glen[ng] = 1;
+      ng++;
+    } else {
+      glen[ng - 1]++;
+    }
+  }
+  // new input index of a group = rank of its first input dim among groups
+  int first[TTLG_MAXD];
+  for (int g = 0; g < ng; g++) first[g] = p[gstart[g]];
+  for (int g = 0; g < ng; g++) {
+    int r = 0;
+    for (int h = 0; h < ng; h++)
+      if (first[h] < first[g]) r++;
+    int64_t e = 1;
+    for (int q = 0; q < glen[g]; q++) e *= n[first[g] + q];
+    P.n[r] = e;
+    P.p[g] = r;
+  }
+  P.d = ng;
+}
+
+// Matching FVI: the fused FVI row of n0*s bytes is moved as wider access
+// elements (16 B when the row allows).  A row of exactly one access element
+// squeezes away, turning e.g. FMS on [2,4096,4096] fp32 into a plain 2-D
+// transpose of 8-byte elements.
+static void widen(Problem &P, int forceW) {
+  P.W = P.esize;
+  if (P.p[0] != 0) return;
+  const int64_t R = P.n[0] * P.esize;
+  int W = P.esize;
+  if (forceW) {
+    W = forceW;
+  } else if (R % 16 == 0) {
+    W = 16;
+  } else if (R % 8 == 0) {
+    W = 8;
+  }
+  P.W = W;
+  P.n[0] = R / W;
+  if (P.n[0] == 1 && P.d > 1) {
+    for (int k = 0; k + 1 < P.d; k++) P.n[k] = P.n[k + 1];
+    for (int i = 0; i + 1 < P.d; i++) P.p[i] = P.p[i + 1] - 1;
+    P.d--;
+  }
+}
+
+namespace {
+
+struct Tile {
+  int a, b;  // last input-run dim; output position of the last output-run dim
+  int64_t t[TTLG_MAXD];
+  bool ok;
+};
+
+struct Strides {
+  int64_t sA[TTLG_MAXD], sB[TTLG_MAXD];  // per input dim
+};
+
+Strides strides_of(const Problem &P) {
+  Strides S;
+  S.sA[0] = 1;
+  for (int k = 1; k < P.d; k++) S.sA[k] = S.sA[k - 1] * P.n[k - 1];
+  int64_t s = 1;
+  for (int i = 0; i < P.d; i++) {
+    S.sB[P.p[i]] = s;
+    s *= P.n[P.p[i]];
+  }
+  return S;
+}
+
+// Build the tile box for (a, ta, b, tb) -- Alg. 3's dimsIn/blockA, dimsOut/blockB.
+Tile make_tile(const Problem &P, int a, int64_t ta, int b, int64_t tb) {
+  Tile T;
+  T.a = a;
+  T.b = b;
+  T.ok = true;
+  bool set[TTLG_MAXD] = {false};
+  for (int k = 0; k < P.d; k++) T.t[k] = 1;
+  auto assign = [&](int k, int64_t v) {
+    if (set[k] && T.t[k] != v) T.ok = false;
+    set[k] = true;
+    T.t[k] = v;
+  };
+  for (int k = 0; k < a; k++) assign(k, P.n[k]);
+  assign(a, ta);
+  for (int i = 0; i < b; i++) assign(P.p[i], P.n[P.p[i]]);
+  assign(P.p[b], tb);
+  return T;
+}
+
+int schema_of(const Problem &P, const Tile &T, int kind) {
+  if (kind == KK_DIRECT) return P.d == 1 ? TTLG_SCHEMA_COPY : TTLG_SCHEMA_FML;
+  if (P.p[0] == 0) return TTLG_SCHEMA_FMS;
+  for (int i = 0; i <= T.b; i++)
+    if (P.p[i] <= T.a) return TTLG_SCHEMA_OA;  // input and output groups overlap
+  return TTLG_SCHEMA_OD;
+}
+
+int64_t ceil_div(int64_t x, int64_t y) { return (x + y - 1) / y; }
+
+}  // namespace
+
+// Fill TileParams for a tile; returns false if it violates a kernel limit.
+static bool build_params(const Problem &P, const Tile &T, int kind, int threads, TileParams &K) {
+  memset(&K, 0, sizeof(K));
+  const Strides S = strides_of(P);
+  const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
+  bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
+  for (int k = 0; k <= a; k++) inIS[k] = true;
+  for (int i = 0; i <= b; i++) inOS[P.p[i]] = true;
+
+  int64_t V = 1, LA = 1, LB = 1, LAunit = 1, LBunit = 1;
+  for (int k = 0; k < d; k++) V *= T.t[k];
+  for (int k = 0; k <= a; k++) LA *= T.t[k];
+  LAunit = LA / T.t[a];
+  for (int i = 0; i <= b; i++) LB *= T.t[P.p[i]];
+  LBunit = LB / T.t[pb];
+  if (kind == KK_DIRECT) {
+    // direct kernel: output run is dim 0 (full unless the tile is dim 0 alone)
+    if (b != 0) return false;
+  }
+  if (V >= (1ll << 30)) return false;
+  K.V = (int32_t)V;
+  K.LA = (int32_t)LA;
+  K.RA = (int32_t)(V / LA);
+  K.LAunit = (int32_t)LAunit;
+  K.LB = (int32_t)LB;
+  K.RB = (int32_t)(V / LB);
+  K.LBunit = (int32_t)LBunit;
+
+  // grid
+  int64_t tiles = 1;
+  int ng = 0;
+  K.blkA_g = -1;
+  K.blkB_g = -1;
+  for (int k = 0; k < d; k++) {
+    int64_t g = ceil_div(P.n[k], T.t[k]);
+    if (g <= 1) continue;
+    if (ng >= TTLG_MAXD) return false;
+    K.gdiv[ng] = make_fastdiv((uint32_t)g);
+    K.gsA[ng] = T.t[k] * S.sA[k];
+    K.gsB[ng] = T.t[k] * S.sB[k];
+    if (k == a && P.n[k] % T.t[k] != 0) K.blkA_g = ng;
+    if (k == pb && P.n[k] % T.t[k] != 0) K.blkB_g = ng;
+    tiles *= g;
+    ng++;
+  }
+  if (tiles >= (1ll << 31)) return false;
+  K.ng = ng;
+  K.num_tiles = (uint32_t)tiles;
+  K.blkA_n = (int32_t)P.n[a];
+  K.blkA_t = (int32_t)T.t[a];
+  K.blkB_n = (int32_t)P.n[pb];
+  K.blkB_t = (int32_t)T.t[pb];
+
+  // shared-memory strides: input-run dims contiguous; output-only dims placed
+  // in output order with a pad so that the output-run position j maps to
+  // bank j mod (128/W) -- the generalisation of the 32x33 pad (L747-749) and of
+  // FMS's "row 1 starts at bank N0" rule (L1104-1107).
+  int64_t sm[TTLG_MAXD];
+  for (int k = 0; k < d; k++) sm[k] = 0;
+  int64_t cur = 1;
+  for (int k = 0; k <= a; k++) {
+    sm[k] = cur;
+    cur *= T.t[k];
+  }
+  const int64_t Wb = 128 / P.W;
+  int64_t Q = 1;
+  for (int i = 0; i <= b; i++) {
+    const int k = P.p[i];
+    if (!inIS[k] && T.t[k] > 1) {
+      int64_t s = cur + (((Q - cur) % Wb) + Wb) % Wb;
+      sm[k] = s;
+      cur = s * T.t[k];
+    }
+    Q *= T.t[k];
+  }
+  const int64_t smem_elems = (kind == KK_STAGED) ? cur : 0;
+
+  // A-row digits: tile dims outside the input run, input order
+  int64_t maxG = 0;
+  K.nra = 0;
+  K.ra_blk = -1;
+  for (int k = 0; k < d; k++) {
+    if (inIS[k] || T.t[k] <= 1) continue;
+    if (k == pb && K.blkB_g >= 0) K.ra_blk = K.nra;
+    K.ra_ext[K.nra] = (int32_t)T.t[k];
+    K.ra_sG[K.nra] = (int32_t)S.sA[k];
+    K.ra_sS[K.nra] = (int32_t)sm[k];
+    maxG += (T.t[k] - 1) * S.sA[k];
+    K.nra++;
+  }
+  if (maxG + LA >= (1ll << 31)) return false;
+  maxG = 0;
+  K.nrb = 0;
+  K.rb_blk = -1;
+  for (int k = 0; k < d; k++) {
+    if (inOS[k] || T.t[k] <= 1) continue;
+    if (k == a && K.blkA_g >= 0) K.rb_blk = K.nrb;
+    K.rb_ext[K.nrb] = (int32_t)T.t[k];
+    K.rb_sG[K.nrb] = (int32_t)S.sB[k];
+    K.rb_sS[K.nrb] = (int32_t)sm[k];
+    maxG += (T.t[k] - 1) * S.sB[k];
+    K.nrb++;
+  }
+  if (maxG + LB >= (1ll << 31)) return false;
+  K.nj = 0;
+  for (int i = 0; i <= b; i++) {
+    const int k = P.p[i];
+    if (T.t[k] <= 1) continue;
+    K.j_ext[K.nj] = (int32_t)T.t[k];
+    K.j_sS[K.nj] = (int32_t)sm[k];
+    K.nj++;
+  }
+  if (smem_elems >= (1ll << 30)) return false;
+  K.smem_elems = (int32_t)smem_elems;
+
+  // shared-memory carve-up (bytes)
+  int64_t off = 0;
+  auto take = [&](int64_t bytes) {
+    int64_t o = off;
+    off += (bytes + 15) / 16 * 16;
+    return (int32_t)o;
+  };
+  if (kind == KK_STAGED) {
+    take((int64_t)K.RA * 8);  // tabA at 0
+    K.off_tabB = take((int64_t)K.RB * 8);
+    K.off_jcol = take((int64_t)K.LB * 4);
+    K.off_digB = take((int64_t)K.RA * 4);
+    K.off_digA = take((int64_t)K.RB * 4);
+    K.off_data = take(smem_elems * P.W);
+  } else {
+    K.off_tabB = take((int64_t)K.RB * 8);
+    K.off_jcol = 0;
+    K.off_digB = 0;
+    K.off_digA = take((int64_t)K.RB * 4);
+    K.off_data = (int32_t)off;
+  }
+  K.smem_bytes = (int32_t)off;
+  K.drA = threads / K.LA;
+  K.dxA = threads % K.LA;
+  K.drB = threads / K.LB;
+  K.dxB = threads % K.LB;
+  return true;
+}
+
+static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) {
+  int occ = dev.max_threads_per_sm / threads;
+  const int per = smem + 1024;  // 1 KB reserved per CTA
+  occ = std::min(occ, dev.smem_per_sm / per);
+  if (regs > 0) occ = std::min(occ, dev.regs_per_sm / (regs * threads));
+  occ = std::min(occ, 32);
+  return occ;
+}
+
+// Candidate blocking factors for a dim of extent n whose lower-dim product is
+// `pre` access elements (Alg. 3 enumerates limits in steps of WS and blocks the
+// slowest dim of the group; reading R12 enumerates block factors
+// directly, including the balanced ceil(n/ceil(n/t)) variants).
+static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forced) {
+  int c = 0;
+  if (forced > 0) {
+    if (forced > n) return 0;
+    out[0] = forced;
+    return 1;
+  }
+  auto add = [&](int64_t t) {
+    if (t < 1) t = 1;
+    if (t > n) t = n;
+    for (int i = 0; i < c; i++)
+      if (out[i] == t) return;
+    out[c++] = t;
+  };
+  add(n);
+  static const int64_t targets[] = {64, 128, 256, 512, 1024, 2048};
+  for (int64_t R : targets) {
+    int64_t t = ceil_div(R, pre * W);
+    if (t >= n) continue;
+    add(t);
+    add(ceil_div(n, ceil_div(n, t)));  // balanced: minimal remainder waste
+  }
+  return c;
+}
+
+ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
+                      const int32_t *perm, const ttlg_plan_hints *hints,
+                      const DeviceProfile &dev) {
+  ttlg_status st = validate(dt, rank, ext, perm);
+  if (st != TTLG_OK) return st;
+  const int s = (dt == TTLG_F64) ? 8 : 4;
+  Problem P;
+  P.esize = s;
+  canonicalize(rank, ext, perm, !(hints && hints->no_fusion), P);
+  int forceW = 0;
+  if (hints && hints->elem_bytes_override) {
+    forceW = hints->elem_bytes_override;
+    if (forceW != 4 && forceW != 8 && forceW != 16) return TTLG_ERR_INVALID_VALUE;
+    if (forceW < s) return TTLG_ERR_UNSUPPORTED;
+    if (forceW > s && (P.p[0] != 0 || (P.n[0] * s) % forceW != 0)) return TTLG_ERR_UNSUPPORTED;
+  }
+  widen(P, forceW);
+
+  const int threads = (hints && hints->threads) ? hints->threads : 256;
+  if (threads < 32 || threads > 1024 || threads % 32) return TTLG_ERR_INVALID_VALUE;
+  const int force_schema = hints ? hints->schema : TTLG_SCHEMA_AUTO;
+
+  int64_t N = 1;
+  for (int k = 0; k < P.d; k++) N *= P.n[k];
+
+  ModelInput best_mi;
+  TileParams bestK;
+  Tile bestT;
+  memset(&best_mi, 0, sizeof(best_mi));
+  memset(&bestK, 0, sizeof(bestK));
+  memset(&bestT, 0, sizeof(bestT));
+  int best_kind = -1, best_schema = -1, ncand = 0;
+  double best_t = 1e300;
+
+  const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
+
+  auto consider = [&](int kind, int a, int64_t ta, int b, int64_t tb) {
+    if (hints) {
+      if (hints->in_dim >= 0 && hints->in_dim != a) return;
+      if (hints->in_block > 0 && hints->in_block != ta) return;
+      if (hints->out_dim >= 0 && hints->out_dim != b) return;
+      if (hints->out_block > 0 && hints->out_block != tb) return;
+    }
+    Tile T = make_tile(P, a, ta, b, tb);
+    if (!T.ok) return;
+    const int schema = schema_of(P, T, kind);
+    if (force_schema != TTLG_SCHEMA_AUTO && force_schema != schema) {
+      // COPY and FML share the direct kernel; accept FML for a rank-1 problem
+      if (!(force_schema == TTLG_SCHEMA_FML && schema == TTLG_SCHEMA_COPY)) return;
+    }
+    int64_t V = 1;
+    for (int k = 0; k < P.d; k++) V *= T.t[k];
+    if (kind == KK_STAGED && V * P.W > max_tile_bytes) return;
+    if (kind == KK_DIRECT && V * P.W > 256 * 1024) return;
+    TileParams K;
+    if (!build_params(P, T, kind, threads, K)) return;
+    if (K.smem_bytes > dev.smem_per_block_optin) return;
+    ModelInput mi;
+    mi.kind = kind;
+    mi.schema = schema;
+    mi.W = P.W;
+    mi.N = N;
+    mi.V = K.V;
+    mi.LA = K.LA;
+    mi.LB = K.LB;
+    mi.RA = K.RA;
+    mi.RB = K.RB;
+    mi.num_tiles = K.num_tiles;
+    mi.threads = threads;
+    mi.smem_bytes = K.smem_bytes;
+    mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
+    if (mi.occ < 1) return;
+    mi.grid = (int)std::min<int64_t>(K.num_tiles, (int64_t)dev.sms * mi.occ);
+    if (hints && hints->grid > 0) mi.grid = hints->grid;
+    // effective run lengths averaged over partial tiles
+    mi.fillA = (double)N / ((double)K.num_tiles * K.V);
+    const double tm = predict_seconds(mi, dev);
+    ncand++;
+    if (tm < best_t) {
+      best_t = tm;
+      best_mi = mi;
+      bestK = K;
+      bestT = T;
+      best_kind = kind;
+      best_schema = schema;
+    }
+  };
+
+  int64_t blocksA[32], blocksB[32];
+  if (P.p[0] == 0) {
+    // ---- direct (FML / COPY): input run = dims 0..a (contiguous), output run = dim 0
+    int64_t pre = 1;
+    for (int a = 0; a < P.d; a++) {
+      const int nb = cand_blocks(P.n[a], pre, P.W, blocksA, hints ? hints->in_block : 0);
+      for (int i = 0; i < nb; i++) {
+        const int64_t ta = blocksA[i];
+        if (pre * ta * P.W < 1024 && ta < P.n[a] && !(hints && hints->in_block))
+          continue;  // tiny tiles only if forced by extents
+        consider(KK_DIRECT, a, ta, 0, a == 0 ? ta : P.n[0]);
+      }
+      pre *= P.n[a];
+      if (pre * P.W >= 256 * 1024 && !(hints && hints->in_dim > a)) break;
+    }
+  }
+  if (P.d > 1) {
+    // ---- staged (OD / OA / FMS): enumerate input and output groups
+    int64_t preA = 1;
+    for (int a = 0; a < P.d; a++) {
+      const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0);
+      int64_t preB = 1;
+      for (int b = 0; b < P.d; b++) {
+        const int pb = P.p[b];
+        const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0);
+        for (int i = 0; i < nbA; i++) {
+          for (int j = 0; j < nbB; j++) {
+            consider(KK_STAGED, a, blocksA[i], b, blocksB[j]);
+          }
+        }
+        preB *= P.n[pb];
+        if (preB * P.W >= 4096 && !(hints && hints->out_dim > b)) break;
+      }
+      preA *= P.n[a];
+      if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) break;
+    }
+  }
+  if (best_kind < 0) return force_schema == TTLG_SCHEMA_AUTO ? TTLG_ERR_INTERNAL : TTLG_ERR_UNSUPPORTED;
+
+  plan->kind = best_kind;
+  plan->W = P.W;
+  plan->threads = threads;
+  plan->grid = best_mi.grid;
+  plan->nbytes = N * P.W;
+  plan->kp = bestK;
+  ttlg_plan_info &I = plan->info;
+  memset(&I, 0, sizeof(I));
+  I.schema = best_schema;
+  I.dtype = dt;
+  I.rank = rank;
+  I.fused_rank = P.d;
+  for (int k = 0; k < P.d; k++) {
+    I.fused_extents[k] = P.n[k];
+    I.fused_perm[k] = P.p[k];
+    I.tile_extents[k] = bestT.t[k];
+  }
+  I.access_bytes = P.W;
+  I.in_dim = bestT.a;
+  I.out_dim = bestT.b;
+  I.in_run = bestK.LA;
+  I.out_run = bestK.LB;
+  I.tile_volume = bestK.V;
+  I.num_tiles = bestK.num_tiles;
+  I.grid = plan->grid;
+  I.threads = threads;
+  I.smem_bytes = bestK.smem_bytes;
+  I.bytes = 2 * N * P.W;
+  I.predicted_seconds = best_t;
+  I.candidates = ncand;
+  I.param_bytes = (int32_t)sizeof(TileParams);
+  return TTLG_OK;
+}
+
+}  // namespace ttlg

@@ -1,0 +1,146 @@
+// ttlg_internal.h -- plan and kernel-parameter layout shared by the host
+// planner (planner.cpp), the C ABI (api.cpp) and the sm_100a kernels
+// (kernels.cu).  Product code; never includes anything from oracle/.
+#pragma once
+
+#include <stdint.h>
+
+#include "../../include/ttlg.h"
+
+#define TTLG_MAXD TTLG_MAX_RANK
+
+namespace ttlg {
+
+// Fast unsigned division by a run-time constant (multiply-high + shift).
+// Valid for dividends n < 2^31 (tile indices and row indices always are).
+// quotient = (umulhi(n, mul) + (mul_hi_bit ? n : 0)) >> shr; we use the
+// 31+ceil(log2 d) formulation so that mul fits in 32 bits.
+struct FastDiv {
+  uint32_t div;
+  uint32_t mul;
+  uint32_t shr;
+};
+
+inline FastDiv make_fastdiv(uint32_t d) {
+  FastDiv f;
+  f.div = d;
+  if (d <= 1) {
+    f.mul = 0;
+    f.shr = 0;
+    return f;
+  }
+  uint32_t l = 0;
+  while ((1ull << l) < d) l++;  // ceil(log2 d)
+  uint32_t p = 31 + l;
+  f.mul = (uint32_t)(((1ull << p) + d - 1) / d);
+  f.shr = p - 32;
+  return f;
+}
+
+inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
+  if (f.div <= 1) return n;
+  return (uint32_t)((((uint64_t)n * f.mul) >> 32) >> f.shr);
+}
+
+// Kernel kinds.
+enum KernelKind : int32_t {
+  KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
+  KK_STAGED = 1,  // OD / OA / FMS: slice staged through shared memory
+};
+
+// Everything one launch needs, passed by value as a __grid_constant__ kernel
+// parameter (lives in the constant bank; replaces the paper's texture-bound
+// offset arrays, and its rank-specialised macro code,
+// L1138-1155: loops over these arrays are unrolled to TTLG_MAXD with guards so
+// every index is a compile-time constant).
+//
+// Tile ("slice" in the paper) geometry, all in access-element units:
+//   the tile is the box prod_k t[k] over fused input dims; the input run is
+//   the input-prefix dims 0..a (a possibly blocked), contiguous in A, length LA;
+//   the output run is the output-prefix dims perm[0..b] (perm[b] possibly
+//   blocked), contiguous in B, length LB.  A-rows enumerate the tile digits
+//   outside the input run (RA = V/LA), B-rows those outside the output run
+//   (RB = V/LB).  Per-row tables (built in shared memory once per CTA) hold the
+//   relative global offset and the shared-memory offset of each row.
+struct TileParams {
+  // ---- tile grid (tile index -> tile base), grid dims in input order, first fastest
+  uint32_t num_tiles;
+  int32_t ng;
+  FastDiv gdiv[TTLG_MAXD];
+  int64_t gsA[TTLG_MAXD];  // t[k] * strideA[k]
+  int64_t gsB[TTLG_MAXD];  // t[k] * strideB[k]
+  // ---- partial tiles: the two blockable dims (a = last input-run dim, pb = perm[b])
+  int32_t blkA_g, blkB_g;  // grid-dim index of dim a / dim pb, -1 if never partial
+  int32_t blkA_n, blkA_t, blkB_n, blkB_t;
+  // ---- run geometry
+  int32_t V;               // tile volume
+  int32_t LA, RA, LAunit;  // LAlim = LAunit * lim_a
+  int32_t LB, RB, LBunit;  // LBlim = LBunit * lim_pb
+  // ---- A-row digits (tile dims outside the input run), input order
+  int32_t nra, ra_blk;     // ra_blk: which A-row digit is dim pb (-1: none)
+  int32_t ra_ext[TTLG_MAXD];
+  int32_t ra_sG[TTLG_MAXD];  // stride in A
+  int32_t ra_sS[TTLG_MAXD];  // stride in the smem tile
+  // ---- B-row digits (tile dims outside the output run), input order
+  int32_t nrb, rb_blk;     // rb_blk: which B-row digit is dim a (-1: none)
+  int32_t rb_ext[TTLG_MAXD];
+  int32_t rb_sG[TTLG_MAXD];  // stride in B
+  int32_t rb_sS[TTLG_MAXD];
+  // ---- output-run digits, output order (-> smem column offsets)
+  int32_t nj;
+  int32_t j_ext[TTLG_MAXD];
+  int32_t j_sS[TTLG_MAXD];
+  // ---- shared-memory layout (bytes) and per-thread stepping
+  int32_t smem_elems;      // data tile elements incl. padding
+  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, smem_bytes;
+  int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
+};
+
+struct Problem {
+  int esize;       // bytes per element as given (4/8)
+  int W;           // access-element bytes after widening (4/8/16)
+  int d;           // fused rank
+  int64_t n[TTLG_MAXD];
+  int32_t p[TTLG_MAXD];
+};
+
+struct DeviceProfile {
+  int sms;
+  int smem_per_block_optin;
+  int smem_per_sm;
+  int max_threads_per_sm;
+  int regs_per_sm;
+  double hbm_gbs;  // measured copy bandwidth used by the model
+  bool virt;       // true: no device, virtual B200
+};
+
+}  // namespace ttlg
+
+struct ttlg_plan_s {
+  int device;  // -1 when planned against the virtual profile
+  int kind;    // ttlg::KernelKind
+  int W;       // access bytes
+  int threads;
+  int grid;
+  int64_t nbytes;  // N * s
+  ttlg::TileParams kp;
+  ttlg_plan_info info;
+  // original request (for the misaligned-pointer fallback)
+  int dt, rank;
+  int64_t ext[TTLG_MAXD];
+  int32_t perm[TTLG_MAXD];
+  ttlg_plan_hints hints;
+  bool has_hints;
+};
+
+namespace ttlg {
+// planner.cpp
+ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
+ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
+                      const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev);
+// api.cpp
+const DeviceProfile &device_profile(int device);
+// kernels.cu
+ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream);
+int kernel_regs(int kind, int W);  // registers per thread of a kernel variant (cached; 0 if unknown)
+}  // namespace ttlg

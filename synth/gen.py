@@ -113,3 +113,12 @@ def gen_tensor_torch(seed: int, n_elems: int, elem_bytes: int, device="cpu",
             ob[c0:c1] = lo.to(torch.int32)
         del z, l
     return out
+
+
+def gen_at_np(seed: int, idx, elem_bytes: int, mode: str = "splitmix") -> np.ndarray:
+    """Generator values at arbitrary linear indices (for sampled checks)."""
+    l = np.asarray(idx, dtype=np.uint64)
+    bits = l.copy() if mode == "index" else splitmix64_np(np.uint64(seed) ^ l)
+    if elem_bytes == 8:
+        return bits
+    return (bits & np.uint64(0xFFFFFFFF)).astype(np.uint32)

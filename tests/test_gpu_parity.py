@@ -1,0 +1,263 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle, bit for bit
+(tolerance 0: a transposition does no arithmetic, reading R3).
+
+- oracle-sized cases: every config, element by element, at sizes spanning
+  several tiles with ragged tails, under the auto plan AND every applicable
+  forced schema;
+- full BASELINE sizes in the launch configuration bench.py times: sampled
+  outputs checked one by one through oracle.source_index (lin_B -> lin_A),
+  plus the exactly-once/index-encoding property on whole tensors;
+- edge cases: rank 1, rank 15, extent-1 dims, odd extents, misaligned pointers
+  (narrow-access fallback), canary bands around B, A unchanged, single-use
+  path, non-default streams.
+"""
+import itertools
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle  # noqa: E402  (test infrastructure)
+import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg  # noqa: E402
+from synth import configs, gen_tensor_torch, gen_at_np, case_seed  # noqa: E402
+
+pytestmark = pytest.mark.gpu
+DEV = "cuda:0"
+
+
+def _bits(t):
+    t = t.contiguous()
+    if t.element_size() == 8:
+        return t.view(torch.int64).cpu().numpy().view(np.uint64)
+    return t.view(torch.int32).cpu().numpy().view(np.uint32)
+
+
+def _dt(eb):
+    return "f64" if eb == 8 else "f32"
+
+
+def _run(ext, perm, eb, seed, plan_kwargs=None, single_use=False, canary=0):
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(seed, n, eb, device=DEV)
+    Bfull = torch.empty(n + 2 * canary, dtype=A.dtype, device=DEV)
+    if canary:
+        Bfull.view(torch.int64 if eb == 8 else torch.int32).fill_(0x5A5A5A5A)
+    B = Bfull[canary:canary + n]
+    stream = torch.cuda.current_stream().cuda_stream
+    if single_use:
+        ttlg.transpose(_dt(eb), ext, perm, A.data_ptr(), B.data_ptr(), stream)
+        info = None
+    else:
+        p = ttlg.plan(_dt(eb), ext, perm, **(plan_kwargs or {}))
+        info = p.describe()
+        p.execute(A.data_ptr(), B.data_ptr(), stream)
+    torch.cuda.synchronize()
+    A_host = _bits(A)
+    expect = oracle.transpose(A_host, ext, perm)
+    got = _bits(B)
+    if canary:
+        band = _bits(Bfull)
+        assert (band[:canary] == band[0]).all() and (band[-canary:] == band[0]).all(), \
+            "write outside B"
+    # A must be untouched
+    assert np.array_equal(_bits(A), A_host)
+    return got, expect, info
+
+
+def _assert_equal(got, expect, what):
+    if not np.array_equal(got, expect):
+        bad = np.nonzero(got != expect)[0]
+        pytest.fail(f"{what}: {bad.size} mismatches, first at {bad[:8].tolist()}")
+
+
+# ---- config 1: all 24 perms of 16^4 fp64, auto + every applicable forced schema ------------
+@pytest.mark.parametrize("case", configs.config1(), ids=lambda c: "".join(map(str, c.perm)))
+def test_config1_all_schemas(case):
+    got, exp, info = _run(case.extents, case.perm, 8, case_seed(case.case_id), canary=64)
+    _assert_equal(got, exp, f"auto {info['schema']}")
+    for s in ("OD", "OA", "FMS", "FML"):
+        try:
+            ttlg.plan("f64", case.extents, case.perm, schema=s)
+        except ttlg.TtlgError:
+            continue
+        got, exp, info = _run(case.extents, case.perm, 8, case_seed(case.case_id),
+                              plan_kwargs={"schema": s}, canary=64)
+        _assert_equal(got, exp, f"forced {s}")
+
+
+def _scaled_cases():
+    out = []
+    for grp in ("c2", "c3", "c4", "c5"):
+        for c in configs.all_configs()[grp]:
+            out.append(configs.scaled(c, 1 << 20))
+    return out
+
+
+@pytest.mark.parametrize("case", _scaled_cases(), ids=lambda c: c.label())
+def test_scaled_configs_auto(case):
+    got, exp, info = _run(case.extents, case.perm, case.elem_bytes, case_seed(case.case_id),
+                          canary=32)
+    _assert_equal(got, exp, f"auto {info['schema']} {info}")
+
+
+@pytest.mark.parametrize("case", _scaled_cases()[::3], ids=lambda c: c.label())
+def test_scaled_configs_forced(case):
+    for s in ("OD", "OA", "FMS", "FML"):
+        try:
+            ttlg.plan(_dt(case.elem_bytes), case.extents, case.perm, schema=s)
+        except ttlg.TtlgError:
+            continue
+        got, exp, info = _run(case.extents, case.perm, case.elem_bytes,
+                              case_seed(case.case_id), plan_kwargs={"schema": s})
+        _assert_equal(got, exp, f"forced {s} {info}")
+
+
+# ---- ragged / odd extents, every rank-4 and a sample of rank-5/6 perms -----------------------
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.parametrize("ext", [(15, 17, 13, 19), (3, 33, 65, 7), (5, 2, 129, 31),
+                                 (27, 27, 27, 27), (1, 40, 1, 33)])
+def test_odd_extents_rank4(ext, eb):
+    for k, perm in enumerate(itertools.permutations(range(4))):
+        got, exp, info = _run(list(ext), list(perm), eb, 1000 + k)
+        _assert_equal(got, exp, f"{ext} {perm} {info['schema']}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_rank6_sample(eb):
+    rng = np.random.default_rng(6)
+    perms = list(itertools.permutations(range(6)))
+    for k in rng.choice(len(perms), 40, replace=False):
+        ext = [int(x) for x in rng.integers(2, 12, size=6)]
+        got, exp, info = _run(ext, list(perms[k]), eb, 2000 + int(k))
+        _assert_equal(got, exp, f"{ext} {perms[k]} {info['schema']}")
+
+
+def test_block_sweep_fig5():
+    """Every slice variant of the Fig. 5 sweep gives identical bytes (L1421-1436)."""
+    ext, perm = [27] * 5, [4, 1, 2, 0, 3]
+    for blk in (1, 2, 5, 7, 13, 27):
+        got, exp, info = _run(ext, perm, 8, 7100, plan_kwargs={"schema": "OD", "in_dim": 1,
+                                                                  "in_block": blk})
+        _assert_equal(got, exp, f"blockA={blk}")
+
+
+# ---- edge cases ---------------------------------------------------------------------------------
+def test_rank1_and_identity():
+    for ext, perm in [([1], [0]), ([7], [0]), ([1 << 20], [0]), ([33, 17], [0, 1])]:
+        got, exp, _ = _run(ext, perm, 4, 5)
+        _assert_equal(got, exp, f"{ext}")
+
+
+def test_rank15():
+    ext = [2] * 15
+    rng = np.random.default_rng(15)
+    for _ in range(6):
+        perm = [int(x) for x in rng.permutation(15)]
+        got, exp, info = _run(ext, perm, 8, 15)
+        _assert_equal(got, exp, f"rank15 {perm}")
+
+
+def test_extent_one_dims():
+    got, exp, _ = _run([1, 64, 1, 1, 48, 1], [4, 2, 1, 0, 5, 3], 8, 9)
+    _assert_equal(got, exp, "squeeze")
+
+
+def test_single_use_path():
+    for c in configs.config1()[::5]:
+        got, exp, _ = _run(c.extents, c.perm, 8, case_seed(c.case_id), single_use=True)
+        _assert_equal(got, exp, "ttlg_transpose")
+
+
+def test_misaligned_pointers_fall_back_to_element_width():
+    ext, perm = [4, 256, 96], [0, 2, 1]          # 16-byte rows -> widened plan
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(3, n + 1, 4, device=DEV)
+    B = torch.empty(n + 1, dtype=torch.float32, device=DEV)
+    p = ttlg.plan("f32", ext, perm)
+    assert p.describe()["access_bytes"] == 16
+    p.execute(A[1:].data_ptr(), B[1:].data_ptr(), torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    _assert_equal(_bits(B[1:]), oracle.transpose(_bits(A[1:]), ext, perm), "misaligned")
+
+
+def test_nondefault_stream_and_aliasing():
+    s = torch.cuda.Stream()
+    ext, perm = [64, 48, 40], [2, 0, 1]
+    A = gen_tensor_torch(4, 64 * 48 * 40, 8, device=DEV)
+    B = torch.empty_like(A)
+    p = ttlg.plan("f64", ext, perm)
+    with torch.cuda.stream(s):
+        p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)
+    s.synchronize()
+    _assert_equal(_bits(B), oracle.transpose(_bits(A), ext, perm), "stream")
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute(A.data_ptr(), A.data_ptr(), 0)
+    assert e.value.code == 2
+
+
+def test_transpose_tensor_torch_semantics():
+    x = gen_tensor_torch(8, 6 * 7 * 8 * 9, 4, device=DEV).view(6, 7, 8, 9)
+    for perm_t in [(3, 2, 1, 0), (0, 2, 1, 3), (1, 3, 0, 2)]:
+        y = ttlg.transpose_tensor(x, perm_t)
+        torch.cuda.synchronize()
+        assert torch.equal(y.view(torch.int32).cpu(),
+                           x.permute(perm_t).contiguous().view(torch.int32).cpu())
+    e = torch.empty(0, 5, device=DEV)
+    assert ttlg.transpose_tensor(e, (1, 0)).shape == (5, 0)
+
+
+# ---- full BASELINE sizes, launch config as bench.py -----------------------------------------------
+def _sampled_full(case, nsamp=200_000):
+    n = case.n_elems
+    eb = case.elem_bytes
+    seed = case_seed(case.case_id)
+    A = gen_tensor_torch(seed, n, eb, device=DEV)
+    B = torch.empty_like(A)
+    p = ttlg.plan(_dt(eb), case.extents, case.perm)
+    p.execute(A.data_ptr(), B.data_ptr(), torch.cuda.current_stream().cuda_stream)
+    rng = np.random.default_rng(case.case_id)
+    linB = np.unique(np.concatenate([rng.integers(0, n, nsamp), np.arange(64),
+                                     np.arange(n - 64, n)]))
+    Bv = B.view(torch.int64 if eb == 8 else torch.int32)
+    got = Bv[torch.from_numpy(linB).to(DEV)].cpu().numpy().view(np.uint64 if eb == 8 else np.uint32)
+    linA = oracle.source_index(case.extents, case.perm, linB)
+    exp = gen_at_np(seed, linA, eb)
+    info = p.describe()
+    del A, B
+    torch.cuda.empty_cache()
+    return got, exp, info
+
+
+@pytest.mark.parametrize("case", configs.config2(), ids=lambda c: c.label())
+def test_full_ttc57_sampled(case):
+    got, exp, info = _sampled_full(case)
+    _assert_equal(got, exp, f"{info['schema']}")
+
+
+@pytest.mark.parametrize("case", configs.config3() + configs.config4(),
+                         ids=lambda c: c.label())
+def test_full_ccsdt_smallfvi_sampled(case):
+    got, exp, info = _sampled_full(case, nsamp=50_000)
+    _assert_equal(got, exp, f"{info['schema']}")
+
+
+@pytest.mark.parametrize("case", configs.config5(), ids=lambda c: c.label())
+def test_full_8GiB_sampled(case):
+    got, exp, info = _sampled_full(case, nsamp=50_000)
+    _assert_equal(got, exp, f"{info['schema']}")
+
+
+def test_full_exactly_once_index_encoding():
+    """Whole-tensor check at a TTC size: with A_bits[l] = l, B must be exactly
+    oracle.source_index(arange(N)) (closed form from the definition)."""
+    for case in configs.config2()[::7]:
+        n = case.n_elems
+        A = gen_tensor_torch(0, n, 8, device=DEV, mode="index")
+        B = torch.empty_like(A)
+        p = ttlg.plan("f64", case.extents, case.perm)
+        p.execute(A.data_ptr(), B.data_ptr(), torch.cuda.current_stream().cuda_stream)
+        got = B.view(torch.int64).cpu().numpy()
+        exp = oracle.source_index(case.extents, case.perm, np.arange(n, dtype=np.int64))
+        assert np.array_equal(got, exp), case.label()
+        del A, B

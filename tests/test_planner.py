@@ -1,0 +1,201 @@
+"""Host-side logic through the C ABI, on a CPU-only box (virtual B200 profile):
+ABI exports, argument validation, squeeze + index fusion,
+schema applicability (Alg. 1), forced schemas, kernel-parameter
+legality, model sanity, and the torch <-> FVI-first convention conversion."""
+import ctypes
+import itertools
+import os
+import re
+import subprocess
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
+from paper_conf_ipps_veduradasskhpkn18_b200 import _ffi
+from synth import configs
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+# ---- ABI ----------------------------------------------------------------------------
+def test_header_symbols_exported():
+    hdr = open(os.path.join(ROOT, "include", "ttlg.h")).read()
+    declared = set(re.findall(r"\b(ttlg_[a-z_]+)\s*\(", hdr))
+    out = subprocess.run(["nm", "-D", "--defined-only", _ffi.LIB_PATH], capture_output=True,
+                         text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (ttlg_[a-z_]+)\b", out))
+    assert declared, "no declarations parsed"
+    assert declared <= exported, declared - exported
+    assert set(_ffi.EXPORTS) == declared
+
+
+def test_status_strings_and_version():
+    assert _ffi.lib.ttlg_version() == 100
+    assert _ffi.lib.ttlg_status_string(0) == b"TTLG_OK"
+    assert _ffi.lib.ttlg_status_string(2) == b"TTLG_ERR_ALIASING"
+    assert _ffi.lib.ttlg_schema_name(3) == b"OD"
+
+
+def test_library_has_sm100a_code():
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", _ffi.LIB_PATH],
+                         capture_output=True, text=True, check=True).stdout
+    assert "sm_100a" in out
+
+
+# ---- validation ------------------------------------------------------------------------
+@pytest.mark.parametrize("ext,perm", [
+    ([], []), ([2] * 16, list(range(16))), ([0, 3], [1, 0]), ([2, 3], [0, 0]),
+    ([2, 3], [0, 2]), ([-1, 3], [1, 0]), ([1 << 40, 1 << 30], [1, 0])])
+def test_invalid_arguments(ext, perm):
+    with pytest.raises(ttlg.TtlgError) as e:
+        ttlg.plan("f64", ext, perm)
+    assert e.value.code == 1
+
+
+def test_bad_dtype_code():
+    with pytest.raises(ttlg.TtlgError):
+        ttlg.plan(7, [4, 4], [1, 0])
+
+
+def test_execute_without_gpu_is_device_error():
+    p = ttlg.plan("f32", [64, 64], [1, 0])
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute(1 << 20, 1 << 30)
+    assert e.value.code == 3  # TTLG_ERR_DEVICE (no device here), never a CPU fallback
+
+
+def test_aliasing_detected_before_device_check():
+    p = ttlg.plan("f64", [64, 64], [1, 0])
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute(1 << 20, (1 << 20) + 8)
+    assert e.value.code == 2
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute((1 << 20) + 4, 1 << 30)   # not element aligned
+    assert e.value.code == 1
+
+
+# ---- fusion -----------------------------------------------------------------------------
+def test_paper_fusion_example():
+    # [i0,i1,i2,i3] => [i3,i1,i2,i0] fuses i1,i2 into rank 3
+    d = ttlg.plan("f32", [5, 6, 7, 8], [3, 1, 2, 0]).describe()
+    assert d["fused_rank"] == 3
+    assert d["fused_extents"] == [5, 42, 8]
+    assert d["fused_perm"] == [2, 1, 0]
+
+
+def test_fused_rank_histogram_720():
+    # the "staircase" of Figs 6-11 (L1586-1588): scaled ranks of all 720 6-D perms
+    hist = {}
+    for p in itertools.permutations(range(6)):
+        d = ttlg.plan("f32", [3] * 6, p).describe()["fused_rank"]
+        hist[d] = hist.get(d, 0) + 1
+    assert hist == {1: 1, 2: 5, 3: 30, 4: 110, 5: 265, 6: 309}
+
+
+def test_squeeze_and_identity():
+    d = ttlg.plan("f64", [1, 7, 1, 9], [3, 2, 0, 1]).describe()
+    assert d["fused_rank"] == 2 and d["fused_extents"] == [7, 9] and d["fused_perm"] == [1, 0]
+    d = ttlg.plan("f32", [4, 5, 6], [0, 1, 2]).describe()
+    assert d["schema"] == "COPY" and d["fused_rank"] == 1
+    d = ttlg.plan("f64", [1, 1], [1, 0]).describe()
+    assert d["schema"] == "COPY"
+
+
+def test_widening_small_fvi():
+    # [2,4096,4096] fp32 perm 0 2 1: 8-byte rows -> one access element -> 2-D transpose
+    d = ttlg.plan("f32", [2, 4096, 4096], [0, 2, 1]).describe()
+    assert d["access_bytes"] == 8 and d["fused_rank"] == 2 and d["fused_perm"] == [1, 0]
+    d = ttlg.plan("f32", [4, 4096, 4096], [0, 2, 1]).describe()
+    assert d["access_bytes"] == 16 and d["fused_rank"] == 2
+    d = ttlg.plan("f32", [3, 4096, 4096], [0, 2, 1]).describe()
+    assert d["access_bytes"] == 4 and d["fused_rank"] == 3
+
+
+# ---- schema applicability -------------------------------------------------------------------
+def _groups(d):
+    a, b = d["in_dim"], d["out_dim"]
+    IS = set(range(a + 1))
+    OS = set(d["fused_perm"][: b + 1])
+    return IS, OS
+
+
+def _check_plan_legal(d):
+    IS, OS = _groups(d)
+    fp, te, fe = d["fused_perm"], d["tile_extents"], d["fused_extents"]
+    for k in range(d["fused_rank"]):
+        assert 1 <= te[k] <= fe[k]
+        if k not in IS and k not in OS:
+            assert te[k] == 1
+    for k in range(d["in_dim"]):
+        assert te[k] == fe[k]                      # only the slowest input-group dim is blocked
+    for i in range(d["out_dim"]):
+        assert te[fp[i]] == fe[fp[i]]              # only the slowest output-group dim is blocked
+    if d["schema"] == "OD":
+        assert not (IS & OS)
+    if d["schema"] == "OA":
+        assert IS & OS and fp[0] != 0
+    if d["schema"] in ("FML", "FMS", "COPY"):
+        assert fp[0] == 0
+    assert d["param_bytes"] <= 32764
+    assert d["smem_bytes"] <= 227 * 1024
+    assert d["predicted_seconds"] >= d["bytes"] / 6555.5e9 * 0.999
+
+
+@pytest.mark.parametrize("group", ["c1", "c2", "c3", "c4", "c5"])
+def test_auto_plans_legal(group):
+    for c in configs.all_configs()[group]:
+        d = ttlg.plan("f64" if c.elem_bytes == 8 else "f32", c.extents, c.perm).describe()
+        _check_plan_legal(d)
+
+
+def test_forced_schemas():
+    ok = {"OD": 0, "OA": 0, "FMS": 0, "FML": 0}
+    for c in configs.config1():
+        fp0 = c.perm[0]
+        for s in ("OD", "OA", "FMS", "FML"):
+            try:
+                d = ttlg.plan("f64", c.extents, c.perm, schema=s).describe()
+            except ttlg.TtlgError as e:
+                assert e.code == 7
+                continue
+            assert d["schema"] == s or (s == "FML" and d["schema"] == "COPY")
+            _check_plan_legal(d)
+            ok[s] += 1
+        # applicability: OD whenever the fused FVI differs; FML whenever it matches
+        d0 = ttlg.plan("f64", c.extents, c.perm).describe()
+        if d0["fused_perm"][0] != 0:
+            ttlg.plan("f64", c.extents, c.perm, schema="OD")
+        else:
+            ttlg.plan("f64", c.extents, c.perm, schema="FML")
+    assert all(v > 0 for v in ok.values()), ok
+
+
+def test_forced_blocks_respected():
+    d = ttlg.plan("f64", [27] * 5, [4, 1, 2, 0, 3], schema="OD", in_dim=1, in_block=7,
+                  out_dim=0, out_block=27).describe()
+    # Fig. 5's choice (L1435-1436): input slice 27x7 = 189, output slice 27
+    assert d["in_run"] == 189 and d["out_run"] == 27
+
+
+def test_predict_time_monotone_in_volume():
+    t1 = ttlg.predict_time("f64", [256, 256, 64], [2, 1, 0])
+    t2 = ttlg.predict_time("f64", [256, 256, 512], [2, 1, 0])
+    assert t2 > 4 * t1
+    assert t2 >= 2 * 256 * 256 * 512 * 8 / 6555.5e9
+
+
+# ---- torch convention -------------------------------------------------------------------------
+def test_torch_to_c_matches_numpy_transpose():
+    import oracle
+    rng = np.random.default_rng(0)
+    for _ in range(50):
+        d = int(rng.integers(1, 6))
+        shape = [int(x) for x in rng.integers(1, 5, size=d)]
+        perm_t = [int(x) for x in rng.permutation(d)]
+        X = np.arange(int(np.prod(shape)), dtype=np.uint64).reshape(shape)
+        ext, perm = ttlg.torch_to_c(shape, perm_t)
+        got = oracle.transpose(X.ravel(), ext, perm)
+        assert np.array_equal(got, np.ascontiguousarray(X.transpose(perm_t)).ravel())
+    # 2-D: (1, 0) <-> (1, 0)
+    assert ttlg.torch_to_c([3, 5], [1, 0]) == ([5, 3], [1, 0])
