@@ -87,6 +87,9 @@ typedef struct {
   int32_t threads;                       /* 0 = auto; else threads per block             */
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
+  int32_t variant;                       /* kernel variant bits (tests / calibration):
+                                            1 = register-staged instead of cp.async
+                                            pipeline, 2 = no streaming cache hints       */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -108,6 +111,7 @@ typedef struct {
   double predicted_seconds;               /* performance-model prediction                */
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
+  int32_t kernel;                         /* 0 direct, 1 register-staged, 2 cp.async pipe */
 } ttlg_plan_info;
 
 void ttlg_plan_hints_init(ttlg_plan_hints *hints);

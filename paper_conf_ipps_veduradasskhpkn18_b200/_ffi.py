@@ -37,7 +37,7 @@ class PlanHints(ctypes.Structure):
                 ("in_block", ctypes.c_int64), ("out_dim", ctypes.c_int32),
                 ("out_block", ctypes.c_int64), ("elem_bytes_override", ctypes.c_int32),
                 ("threads", ctypes.c_int32), ("grid", ctypes.c_int32),
-                ("no_fusion", ctypes.c_int32)]
+                ("no_fusion", ctypes.c_int32), ("variant", ctypes.c_int32)]
 
 
 class PlanInfo(ctypes.Structure):
@@ -53,7 +53,7 @@ class PlanInfo(ctypes.Structure):
                 ("grid", ctypes.c_int32), ("threads", ctypes.c_int32),
                 ("smem_bytes", ctypes.c_int32), ("bytes", ctypes.c_int64),
                 ("predicted_seconds", ctypes.c_double), ("candidates", ctypes.c_int32),
-                ("param_bytes", ctypes.c_int32)]
+                ("param_bytes", ctypes.c_int32), ("kernel", ctypes.c_int32)]
 
     def to_dict(self) -> dict:
         d = self.fused_rank
@@ -71,6 +71,7 @@ class PlanInfo(ctypes.Structure):
             "grid": self.grid, "threads": self.threads, "smem_bytes": self.smem_bytes,
             "bytes": self.bytes, "predicted_seconds": self.predicted_seconds,
             "candidates": self.candidates, "param_bytes": self.param_bytes,
+            "kernel": ["direct", "staged", "pipe"][self.kernel],
         }
 
 

@@ -30,7 +30,8 @@ def _dtype_code(dtype) -> int:
 
 
 def make_hints(schema=None, in_dim=None, in_block=None, out_dim=None, out_block=None,
-               access_bytes=None, threads=None, grid=None, no_fusion=False) -> PlanHints:
+               access_bytes=None, threads=None, grid=None, no_fusion=False,
+               variant=None) -> PlanHints:
     h = PlanHints()
     lib.ttlg_plan_hints_init(ctypes.byref(h))
     if schema is not None:
@@ -50,6 +51,8 @@ def make_hints(schema=None, in_dim=None, in_block=None, out_dim=None, out_block=
     if grid is not None:
         h.grid = grid
     h.no_fusion = 1 if no_fusion else 0
+    if variant is not None:
+        h.variant = variant
     return h
 
 

@@ -49,6 +49,35 @@ __device__ __forceinline__ uint32_t fdiv(uint32_t n, const FastDiv &f) {
   return __umulhi(n, f.mul) >> f.shr;  // grid divisors are always >= 2
 }
 
+template <bool CS, typename T>
+__device__ __forceinline__ T ld_stream(const T *p) {
+  if constexpr (CS) return __ldcs(p);
+  else return *p;
+}
+template <bool CS, typename T>
+__device__ __forceinline__ void st_stream(T *p, T v) {
+  if constexpr (CS) __stcs(p, v);
+  else *p = v;
+}
+
+// cp.async (LDGSTS): global -> shared without a register round trip.
+template <int W>
+__device__ __forceinline__ void cp_async(void *smem_ptr, const void *gptr) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem_ptr);
+  if constexpr (W == 16)
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gptr) : "memory");
+  else
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(s), "l"(gptr), "n"(W)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() {
+  asm volatile("cp.async.commit_group;\n" ::: "memory");
+}
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
+}
+
 struct TileCtx {
   int64_t bA, bB;
   int limA, limB;
@@ -95,7 +124,7 @@ __device__ __forceinline__ TileCtx decode_tile(const TileParams &P, uint32_t til
     (DIG)[i] = dg;                                                           \
   }
 
-template <int W, int U>
+template <int W, int U, bool CS>
 __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TileParams P,
                                                 const void *__restrict__ Av,
                                                 void *__restrict__ Bv) {
@@ -124,7 +153,7 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TilePara
       for (int u = 0; u < U; u++) {
         ob[u] = -1;
         if (e < lim) {
-          v[u] = __ldcs(Ab + e);
+          v[u] = ld_stream<CS>(Ab + e);
           ob[u] = tabB[r].x + j;
         }
         e += NT;
@@ -137,12 +166,12 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TilePara
       }
 #pragma unroll
       for (int u = 0; u < U; u++)
-        if (ob[u] >= 0) __stcs(Bb + ob[u], v[u]);
+        if (ob[u] >= 0) st_stream<CS>(Bb + ob[u], v[u]);
     }
   }
 }
 
-template <int W, int U>
+template <int W, int U, bool CS>
 __global__ void __launch_bounds__(256) k_staged(const __grid_constant__ TileParams P,
                                                 const void *__restrict__ Av,
                                                 void *__restrict__ Bv) {
@@ -193,7 +222,7 @@ __global__ void __launch_bounds__(256) k_staged(const __grid_constant__ TilePara
           so[u] = -1;
           if (r < P.RA && (full || (x < LAlim && digB[r] < c.limB))) {
             const int2 t = tabA[r];
-            v[u] = __ldcs(Ab + t.x + x);
+            v[u] = ld_stream<CS>(Ab + t.x + x);
             so[u] = t.y + x;
           }
           x += P.dxA;
@@ -218,7 +247,7 @@ __global__ void __launch_bounds__(256) k_staged(const __grid_constant__ TilePara
         for (int u = 0; u < U; u++) {
           if (r < P.RB && (full || (j < LBlim && digA[r] < c.limA))) {
             const int2 t = tabB[r];
-            __stcs(Bb + t.x + j, data[t.y + jcol[j]]);
+            st_stream<CS>(Bb + t.x + j, data[t.y + jcol[j]]);
           }
           j += P.dxB;
           r += P.drB;
@@ -233,23 +262,127 @@ __global__ void __launch_bounds__(256) k_staged(const __grid_constant__ TilePara
   }
 }
 
+// k_pipe: the staged schema with the load phase issued as cp.async into one
+// of two shared-memory buffers, one tile ahead: tile k+1 streams in while
+// tile k is written out, so every CTA keeps a whole tile of loads in flight
+// (the B200 replacement of the paper's coarsening for latency hiding, L1115-1136).
+template <int W, int U, bool CS>
+__global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams P,
+                                              const void *__restrict__ Av,
+                                              void *__restrict__ Bv) {
+  using T = typename Vec<W>::T;
+  extern __shared__ __align__(16) unsigned char smem[];
+  int2 *tabA = reinterpret_cast<int2 *>(smem);
+  int2 *tabB = reinterpret_cast<int2 *>(smem + P.off_tabB);
+  int *jcol = reinterpret_cast<int *>(smem + P.off_jcol);
+  int *digB = reinterpret_cast<int *>(smem + P.off_digB);
+  int *digA = reinterpret_cast<int *>(smem + P.off_digA);
+  T *buf0 = reinterpret_cast<T *>(smem + P.off_data);
+  T *buf1 = reinterpret_cast<T *>(smem + P.off_data2);
+  const T *A = reinterpret_cast<const T *>(Av);
+  T *B = reinterpret_cast<T *>(Bv);
+
+  TTLG_BUILD_ROWS(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk, tabA, digB);
+  TTLG_BUILD_ROWS(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
+  for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
+    int rem = j, s = 0;
+#pragma unroll
+    for (int k = 0; k < TTLG_MAXD; k++) {
+      if (k < P.nj) {
+        const int e = P.j_ext[k];
+        const int cq = rem / e;
+        s += (rem - cq * e) * P.j_sS[k];
+        rem = cq;
+      }
+    }
+    jcol[j] = s;
+  }
+  __syncthreads();
+
+  const int tid = threadIdx.x;
+  const int rA0 = tid / P.LA, xA0 = tid % P.LA;
+  const int rB0 = tid / P.LB, xB0 = tid % P.LB;
+
+  auto issue = [&](const TileCtx &c, T *buf) {
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int LAlim = P.LAunit * c.limA;
+    const T *Ab = A + c.bA;
+    int r = rA0, x = xA0;
+    while (r < P.RA) {
+      if (full || (x < LAlim && digB[r] < c.limB)) {
+        const int2 t = tabA[r];
+        cp_async<W>(buf + t.y + x, Ab + t.x + x);
+      }
+      x += P.dxA;
+      r += P.drA;
+      if (x >= P.LA) {
+        x -= P.LA;
+        r++;
+      }
+    }
+  };
+
+  uint32_t tile = blockIdx.x;
+  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
+  if (tile < P.num_tiles) issue(cur, buf0);
+  cp_async_commit();
+  for (int k = 0; tile < P.num_tiles; k++) {
+    const uint32_t next = tile + gridDim.x;
+    TileCtx nx = cur;
+    if (next < P.num_tiles) {
+      nx = decode_tile(P, next);
+      issue(nx, (k & 1) ? buf0 : buf1);
+    }
+    cp_async_commit();
+    cp_async_wait<1>();
+    __syncthreads();
+    {
+      const T *data = (k & 1) ? buf1 : buf0;
+      const bool full = (cur.limA == P.blkA_t) && (cur.limB == P.blkB_t);
+      const int LBlim = P.LBunit * cur.limB;
+      T *Bb = B + cur.bB;
+      int r = rB0, j = xB0;
+      while (r < P.RB) {
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          if (r < P.RB && (full || (j < LBlim && digA[r] < cur.limA))) {
+            const int2 t = tabB[r];
+            st_stream<CS>(Bb + t.x + j, data[t.y + jcol[j]]);
+          }
+          j += P.dxB;
+          r += P.drB;
+          if (j >= P.LB) {
+            j -= P.LB;
+            r++;
+          }
+        }
+      }
+    }
+    __syncthreads();
+    cur = nx;
+    tile = next;
+  }
+  cp_async_wait<0>();
+}
+
 // ---------------------------------------------------------------------------
 // launch plumbing
-typedef void (*KernelFn)(TileParams, const void *, void *);
+template <int W, bool CS>
+static const void *kernel_ptr_w(int kind) {
+  constexpr int U = (W == 16) ? 4 : 8;
+  switch (kind) {
+    case KK_DIRECT: return (const void *)k_direct<W, U, CS>;
+    case KK_STAGED: return (const void *)k_staged<W, U, CS>;
+    case KK_PIPE: return (const void *)k_pipe<W, U, CS>;
+  }
+  return nullptr;
+}
 
-static const void *kernel_ptr(int kind, int W) {
-  if (kind == KK_DIRECT) {
-    switch (W) {
-      case 4: return (const void *)k_direct<4, 8>;
-      case 8: return (const void *)k_direct<8, 8>;
-      case 16: return (const void *)k_direct<16, 4>;
-    }
-  } else {
-    switch (W) {
-      case 4: return (const void *)k_staged<4, 8>;
-      case 8: return (const void *)k_staged<8, 8>;
-      case 16: return (const void *)k_staged<16, 4>;
-    }
+static const void *kernel_ptr(int kind, int W, bool cs) {
+  switch (W) {
+    case 4: return cs ? kernel_ptr_w<4, true>(kind) : kernel_ptr_w<4, false>(kind);
+    case 8: return cs ? kernel_ptr_w<8, true>(kind) : kernel_ptr_w<8, false>(kind);
+    case 16: return cs ? kernel_ptr_w<16, true>(kind) : kernel_ptr_w<16, false>(kind);
   }
   return nullptr;
 }
@@ -257,13 +390,13 @@ static const void *kernel_ptr(int kind, int W) {
 static int widx(int W) { return W == 4 ? 0 : (W == 8 ? 1 : 2); }
 
 int kernel_regs(int kind, int W) {
-  static int regs[2][3] = {{-1, -1, -1}, {-1, -1, -1}};
+  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
   static std::mutex mu;
   std::lock_guard<std::mutex> g(mu);
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, true)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -274,19 +407,22 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W);
+  const bool cs = !(plan->variant & 2);
+  const void *fn = kernel_ptr(plan->kind, plan->W, cs);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {
-    // opt in once per (kernel, device, size class)
-    static int done[2][3][8];
+    // opt in once per (kernel variant, device)
+    static bool done[KK_NUM][3][2][16];
     int dev = 0;
     cudaGetDevice(&dev);
-    if (dev < 8 && !done[plan->kind][widx(plan->W)][dev]) {
+    if (dev >= 16) return TTLG_ERR_DEVICE;
+    bool &d = done[plan->kind][widx(plan->W)][cs][dev];
+    if (!d) {
       if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024) !=
           cudaSuccess)
         return TTLG_ERR_CUDA;
-      done[plan->kind][widx(plan->W)][dev] = 1;
+      d = true;
     }
   }
   TileParams kp = plan->kp;

@@ -37,14 +37,17 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   // bytes in flight: each CTA keeps up to UNROLL*threads access elements of
   // loads outstanding (Little's law with the loaded-DRAM latency)
   const double unroll = (mi.kind == KK_DIRECT) ? kModelUnrollDirect : kModelUnrollStaged;
-  const double inflight = (double)mi.occ * std::min<double>(mi.V, unroll * mi.threads) * W;
+  // the cp.async pipeline keeps a whole tile of loads in flight per CTA
+  const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
+                                              : std::min<double>(mi.V, unroll * mi.threads);
+  const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = dev.sms * inflight / kModelLatency;
   const double bw_eff = std::min(bw, bw_lat);
-  const double per_cta = std::ceil(tiles / mi.grid);
-  const double wave = per_cta / (tiles / mi.grid);
+  const double tiles_per_cta = std::ceil(tiles / mi.grid);
+  const double wave = tiles_per_cta / (tiles / mi.grid);
   F.f[0] = 1.0;
   F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
-  F.f[2] = per_cta / std::max(1, mi.occ);
+  F.f[2] = tiles_per_cta / std::max(1, mi.occ);
   F.f[3] = runs / dev.sms;
   return F;
 }

@@ -254,7 +254,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     }
     Q *= T.t[k];
   }
-  const int64_t smem_elems = (kind == KK_STAGED) ? cur : 0;
+  const int64_t smem_elems = (kind != KK_DIRECT) ? cur : 0;
 
   // A-row digits: tile dims outside the input run, input order
   int64_t maxG = 0;
@@ -301,13 +301,14 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     off += (bytes + 15) / 16 * 16;
     return (int32_t)o;
   };
-  if (kind == KK_STAGED) {
+  if (kind != KK_DIRECT) {
     take((int64_t)K.RA * 8);  // tabA at 0
     K.off_tabB = take((int64_t)K.RB * 8);
     K.off_jcol = take((int64_t)K.LB * 4);
     K.off_digB = take((int64_t)K.RA * 4);
     K.off_digA = take((int64_t)K.RB * 4);
     K.off_data = take(smem_elems * P.W);
+    K.off_data2 = (kind == KK_PIPE) ? take(smem_elems * P.W) : K.off_data;
   } else {
     K.off_tabB = take((int64_t)K.RB * 8);
     K.off_jcol = 0;
@@ -413,7 +414,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     int64_t V = 1;
     for (int k = 0; k < P.d; k++) V *= T.t[k];
-    if (kind == KK_STAGED && V * P.W > max_tile_bytes) return;
+    if (kind != KK_DIRECT && V * P.W > max_tile_bytes) return;
     if (kind == KK_DIRECT && V * P.W > 256 * 1024) return;
     TileParams K;
     if (!build_params(P, T, kind, threads, K)) return;
@@ -465,6 +466,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (pre * P.W >= 256 * 1024 && !(hints && hints->in_dim > a)) break;
     }
   }
+  const int staged_kind = (hints && (hints->variant & 1)) ? KK_STAGED : KK_PIPE;
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
@@ -476,7 +478,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0);
         for (int i = 0; i < nbA; i++) {
           for (int j = 0; j < nbB; j++) {
-            consider(KK_STAGED, a, blocksA[i], b, blocksB[j]);
+            consider(staged_kind, a, blocksA[i], b, blocksB[j]);
           }
         }
         preB *= P.n[pb];
@@ -489,6 +491,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (best_kind < 0) return force_schema == TTLG_SCHEMA_AUTO ? TTLG_ERR_INTERNAL : TTLG_ERR_UNSUPPORTED;
 
   plan->kind = best_kind;
+  plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
   plan->threads = threads;
   plan->grid = best_mi.grid;
@@ -519,6 +522,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   I.predicted_seconds = best_t;
   I.candidates = ncand;
   I.param_bytes = (int32_t)sizeof(TileParams);
+  I.kernel = best_kind;
   return TTLG_OK;
 }
 

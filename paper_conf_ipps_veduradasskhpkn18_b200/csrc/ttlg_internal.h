@@ -45,7 +45,9 @@ inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
 // Kernel kinds.
 enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
-  KK_STAGED = 1,  // OD / OA / FMS: slice staged through shared memory
+  KK_STAGED = 1,  // OD / OA / FMS: slice staged through shared memory (register loads)
+  KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered staging (default)
+  KK_NUM = 3,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -92,7 +94,7 @@ struct TileParams {
   int32_t j_sS[TTLG_MAXD];
   // ---- shared-memory layout (bytes) and per-thread stepping
   int32_t smem_elems;      // data tile elements incl. padding
-  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, smem_bytes;
+  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
 };
 
@@ -122,6 +124,7 @@ struct ttlg_plan_s {
   int W;       // access bytes
   int threads;
   int grid;
+  int variant;  // hint bits: 1 = register-staged kernel, 2 = no streaming cache hints
   int64_t nbytes;  // N * s
   ttlg::TileParams kp;
   ttlg_plan_info info;

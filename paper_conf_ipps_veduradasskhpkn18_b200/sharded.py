@@ -1,0 +1,127 @@
+"""Sharded transposition across GPUs (one process per GPU, torch.distributed).
+
+Not in the paper (single K40c, Table III); required by
+BASELINE.json's north star and config 5.  A is distributed along its
+outermost input dim d-1 (rank p holds i_{d-1} in [p*c, (p+1)*c), c = n_{d-1}/P,
+a contiguous slab of A); B is returned distributed along its outermost output
+dim o_{d-1} = input dim q = perm[d-1] (also a contiguous slab of B).
+
+* q == d-1 ("no move"): every rank transposes its own slab with the same
+  permutation -- zero communication, near-linear weak scaling.
+* q != d-1 ("moved"): one exchange step, the only collective of the library:
+    1. local transpose of the slab (extent c on dim d-1).  Its outermost
+       output dim is o_{d-1} = q, so its P sub-ranges of i_q are contiguous
+       chunks -> the local output IS the all-to-all send buffer;
+    2. all_to_all_single with equal splits (NCCL over NVLink/NVSwitch);
+    3. fold: the P received chunks, source rank outermost, are the FVI-first
+       tensor [X, Y, P] with X = prod of the local output extents up to and
+       including o_k (k = position of d-1 in perm, extent c), Y = the rest;
+       the B slab is [X, P, Y], i.e. the transposition (0 2 1) of it
+       (matching FVI -> FML/FMS kernels).
+  Requires P | n_{d-1} and P | n_q (else ValueError: run replicas instead).
+
+`local_fn(extents, perm, src, dst)` performs one dense transposition; the
+default is the CUDA library (ttlg_transpose on the current stream).  CPU unit
+tests inject the oracle there to check the decomposition over gloo.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+from typing import Callable, List, Optional, Sequence
+
+
+@dataclass
+class ShardPlan:
+    world: int
+    extents: List[int]        # global input extents (FVI first)
+    perm: List[int]
+    moved: bool               # True: needs the all-to-all
+    local_extents: List[int]  # this rank's A slab
+    out_local_extents: List[int]  # this rank's B slab (output order)
+    fold_extents: Optional[List[int]]  # [X, Y, P] for the fold (moved only)
+    n_local: int              # elements per rank
+
+
+def plan_shards(extents: Sequence[int], perm: Sequence[int], world: int) -> ShardPlan:
+    ext = [int(e) for e in extents]
+    perm = [int(p) for p in perm]
+    d = len(ext)
+    if sorted(perm) != list(range(d)):
+        raise ValueError("perm must be a permutation")
+    if ext[d - 1] % world:
+        raise ValueError(f"P={world} must divide the sharded input extent {ext[d - 1]}")
+    c = ext[d - 1] // world
+    local = ext[:-1] + [c]
+    n_local = 1
+    for e in local:
+        n_local *= e
+    q = perm[d - 1]
+    out_global = [ext[p] for p in perm]
+    if q == d - 1:
+        out_local = out_global[:-1] + [c]
+        return ShardPlan(world, ext, perm, False, local, out_local, None, n_local)
+    if ext[q] % world:
+        raise ValueError(f"P={world} must divide the output-sharded extent {ext[q]}")
+    cq = ext[q] // world
+    k = perm.index(d - 1)
+    # local output extents (output order) of the slab transpose
+    lo = [local[p] for p in perm]
+    X = 1
+    for i in range(k + 1):
+        X *= lo[i]
+    Y = 1
+    for i in range(k + 1, d - 1):
+        Y *= lo[i]
+    Y *= cq
+    out_local = out_global[:-1] + [cq]
+    return ShardPlan(world, ext, perm, True, local, out_local, [X, Y, world], n_local)
+
+
+def _default_local_fn(extents, perm, src, dst):
+    import torch
+    from .api import transpose, _dt_of_tensor
+    transpose(_dt_of_tensor(src), extents, perm, src.data_ptr(), dst.data_ptr(),
+              torch.cuda.current_stream(src.device).cuda_stream)
+
+
+def sharded_transpose(A_local, extents: Sequence[int], perm: Sequence[int], group=None,
+                      local_fn: Optional[Callable] = None, work=None, phase_events=None):
+    """Transpose a tensor sharded along its outermost input dim; returns this
+    rank's slab of B (flat, output-order layout of `out_local_extents`).
+    `work`: optional preallocated (send, recv) flat buffers of n_local elements.
+    `phase_events`: optional list that receives (name, start, end) CUDA events."""
+    import torch
+    import torch.distributed as dist
+
+    world = dist.get_world_size(group)
+    sp = plan_shards(extents, perm, world)
+    fn = local_fn or _default_local_fn
+    if A_local.numel() != sp.n_local:
+        raise ValueError(f"local slab has {A_local.numel()} elements, expected {sp.n_local}")
+
+    def ev():
+        if phase_events is None or not A_local.is_cuda:
+            return None
+        e = torch.cuda.Event(enable_timing=True)
+        e.record()
+        return e
+
+    if not sp.moved:
+        out = work[1] if work is not None else torch.empty_like(A_local)
+        e0 = ev()
+        fn(sp.local_extents, sp.perm, A_local, out)
+        if phase_events is not None and e0 is not None:
+            phase_events.append(("local", e0, ev()))
+        return out
+    send = work[0] if work is not None else torch.empty_like(A_local)
+    recv = work[1] if work is not None else torch.empty_like(A_local)
+    e0 = ev()
+    fn(sp.local_extents, sp.perm, A_local, send)
+    e1 = ev()
+    dist.all_to_all_single(recv, send, group=group)
+    e2 = ev()
+    out = send  # the send buffer is free again: fold into it
+    fn(sp.fold_extents, [0, 2, 1], recv, out)
+    if phase_events is not None and e0 is not None:
+        phase_events += [("local", e0, e1), ("alltoall", e1, e2), ("fold", e2, ev())]
+    return out
