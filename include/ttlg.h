@@ -88,8 +88,8 @@ typedef struct {
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
   int32_t variant;                       /* kernel variant bits (tests / calibration):
-                                            1 = register-staged instead of cp.async
-                                            pipeline, 2 = no streaming cache hints       */
+                                            1 = single-buffered staging (no cp.async
+                                            pipelining), 2 = no streaming cache hints    */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -111,7 +111,10 @@ typedef struct {
   double predicted_seconds;               /* performance-model prediction                */
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
-  int32_t kernel;                         /* 0 direct, 1 register-staged, 2 cp.async pipe */
+  int32_t kernel;                         /* 0 direct (FML/COPY), 1 staged cp.async pipe  */
+  int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
+  int32_t num_features;                   /* model feature vector (§V features, B200)    */
+  double features[8];
 } ttlg_plan_info;
 
 void ttlg_plan_hints_init(ttlg_plan_hints *hints);
@@ -151,6 +154,16 @@ ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,
                               const int32_t *perm, double *seconds);
 
 ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info);
+
+/* Every candidate the planner scores for this problem (Alg. 3's enumeration),
+ * with its model features and predicted time -- for calibration (§V) and
+ * measure-mode / model-regret studies.  Writes up to max_out entries to out and
+ * the number written to *n_out.  Any candidate can be executed by passing its
+ * schema / in_dim / tile_extents[in_dim] / out_dim / tile_extents[perm[out_dim]]
+ * as hints to ttlg_plan_ex. */
+ttlg_status ttlg_plan_candidates(ttlg_dtype dt, int rank, const int64_t *extents,
+                                 const int32_t *perm, const ttlg_plan_hints *hints,
+                                 ttlg_plan_info *out, int32_t max_out, int32_t *n_out);
 
 const char *ttlg_status_string(ttlg_status s);
 const char *ttlg_schema_name(int schema);

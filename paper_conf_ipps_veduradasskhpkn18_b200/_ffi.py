@@ -23,7 +23,7 @@ STATUS = {0: "TTLG_OK", 1: "TTLG_ERR_INVALID_VALUE", 2: "TTLG_ERR_ALIASING",
 EXPORTS = ["ttlg_plan", "ttlg_plan_ex", "ttlg_plan_hints_init", "ttlg_execute",
            "ttlg_plan_destroy", "ttlg_transpose", "ttlg_execute_host", "ttlg_predict_time",
            "ttlg_plan_describe", "ttlg_status_string", "ttlg_schema_name", "ttlg_version",
-           "ttlg_model_source"]
+           "ttlg_model_source", "ttlg_plan_candidates"]
 
 
 class TtlgError(RuntimeError):
@@ -53,7 +53,9 @@ class PlanInfo(ctypes.Structure):
                 ("grid", ctypes.c_int32), ("threads", ctypes.c_int32),
                 ("smem_bytes", ctypes.c_int32), ("bytes", ctypes.c_int64),
                 ("predicted_seconds", ctypes.c_double), ("candidates", ctypes.c_int32),
-                ("param_bytes", ctypes.c_int32), ("kernel", ctypes.c_int32)]
+                ("param_bytes", ctypes.c_int32), ("kernel", ctypes.c_int32),
+                ("occupancy", ctypes.c_int32), ("num_features", ctypes.c_int32),
+                ("features", ctypes.c_double * 8)]
 
     def to_dict(self) -> dict:
         d = self.fused_rank
@@ -71,7 +73,9 @@ class PlanInfo(ctypes.Structure):
             "grid": self.grid, "threads": self.threads, "smem_bytes": self.smem_bytes,
             "bytes": self.bytes, "predicted_seconds": self.predicted_seconds,
             "candidates": self.candidates, "param_bytes": self.param_bytes,
-            "kernel": ["direct", "staged", "pipe"][self.kernel],
+            "kernel": ["direct", "pipe"][self.kernel],
+            "occupancy": self.occupancy,
+            "features": [float(x) for x in self.features[:self.num_features]],
         }
 
 
@@ -99,6 +103,9 @@ def _load():
         "ttlg_schema_name": ([ctypes.c_int], ctypes.c_char_p),
         "ttlg_version": ([], ctypes.c_int),
         "ttlg_model_source": ([], ctypes.c_char_p),
+        "ttlg_plan_candidates": ([ctypes.c_int, ctypes.c_int, i64p, i32p, ctypes.POINTER(PlanHints),
+                                  ctypes.POINTER(PlanInfo), ctypes.c_int32,
+                                  ctypes.POINTER(ctypes.c_int32)], ctypes.c_int),
     }
     for name, (args, res) in sig.items():
         f = getattr(lib, name)

@@ -127,6 +127,32 @@ def predict_time(dtype, extents, perm) -> float:
     return out.value
 
 
+def plan_candidates(dtype, extents, perm, max_out: int = 4096, **hints) -> list:
+    """Every candidate slice/schema the planner scores (Alg. 3 enumeration) with its
+    model features and predicted seconds (for calibration / regret studies)."""
+    ext, pr = arrays(extents, perm)
+    out = (PlanInfo * max_out)()
+    n = ctypes.c_int32()
+    hh = make_hints(**hints) if hints else None
+    check(lib.ttlg_plan_candidates(_dtype_code(dtype), len(extents), ext, pr,
+                                   ctypes.byref(hh) if hh is not None else None, out, max_out,
+                                   ctypes.byref(n)), "ttlg_plan_candidates")
+    res = []
+    for i in range(n.value):
+        d = out[i].to_dict()
+        d["hints"] = candidate_hints(d)
+        res.append(d)
+    return res
+
+
+def candidate_hints(d: dict) -> dict:
+    """Hints that reproduce a candidate returned by plan_candidates()."""
+    a, b = d["in_dim"], d["out_dim"]
+    return {"schema": d["schema"] if d["schema"] != "COPY" else "FML", "in_dim": a,
+            "in_block": d["tile_extents"][a], "out_dim": b,
+            "out_block": d["tile_extents"][d["fused_perm"][b]]}
+
+
 def model_source() -> str:
     return lib.ttlg_model_source().decode()
 

@@ -217,6 +217,18 @@ ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,
   return TTLG_OK;
 }
 
+ttlg_status ttlg_plan_candidates(ttlg_dtype dt, int rank, const int64_t *extents,
+                                 const int32_t *perm, const ttlg_plan_hints *hints,
+                                 ttlg_plan_info *out, int32_t max_out, int32_t *n_out) {
+  if (!out || !n_out || max_out < 0) return TTLG_ERR_INVALID_VALUE;
+  ttlg_plan_s p;
+  CandidateSink sink{out, max_out, 0};
+  ttlg_status st = make_plan(&p, dt, rank, extents, perm, hints,
+                             device_profile(current_device()), &sink);
+  *n_out = sink.n;
+  return st;
+}
+
 ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info) {
   if (!plan || !info) return TTLG_ERR_INVALID_VALUE;
   *info = plan->info;

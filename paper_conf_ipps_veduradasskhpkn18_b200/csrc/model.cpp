@@ -24,22 +24,28 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   const double W = mi.W;
   const double tiles = (double)mi.num_tiles;
   const double fill = mi.fillA;
-  double read_bytes, write_bytes, runs;
+  double read_bytes, write_bytes, rows, slots;
+  auto group = [](double L) { return L >= 32 ? 32.0 : std::pow(2.0, std::ceil(std::log2(L))); };
   if (mi.kind == KK_DIRECT) {
     read_bytes = tiles * fill * run_cost(mi.V * W);
-    runs = tiles * fill * (1.0 + mi.RB);
+    rows = tiles * fill * mi.RB;
+    slots = 0.0;
   } else {
     read_bytes = tiles * fill * mi.RA * run_cost(mi.LA * W);
-    runs = tiles * fill * (mi.RA + mi.RB);
+    rows = tiles * fill * (mi.RA + mi.RB);
+    const double gA = group(mi.LA), gB = group(mi.LB);
+    // idle lane slots of the warp-row mapping (the paper's "Cycles" feature,
+    // L1336-1353, counted per lane group instead of per 32x32 tile)
+    slots = tiles * (mi.RA * (std::ceil(mi.LA / gA) * gA - mi.LA) +
+                     mi.RB * (std::ceil(mi.LB / gB) * gB - mi.LB));
   }
   write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
   const double bw = dev.hbm_gbs * 1e9;
-  // bytes in flight: each CTA keeps up to UNROLL*threads access elements of
-  // loads outstanding (Little's law with the loaded-DRAM latency)
-  const double unroll = (mi.kind == KK_DIRECT) ? kModelUnrollDirect : kModelUnrollStaged;
-  // the cp.async pipeline keeps a whole tile of loads in flight per CTA
+  // bytes in flight (Little's law with the loaded-DRAM latency): the cp.async
+  // pipeline keeps a whole tile of loads in flight per CTA; the direct kernel
+  // UNROLL access elements per thread
   const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
-                                              : std::min<double>(mi.V, unroll * mi.threads);
+                                              : std::min<double>(mi.V, kModelUnrollDirect * mi.threads);
   const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = dev.sms * inflight / kModelLatency;
   const double bw_eff = std::min(bw, bw_lat);
@@ -48,7 +54,8 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   F.f[0] = 1.0;
   F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
   F.f[2] = tiles_per_cta / std::max(1, mi.occ);
-  F.f[3] = runs / dev.sms;
+  F.f[3] = slots / dev.sms;
+  F.f[4] = rows / dev.sms;
   return F;
 }
 

@@ -26,7 +26,7 @@ struct ModelInput {
 };
 
 struct ModelFeatures {
-  double f[8];
+  double f[8];  // see model.cpp
 };
 
 // Feature vector (units: seconds at the reference bandwidth, or counts).

@@ -4,12 +4,11 @@
 #pragma once
 
 namespace ttlg {
-constexpr int kModelNumFeatures = 4;
+constexpr int kModelNumFeatures = 5;
 constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
-constexpr double kModelUnrollStaged = 8.0;   // loads in flight per thread (staged)
 constexpr double kModelUnrollDirect = 8.0;   // loads in flight per thread (direct)
-// features: [launch, memory-time, tiles-per-CTA/occ, runs-per-SM]
-constexpr double kCoefDirect[kModelNumFeatures] = {2.5e-6, 1.0, 0.10e-6, 0.2e-9};
-constexpr double kCoefStaged[kModelNumFeatures] = {2.5e-6, 1.0, 0.25e-6, 0.2e-9};
+// features: [launch, memory-time, tiles-per-CTA/occ, idle-lane-slots/SM, rows/SM]
+constexpr double kCoefDirect[kModelNumFeatures] = {2.5e-6, 1.0, 0.15e-6, 0.0, 0.3e-9};
+constexpr double kCoefStaged[kModelNumFeatures] = {2.5e-6, 1.0, 0.30e-6, 0.05e-9, 0.3e-9};
 constexpr const char *kModelSource = "default (uncalibrated)";
 }  // namespace ttlg

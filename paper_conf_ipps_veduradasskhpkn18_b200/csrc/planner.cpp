@@ -180,7 +180,8 @@ int64_t ceil_div(int64_t x, int64_t y) { return (x + y - 1) / y; }
 }  // namespace
 
 // Fill TileParams for a tile; returns false if it violates a kernel limit.
-static bool build_params(const Problem &P, const Tile &T, int kind, int threads, TileParams &K) {
+static bool build_params(const Problem &P, const Tile &T, int kind, int threads, int nbuf,
+                         TileParams &K) {
   memset(&K, 0, sizeof(K));
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
@@ -308,7 +309,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.off_digB = take((int64_t)K.RA * 4);
     K.off_digA = take((int64_t)K.RB * 4);
     K.off_data = take(smem_elems * P.W);
-    K.off_data2 = (kind == KK_PIPE) ? take(smem_elems * P.W) : K.off_data;
+    K.off_data2 = (nbuf == 2) ? take(smem_elems * P.W) : K.off_data;
   } else {
     K.off_tabB = take((int64_t)K.RB * 8);
     K.off_jcol = 0;
@@ -321,6 +322,13 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   K.dxA = threads % K.LA;
   K.drB = threads / K.LB;
   K.dxB = threads % K.LB;
+  auto lg = [](int64_t L) {
+    int l = 0;
+    while ((1 << l) < L && l < 5) l++;
+    return l;
+  };
+  K.lgA = lg(K.LA);
+  K.lgB = lg(K.LB);
   return true;
 }
 
@@ -362,9 +370,40 @@ static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forc
   return c;
 }
 
+static void fill_info(ttlg_plan_info &I, ttlg_dtype dt, int rank, const Problem &P,
+                      const Tile &T, const TileParams &K, const ModelInput &mi, int schema,
+                      int kind, double predicted, int ncand) {
+  memset(&I, 0, sizeof(I));
+  I.schema = schema;
+  I.dtype = dt;
+  I.rank = rank;
+  I.fused_rank = P.d;
+  for (int k = 0; k < P.d; k++) {
+    I.fused_extents[k] = P.n[k];
+    I.fused_perm[k] = P.p[k];
+    I.tile_extents[k] = T.t[k];
+  }
+  I.access_bytes = P.W;
+  I.in_dim = T.a;
+  I.out_dim = T.b;
+  I.in_run = K.LA;
+  I.out_run = K.LB;
+  I.tile_volume = K.V;
+  I.num_tiles = K.num_tiles;
+  I.grid = mi.grid;
+  I.threads = mi.threads;
+  I.smem_bytes = K.smem_bytes;
+  I.bytes = 2 * mi.N * P.W;
+  I.predicted_seconds = predicted;
+  I.candidates = ncand;
+  I.param_bytes = (int32_t)sizeof(TileParams);
+  I.kernel = kind;
+  I.occupancy = mi.occ;
+}
+
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints,
-                      const DeviceProfile &dev) {
+                      const DeviceProfile &dev, CandidateSink *sink) {
   ttlg_status st = validate(dt, rank, ext, perm);
   if (st != TTLG_OK) return st;
   const int s = (dt == TTLG_F64) ? 8 : 4;
@@ -397,6 +436,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   double best_t = 1e300;
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
+  const int nbuf = (hints && (hints->variant & 1)) ? 1 : 2;
 
   auto consider = [&](int kind, int a, int64_t ta, int b, int64_t tb) {
     if (hints) {
@@ -417,7 +457,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (kind != KK_DIRECT && V * P.W > max_tile_bytes) return;
     if (kind == KK_DIRECT && V * P.W > 256 * 1024) return;
     TileParams K;
-    if (!build_params(P, T, kind, threads, K)) return;
+    if (!build_params(P, T, kind, threads, nbuf, K)) return;
     if (K.smem_bytes > dev.smem_per_block_optin) return;
     ModelInput mi;
     mi.kind = kind;
@@ -440,6 +480,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.fillA = (double)N / ((double)K.num_tiles * K.V);
     const double tm = predict_seconds(mi, dev);
     ncand++;
+    if (sink && sink->n < sink->max) {
+      ttlg_plan_info &ci = sink->out[sink->n++];
+      fill_info(ci, dt, rank, P, T, K, mi, schema, kind, tm, 0);
+      const ModelFeatures F = model_features(mi, dev);
+      ci.num_features = kModelFeatureCount;
+      for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
+    }
     if (tm < best_t) {
       best_t = tm;
       best_mi = mi;
@@ -466,7 +513,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (pre * P.W >= 256 * 1024 && !(hints && hints->in_dim > a)) break;
     }
   }
-  const int staged_kind = (hints && (hints->variant & 1)) ? KK_STAGED : KK_PIPE;
+  const int staged_kind = KK_PIPE;
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
@@ -497,32 +544,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->grid = best_mi.grid;
   plan->nbytes = N * P.W;
   plan->kp = bestK;
-  ttlg_plan_info &I = plan->info;
-  memset(&I, 0, sizeof(I));
-  I.schema = best_schema;
-  I.dtype = dt;
-  I.rank = rank;
-  I.fused_rank = P.d;
-  for (int k = 0; k < P.d; k++) {
-    I.fused_extents[k] = P.n[k];
-    I.fused_perm[k] = P.p[k];
-    I.tile_extents[k] = bestT.t[k];
+  fill_info(plan->info, dt, rank, P, bestT, bestK, best_mi, best_schema, best_kind, best_t, ncand);
+  {
+    const ModelFeatures F = model_features(best_mi, dev);
+    plan->info.num_features = kModelFeatureCount;
+    for (int f = 0; f < kModelFeatureCount; f++) plan->info.features[f] = F.f[f];
   }
-  I.access_bytes = P.W;
-  I.in_dim = bestT.a;
-  I.out_dim = bestT.b;
-  I.in_run = bestK.LA;
-  I.out_run = bestK.LB;
-  I.tile_volume = bestK.V;
-  I.num_tiles = bestK.num_tiles;
-  I.grid = plan->grid;
-  I.threads = threads;
-  I.smem_bytes = bestK.smem_bytes;
-  I.bytes = 2 * N * P.W;
-  I.predicted_seconds = best_t;
-  I.candidates = ncand;
-  I.param_bytes = (int32_t)sizeof(TileParams);
-  I.kernel = best_kind;
   return TTLG_OK;
 }
 

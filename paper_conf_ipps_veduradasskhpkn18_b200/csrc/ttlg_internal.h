@@ -45,9 +45,8 @@ inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
 // Kernel kinds.
 enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
-  KK_STAGED = 1,  // OD / OA / FMS: slice staged through shared memory (register loads)
-  KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered staging (default)
-  KK_NUM = 3,
+  KK_PIPE = 1,    // OD / OA / FMS: slice staged through shared memory with cp.async
+  KK_NUM = 2,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -96,6 +95,7 @@ struct TileParams {
   int32_t smem_elems;      // data tile elements incl. padding
   int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
+  int32_t lgA, lgB;            // log2 of the lane-group size owning one A-row / B-row
 };
 
 struct Problem {
@@ -124,7 +124,7 @@ struct ttlg_plan_s {
   int W;       // access bytes
   int threads;
   int grid;
-  int variant;  // hint bits: 1 = register-staged kernel, 2 = no streaming cache hints
+  int variant;  // hint bits: 1 = single-buffered staging, 2 = no streaming cache hints
   int64_t nbytes;  // N * s
   ttlg::TileParams kp;
   ttlg_plan_info info;
@@ -137,10 +137,18 @@ struct ttlg_plan_s {
 };
 
 namespace ttlg {
+// collects every scored candidate (ttlg_plan_candidates: calibration, regret studies)
+struct CandidateSink {
+  ttlg_plan_info *out;
+  int max;
+  int n;
+};
+constexpr int kModelFeatureCount = 5;
 // planner.cpp
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
-                      const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev);
+                      const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev,
+                      CandidateSink *sink = nullptr);
 // api.cpp
 const DeviceProfile &device_profile(int device);
 // kernels.cu

@@ -1,0 +1,114 @@
+#!/usr/bin/env python
+"""Calibration / measure-mode sweep (§V "DataSet" L1298-1313 and
+"Model" L1402-1419, re-done on B200): for each case, enumerate the planner's
+candidates (ttlg_plan_candidates), execute up to --max-cand of them and record
+(features, predicted, measured) per candidate as JSON lines.
+
+  python tools/calib_sweep.py --group c2 --max-cand 40 > calib_c2.jsonl
+  python tools/calib_sweep.py --recipe 60 --seed 1   (random A17-recipe cases)
+"""
+from __future__ import annotations
+
+import argparse
+import itertools
+import json
+import os
+import random
+import statistics
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def recipe_cases(n, seed, lo_mb=32, hi_mb=512):
+    """Paper dataset recipe (L1298-1313): ranks 3-6, any permutation, five extent
+    orderings (equal, increasing, decreasing, up-down, down-up), volume range."""
+    from synth.configs import Case
+    rng = random.Random(seed)
+    out = []
+    for k in range(n):
+        d = rng.randint(3, 6)
+        eb = rng.choice([4, 8])
+        target = rng.uniform(lo_mb, hi_mb) * 2 ** 20 / eb
+        base = target ** (1.0 / d)
+        kind = rng.choice(["eq", "inc", "dec", "updown", "downup"])
+        f = [1.0] * d
+        for i in range(d):
+            t = i / max(1, d - 1)
+            f[i] = {"eq": 1.0, "inc": 0.5 + t, "dec": 1.5 - t,
+                    "updown": 0.6 + 0.8 * (1 - abs(2 * t - 1)),
+                    "downup": 0.6 + 0.8 * abs(2 * t - 1)}[kind]
+        g = (1.0 / (1e-9 + float(__import__("math").prod(f)))) ** (1.0 / d)
+        ext = [max(2, int(round(base * fi * g * rng.uniform(0.9, 1.1)))) for fi in f]
+        perm = list(range(d))
+        while perm == list(range(d)):
+            rng.shuffle(perm)
+        out.append(Case(8000 + k, tuple(ext), tuple(perm), eb, f"recipe-{kind}"))
+    return out
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--group", default=None)
+    ap.add_argument("--recipe", type=int, default=0)
+    ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--max-cand", type=int, default=40)
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--stride", type=int, default=1)
+    args = ap.parse_args()
+
+    import torch
+    import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
+    from synth import configs, gen_tensor_torch, case_seed
+
+    cases = []
+    if args.group:
+        cases += configs.all_configs()[args.group][::args.stride]
+    if args.recipe:
+        cases += recipe_cases(args.recipe, args.seed)
+    dev = torch.device("cuda:0")
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for c in cases:
+        dt = "f64" if c.elem_bytes == 8 else "f32"
+        cands = ttlg.plan_candidates(dt, c.extents, c.perm)
+        auto = ttlg.plan(dt, c.extents, c.perm).describe()
+        if len(cands) > args.max_cand:
+            # keep the model's best few plus an even spread over the rest
+            cands.sort(key=lambda d: d["predicted_seconds"])
+            step = len(cands) / args.max_cand
+            cands = [cands[int(i * step)] for i in range(args.max_cand)]
+        A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
+        B = torch.empty_like(A)
+        for cd in cands:
+            try:
+                p = ttlg.plan(dt, c.extents, c.perm, **cd["hints"])
+            except ttlg.TtlgError:
+                continue
+            info = p.describe()
+            for _ in range(2):
+                p.execute(A.data_ptr(), B.data_ptr(), stream.cuda_stream)
+            ts = []
+            for _ in range(args.reps):
+                e0.record()
+                p.execute(A.data_ptr(), B.data_ptr(), stream.cuda_stream)
+                e1.record()
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1) * 1e-3)
+            t = statistics.median(ts)
+            print(json.dumps({
+                "case": c.label(), "group": c.group, "bytes": c.alg_bytes, "W": info["access_bytes"],
+                "schema": info["schema"], "kernel": info["kernel"], "hints": cd["hints"],
+                "tile": info["tile_extents"], "LA": info["in_run"], "LB": info["out_run"],
+                "V": info["tile_volume"], "tiles": info["num_tiles"], "grid": info["grid"],
+                "occ": info["occupancy"], "features": info["features"],
+                "pred": info["predicted_seconds"], "meas": t, "gbs": c.alg_bytes / t / 1e9,
+                "is_auto": info["tile_extents"] == auto["tile_extents"]
+                and info["schema"] == auto["schema"]}), flush=True)
+        del A, B
+        torch.cuda.empty_cache()
+
+
+if __name__ == "__main__":
+    main()
