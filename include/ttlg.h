@@ -87,9 +87,7 @@ typedef struct {
   int32_t threads;                       /* 0 = auto; else threads per block             */
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
-  int32_t variant;                       /* kernel variant bits (tests / calibration):
-                                            1 = single-buffered staging (no cp.async
-                                            pipelining), 2 = no streaming cache hints    */
+  int32_t variant;                       /* reserved, must be 0                          */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */

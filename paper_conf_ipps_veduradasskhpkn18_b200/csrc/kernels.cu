@@ -67,15 +67,16 @@ __device__ __forceinline__ void st_stream(T *p, T v) {
     *p = v;
 }
 
-// cp.async (LDGSTS): global -> shared without a register round trip.
+// cp.async (LDGSTS): global -> shared without a register round trip.  No
+// "memory" clobber on the copy itself (ordering is enforced by commit/wait +
+// __syncthreads), so the compiler may keep addresses and table values in
+// registers across it.
 template <int W>
-__device__ __forceinline__ void cp_async(void *smem_ptr, const void *gptr) {
-  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem_ptr);
+__device__ __forceinline__ void cp_async(uint32_t s, const void *gptr) {
   if constexpr (W == 16)
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gptr) : "memory");
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gptr));
   else
-    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(s), "l"(gptr), "n"(W)
-                 : "memory");
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(s), "l"(gptr), "n"(W));
 }
 __device__ __forceinline__ void cp_async_commit() {
   asm volatile("cp.async.commit_group;\n" ::: "memory");
@@ -188,7 +189,9 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TilePara
 
 constexpr int kJReg = 8;  // register-resident column offsets per lane
 
-template <int W, bool CS, int S, bool JREG>
+// GA32 / GB32: the A-row / B-row lane group is a whole warp (runs >= 32
+// elements), so lane offsets along a row are compile-time immediates.
+template <int W, bool CS, int S, bool JREG, bool GA32, bool GB32>
 __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
@@ -220,11 +223,12 @@ __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams
 
   // lane groups: G = 2^lg lanes per row, 32/G rows per warp step
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int gA = 1 << P.lgA, gB = 1 << P.lgB;
-  const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> P.lgA) + (lane >> P.lgA);
-  const int rAstep = nw * (32 >> P.lgA);
-  const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> P.lgB) + (lane >> P.lgB);
-  const int rBstep = nw * (32 >> P.lgB);
+  const int lgA = GA32 ? 5 : P.lgA, lgB = GB32 ? 5 : P.lgB;
+  const int gA = 1 << lgA, gB = 1 << lgB;
+  const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> lgA) + (lane >> lgA);
+  const int rAstep = nw * (32 >> lgA);
+  const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
+  const int rBstep = nw * (32 >> lgB);
   int jc[JREG ? kJReg : 1];
   if constexpr (JREG) {
 #pragma unroll
@@ -234,66 +238,87 @@ __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams
     }
   }
 
-  auto issue = [&](const TileCtx &c, T *buf) {
+  const uint32_t s_buf0 = (uint32_t)__cvta_generic_to_shared(buf0);
+  const uint32_t s_buf1 = (uint32_t)__cvta_generic_to_shared(buf1);
+  const int RA = P.RA, RB = P.RB;
+#pragma unroll
+  for (int i = 0; i < (JREG ? kJReg : 1); i++) jc[i] *= W;  // byte offsets
+
+  // load phase of one tile: A-row r -> smem row, lanes of a group stride the run
+  auto issue = [&](const TileCtx &c, uint32_t sbuf) {
     const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
     const int lim = full ? P.LA : P.LAunit * c.limA;
     const T *Ab = A + c.bA;
-    for (int r = rA0; r < P.RA; r += rAstep) {
+    for (int r = rA0; r < RA; r += rAstep) {
       if (!full && digB[r] >= c.limB) continue;
       const int2 t = tabA[r];
-      const T *src = Ab + t.x;
-      T *dst = buf + t.y;
-      for (int x = xA0; x < lim; x += gA) cp_async<W>(dst + x, src + x);
-    }
-  };
-  auto drain = [&](const TileCtx &c, const T *buf) {
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? P.LB : P.LBunit * c.limB;
-    T *Bb = B + c.bB;
-    for (int r = rB0; r < P.RB; r += rBstep) {
-      if (!full && digA[r] >= c.limA) continue;
-      const int2 t = tabB[r];
-      T *dst = Bb + t.x;
-      const T *src = buf + t.y;
-      if constexpr (JREG) {
+      const T *src = Ab + t.x + xA0;
+      const uint32_t dst = sbuf + (uint32_t)(t.y + xA0) * W;
+      const int n = lim - xA0;  // this lane's span of the row
+      if constexpr (GA32) {
+        int x = 0;
+        for (; x + 96 < n; x += 128) {
 #pragma unroll
-        for (int i = 0; i < kJReg; i++) {
-          const int j = xB0 + i * gB;
-          if (j < lim) st_stream<CS>(dst + j, src[jc[i]]);
+          for (int u = 0; u < 4; u++) cp_async<W>(dst + (uint32_t)(x + 32 * u) * W, src + x + 32 * u);
         }
+        for (; x < n; x += 32) cp_async<W>(dst + (uint32_t)x * W, src + x);
       } else {
-#pragma unroll 4
-        for (int j = xB0; j < lim; j += gB) st_stream<CS>(dst + j, src[jcol[j]]);
+        for (int x = 0; x < n; x += gA) cp_async<W>(dst + (uint32_t)x * W, src + x);
       }
     }
   };
+  // store phase of one tile: B-row r <- smem through the column table
+  auto drain = [&](const TileCtx &c, const unsigned char *sbuf) {
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int lim = full ? P.LB : P.LBunit * c.limB;
+    T *Bb = B + c.bB;
+    for (int r = rB0; r < RB; r += rBstep) {
+      if (!full && digA[r] >= c.limA) continue;
+      const int2 t = tabB[r];
+      T *dst = Bb + t.x + xB0;
+      const unsigned char *src = sbuf + t.y * W;
+      if constexpr (JREG) {
+#pragma unroll
+        for (int i = 0; i < kJReg; i++) {
+          if (xB0 + i * gB < lim)
+            st_stream<CS>(dst + i * gB, *reinterpret_cast<const T *>(src + jc[i]));
+        }
+      } else {
+#pragma unroll 4
+        for (int j = xB0; j < lim; j += gB)
+          st_stream<CS>(dst + (j - xB0), *reinterpret_cast<const T *>(src + jcol[j] * W));
+      }
+    }
+  };
+  const unsigned char *g_buf0 = reinterpret_cast<const unsigned char *>(buf0);
+  const unsigned char *g_buf1 = reinterpret_cast<const unsigned char *>(buf1);
 
   uint32_t tile = blockIdx.x;
   if constexpr (S == 1) {
     for (; tile < P.num_tiles; tile += gridDim.x) {
       const TileCtx c = decode_tile(P, tile);
-      issue(c, buf0);
+      issue(c, s_buf0);
       cp_async_commit();
       cp_async_wait<0>();
       __syncthreads();
-      drain(c, buf0);
+      drain(c, g_buf0);
       __syncthreads();
     }
   } else {
     TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
-    if (tile < P.num_tiles) issue(cur, buf0);
+    if (tile < P.num_tiles) issue(cur, s_buf0);
     cp_async_commit();
     for (int k = 0; tile < P.num_tiles; k++) {
       const uint32_t next = tile + gridDim.x;
       TileCtx nx = cur;
       if (next < P.num_tiles) {
         nx = decode_tile(P, next);
-        issue(nx, (k & 1) ? buf0 : buf1);
+        issue(nx, (k & 1) ? s_buf0 : s_buf1);
       }
       cp_async_commit();
       cp_async_wait<1>();
       __syncthreads();
-      drain(cur, (k & 1) ? buf1 : buf0);
+      drain(cur, (k & 1) ? g_buf1 : g_buf0);
       __syncthreads();
       cur = nx;
       tile = next;
@@ -304,25 +329,25 @@ __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W, bool CS>
-static const void *kernel_ptr_w(int kind, bool jreg, int stages) {
-  if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, CS>;
-  if (stages == 1)
-    return jreg ? (const void *)k_pipe<W, CS, 1, true> : (const void *)k_pipe<W, CS, 1, false>;
-  return jreg ? (const void *)k_pipe<W, CS, 2, true> : (const void *)k_pipe<W, CS, 2, false>;
+template <int W>
+static const void *kernel_ptr_w(int kind, bool jreg, bool ga32, bool gb32) {
+  if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
+  // streaming cache hints on, double-buffered (S = 2)
+#define TTLG_K(J, A, B) (const void *)k_pipe<W, true, 2, J, A, B>
+  if (jreg) {
+    if (ga32) return gb32 ? TTLG_K(true, true, true) : TTLG_K(true, true, false);
+    return gb32 ? TTLG_K(true, false, true) : TTLG_K(true, false, false);
+  }
+  if (ga32) return gb32 ? TTLG_K(false, true, true) : TTLG_K(false, true, false);
+  return gb32 ? TTLG_K(false, false, true) : TTLG_K(false, false, false);
+#undef TTLG_K
 }
 
-static const void *kernel_ptr(int kind, int W, bool cs, bool jreg, int stages) {
+static const void *kernel_ptr(int kind, int W, bool jreg, bool ga32, bool gb32) {
   switch (W) {
-    case 4:
-      return cs ? kernel_ptr_w<4, true>(kind, jreg, stages)
-                : kernel_ptr_w<4, false>(kind, jreg, stages);
-    case 8:
-      return cs ? kernel_ptr_w<8, true>(kind, jreg, stages)
-                : kernel_ptr_w<8, false>(kind, jreg, stages);
-    case 16:
-      return cs ? kernel_ptr_w<16, true>(kind, jreg, stages)
-                : kernel_ptr_w<16, false>(kind, jreg, stages);
+    case 4: return kernel_ptr_w<4>(kind, jreg, ga32, gb32);
+    case 8: return kernel_ptr_w<8>(kind, jreg, ga32, gb32);
+    case 16: return kernel_ptr_w<16>(kind, jreg, ga32, gb32);
   }
   return nullptr;
 }
@@ -336,7 +361,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, true, true, 2)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, true, true, true)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -347,10 +372,8 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const bool cs = !(plan->variant & 2);
-  const int stages = (plan->variant & 1) ? 1 : 2;
   const bool jreg = plan->kp.LB <= kJReg * (1 << plan->kp.lgB);
-  const void *fn = kernel_ptr(plan->kind, plan->W, cs, jreg, stages);
+  const void *fn = kernel_ptr(plan->kind, plan->W, jreg, plan->kp.lgA == 5, plan->kp.lgB == 5);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

@@ -436,7 +436,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   double best_t = 1e300;
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
-  const int nbuf = (hints && (hints->variant & 1)) ? 1 : 2;
+  const int nbuf = 2;  // k_pipe is double-buffered
 
   auto consider = [&](int kind, int a, int64_t ta, int b, int64_t tb) {
     if (hints) {

@@ -124,7 +124,7 @@ struct ttlg_plan_s {
   int W;       // access bytes
   int threads;
   int grid;
-  int variant;  // hint bits: 1 = single-buffered staging, 2 = no streaming cache hints
+  int variant;  // reserved (hints->variant)
   int64_t nbytes;  // N * s
   ttlg::TileParams kp;
   ttlg_plan_info info;
