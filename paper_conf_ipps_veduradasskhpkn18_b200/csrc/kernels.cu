@@ -78,6 +78,33 @@ __device__ __forceinline__ void cp_async(uint32_t s, const void *gptr) {
   else
     asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(s), "l"(gptr), "n"(W));
 }
+// predicated forms (the predicate goes into the PTX guard, so predicated-off
+// lanes cost no branch / reconvergence)
+template <int W>
+__device__ __forceinline__ void cp_async_p(uint32_t s, const void *gptr, bool p) {
+  if constexpr (W == 16)
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n"
+                 " @q cp.async.cg.shared.global [%0], [%1], 16;\n}\n" ::"r"(s),
+                 "l"(gptr), "r"((int)p));
+  else
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n"
+                 " @q cp.async.ca.shared.global [%0], [%1], %3;\n}\n" ::"r"(s),
+                 "l"(gptr), "r"((int)p), "n"(W));
+}
+__device__ __forceinline__ void stcs_p(unsigned int *a, unsigned int v, bool p) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q st.global.cs.u32 [%0], %1;\n}\n"
+               ::"l"(a), "r"(v), "r"((int)p) : "memory");
+}
+__device__ __forceinline__ void stcs_p(uint2 *a, uint2 v, bool p) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n"
+               " @q st.global.cs.v2.u32 [%0], {%1, %2};\n}\n"
+               ::"l"(a), "r"(v.x), "r"(v.y), "r"((int)p) : "memory");
+}
+__device__ __forceinline__ void stcs_p(uint4 *a, uint4 v, bool p) {
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %5, 0;\n"
+               " @q st.global.cs.v4.u32 [%0], {%1, %2, %3, %4};\n}\n"
+               ::"l"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"((int)p) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() {
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
@@ -187,28 +214,67 @@ __global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TilePara
   }
 }
 
-constexpr int kJReg = 8;  // register-resident column offsets per lane
+// shared-memory helpers on 32-bit shared addresses (no generic->shared
+// conversion per access)
+__device__ __forceinline__ int2 lds_int2(uint32_t a) {
+  int2 v;
+  asm volatile("ld.shared.v2.s32 {%0, %1}, [%2];\n" : "=r"(v.x), "=r"(v.y) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ int lds_int(uint32_t a) {
+  int v;
+  asm volatile("ld.shared.s32 %0, [%1];\n" : "=r"(v) : "r"(a));
+  return v;
+}
+template <typename T>
+__device__ __forceinline__ T lds_T(uint32_t a);
+template <>
+__device__ __forceinline__ unsigned int lds_T<unsigned int>(uint32_t a) {
+  unsigned int v;
+  asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(v) : "r"(a));
+  return v;
+}
+template <>
+__device__ __forceinline__ uint2 lds_T<uint2>(uint32_t a) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(v.x), "=r"(v.y) : "r"(a));
+  return v;
+}
+template <>
+__device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "r"(a));
+  return v;
+}
 
-// GA32 / GB32: the A-row / B-row lane group is a whole warp (runs >= 32
-// elements), so lane offsets along a row are compile-time immediates.
-template <int W, bool CS, int S, bool JREG, bool GA32, bool GB32>
+// k_pipe template parameters:
+//   GA32 / GB32: the A-row / B-row lane group is a whole warp (run >= 32), so
+//                lane offsets along a row are compile-time immediates;
+//   NJ > 0:      every lane owns at most NJ output-run positions of a B-row
+//                (LB <= NJ * G_B) and keeps their shared-memory column offsets
+//                in registers; NJ = 0: column offsets read from the table.
+// Loop trip counts are warp-uniform and the bodies predicated, so no
+// divergence/reconvergence bookkeeping is generated in the hot loops.
+template <int W, int NJ, bool GA32, bool GB32>
 __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
   using T = typename Vec<W>::T;
   extern __shared__ __align__(16) unsigned char smem[];
-  int2 *tabA = reinterpret_cast<int2 *>(smem);
-  int2 *tabB = reinterpret_cast<int2 *>(smem + P.off_tabB);
-  int *jcol = reinterpret_cast<int *>(smem + P.off_jcol);
-  int *digB = reinterpret_cast<int *>(smem + P.off_digB);
-  int *digA = reinterpret_cast<int *>(smem + P.off_digA);
-  T *buf0 = reinterpret_cast<T *>(smem + P.off_data);
-  T *buf1 = reinterpret_cast<T *>(smem + P.off_data2);
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_buf0 = s0 + P.off_data, s_buf1 = s0 + P.off_data2;
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
-  build_rows(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk, tabA, digB);
-  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
+  build_rows(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk,
+             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB));
+  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA));
   for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
     int rem = j, s = 0;
     for (int k = 0; k < P.nj; k++) {
@@ -217,11 +283,10 @@ __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams
       s += (rem - cq * e) * P.j_sS[k];
       rem = cq;
     }
-    jcol[j] = s;
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
   }
   __syncthreads();
 
-  // lane groups: G = 2^lg lanes per row, 32/G rows per warp step
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
   const int lgA = GA32 ? 5 : P.lgA, lgB = GB32 ? 5 : P.lgB;
   const int gA = 1 << lgA, gB = 1 << lgB;
@@ -229,125 +294,117 @@ __global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams
   const int rAstep = nw * (32 >> lgA);
   const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
   const int rBstep = nw * (32 >> lgB);
-  int jc[JREG ? kJReg : 1];
-  if constexpr (JREG) {
+  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
+  const int kA = (LA + gA - 1) >> lgA;  // uniform per-row trip count (load)
+  const int kB = (LB + gB - 1) >> lgB;  // uniform per-row trip count (store)
+  int jc[NJ > 0 ? NJ : 1];
+  if constexpr (NJ > 0) {
 #pragma unroll
-    for (int i = 0; i < kJReg; i++) {
+    for (int i = 0; i < NJ; i++) {
       const int j = xB0 + i * gB;
-      jc[i] = j < P.LB ? jcol[j] : 0;
+      jc[i] = j < LB ? lds_int(s_jcol + 4 * j) : 0;
     }
   }
 
-  const uint32_t s_buf0 = (uint32_t)__cvta_generic_to_shared(buf0);
-  const uint32_t s_buf1 = (uint32_t)__cvta_generic_to_shared(buf1);
-  const int RA = P.RA, RB = P.RB;
-#pragma unroll
-  for (int i = 0; i < (JREG ? kJReg : 1); i++) jc[i] *= W;  // byte offsets
-
-  // load phase of one tile: A-row r -> smem row, lanes of a group stride the run
+  // load phase of one tile: A-row r -> smem, cp.async, lanes stride the run
   auto issue = [&](const TileCtx &c, uint32_t sbuf) {
     const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? P.LA : P.LAunit * c.limA;
-    const T *Ab = A + c.bA;
+    const int lim = full ? LA : P.LAunit * c.limA;
+    const T *Ab = A + c.bA + xA0;
+    const uint32_t sb = sbuf + xA0 * W;
     for (int r = rA0; r < RA; r += rAstep) {
-      if (!full && digB[r] >= c.limB) continue;
-      const int2 t = tabA[r];
-      const T *src = Ab + t.x + xA0;
-      const uint32_t dst = sbuf + (uint32_t)(t.y + xA0) * W;
-      const int n = lim - xA0;  // this lane's span of the row
-      if constexpr (GA32) {
-        int x = 0;
-        for (; x + 96 < n; x += 128) {
-#pragma unroll
-          for (int u = 0; u < 4; u++) cp_async<W>(dst + (uint32_t)(x + 32 * u) * W, src + x + 32 * u);
-        }
-        for (; x < n; x += 32) cp_async<W>(dst + (uint32_t)x * W, src + x);
-      } else {
-        for (int x = 0; x < n; x += gA) cp_async<W>(dst + (uint32_t)x * W, src + x);
-      }
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
+      const T *src = Ab + t.x;
+      const uint32_t dst = sb + t.y * W;
+      for (int k = 0; k < kA; k++)
+        cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
     }
   };
-  // store phase of one tile: B-row r <- smem through the column table
-  auto drain = [&](const TileCtx &c, const unsigned char *sbuf) {
+  // store phase of one tile: B-row r <- smem through the column offsets
+  auto drain = [&](const TileCtx &c, uint32_t sbuf) {
     const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? P.LB : P.LBunit * c.limB;
-    T *Bb = B + c.bB;
+    const int lim = full ? LB : P.LBunit * c.limB;
+    T *Bb = B + c.bB + xB0;
     for (int r = rB0; r < RB; r += rBstep) {
-      if (!full && digA[r] >= c.limA) continue;
-      const int2 t = tabB[r];
-      T *dst = Bb + t.x + xB0;
-      const unsigned char *src = sbuf + t.y * W;
-      if constexpr (JREG) {
+      const int2 t = lds_int2(s_tabB + 8 * r);
+      const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
+      T *dst = Bb + t.x;
+      const uint32_t src = sbuf + t.y * W;
+      if constexpr (NJ > 0) {
 #pragma unroll
-        for (int i = 0; i < kJReg; i++) {
-          if (xB0 + i * gB < lim)
-            st_stream<CS>(dst + i * gB, *reinterpret_cast<const T *>(src + jc[i]));
+        for (int i = 0; i < NJ; i++) {
+          if (i < kB)
+            stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
         }
       } else {
 #pragma unroll 4
-        for (int j = xB0; j < lim; j += gB)
-          st_stream<CS>(dst + (j - xB0), *reinterpret_cast<const T *>(src + jcol[j] * W));
+        for (int i = 0; i < kB; i++) {
+          const int j = xB0 + (i << lgB);
+          const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+          stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+        }
       }
     }
   };
-  const unsigned char *g_buf0 = reinterpret_cast<const unsigned char *>(buf0);
-  const unsigned char *g_buf1 = reinterpret_cast<const unsigned char *>(buf1);
 
   uint32_t tile = blockIdx.x;
-  if constexpr (S == 1) {
-    for (; tile < P.num_tiles; tile += gridDim.x) {
-      const TileCtx c = decode_tile(P, tile);
-      issue(c, s_buf0);
-      cp_async_commit();
-      cp_async_wait<0>();
-      __syncthreads();
-      drain(c, g_buf0);
-      __syncthreads();
+  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
+  if (tile < P.num_tiles) issue(cur, s_buf0);
+  cp_async_commit();
+  for (int k = 0; tile < P.num_tiles; k++) {
+    const uint32_t next = tile + gridDim.x;
+    TileCtx nx = cur;
+    if (next < P.num_tiles) {
+      nx = decode_tile(P, next);
+      issue(nx, (k & 1) ? s_buf0 : s_buf1);
     }
-  } else {
-    TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
-    if (tile < P.num_tiles) issue(cur, s_buf0);
     cp_async_commit();
-    for (int k = 0; tile < P.num_tiles; k++) {
-      const uint32_t next = tile + gridDim.x;
-      TileCtx nx = cur;
-      if (next < P.num_tiles) {
-        nx = decode_tile(P, next);
-        issue(nx, (k & 1) ? s_buf0 : s_buf1);
-      }
-      cp_async_commit();
-      cp_async_wait<1>();
-      __syncthreads();
-      drain(cur, (k & 1) ? g_buf1 : g_buf0);
-      __syncthreads();
-      cur = nx;
-      tile = next;
-    }
-    cp_async_wait<0>();
+    cp_async_wait<1>();
+    __syncthreads();
+    drain(cur, (k & 1) ? s_buf1 : s_buf0);
+    __syncthreads();
+    cur = nx;
+    tile = next;
   }
+  cp_async_wait<0>();
 }
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W>
-static const void *kernel_ptr_w(int kind, bool jreg, bool ga32, bool gb32) {
-  if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
-  // streaming cache hints on, double-buffered (S = 2)
-#define TTLG_K(J, A, B) (const void *)k_pipe<W, true, 2, J, A, B>
-  if (jreg) {
-    if (ga32) return gb32 ? TTLG_K(true, true, true) : TTLG_K(true, true, false);
-    return gb32 ? TTLG_K(true, false, true) : TTLG_K(true, false, false);
+template <int W, bool GA32>
+static const void *kernel_ptr_g(int nj, bool gb32) {
+  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false>;  // LB < 32: one slot
+  switch (nj) {
+    case 1: return (const void *)k_pipe<W, 1, GA32, true>;
+    case 2: return (const void *)k_pipe<W, 2, GA32, true>;
+    case 4: return (const void *)k_pipe<W, 4, GA32, true>;
+    case 8: return (const void *)k_pipe<W, 8, GA32, true>;
+    case 16: return (const void *)k_pipe<W, 16, GA32, true>;
   }
-  if (ga32) return gb32 ? TTLG_K(false, true, true) : TTLG_K(false, true, false);
-  return gb32 ? TTLG_K(false, false, true) : TTLG_K(false, false, false);
-#undef TTLG_K
+  return (const void *)k_pipe<W, 0, GA32, true>;
 }
 
-static const void *kernel_ptr(int kind, int W, bool jreg, bool ga32, bool gb32) {
+template <int W>
+static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32) {
+  if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
+  return ga32 ? kernel_ptr_g<W, true>(nj, gb32) : kernel_ptr_g<W, false>(nj, gb32);
+}
+
+// register column slots needed for a B-row: ceil(LB / G_B) rounded up to a power of two
+static int nj_of(const TileParams &K) {
+  const int g = 1 << K.lgB;
+  const int k = (K.LB + g - 1) / g;
+  int nj = 1;
+  while (nj < k) nj <<= 1;
+  return nj <= 16 ? nj : 0;
+}
+
+static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, jreg, ga32, gb32);
-    case 8: return kernel_ptr_w<8>(kind, jreg, ga32, gb32);
-    case 16: return kernel_ptr_w<16>(kind, jreg, ga32, gb32);
+    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32);
+    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32);
+    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32);
   }
   return nullptr;
 }
@@ -361,7 +418,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, true, true, true)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, true, true)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -372,8 +429,8 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const bool jreg = plan->kp.LB <= kJReg * (1 << plan->kp.lgB);
-  const void *fn = kernel_ptr(plan->kind, plan->W, jreg, plan->kp.lgA == 5, plan->kp.lgB == 5);
+  const void *fn = kernel_ptr(plan->kind, plan->W, nj_of(plan->kp), plan->kp.lgA == 5,
+                              plan->kp.lgB == 5);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {
