@@ -168,7 +168,7 @@ __device__ __forceinline__ void build_rows(int R, int nr, const int32_t *ext, co
 }
 
 template <int W, int U, bool CS>
-__global__ void __launch_bounds__(256) k_direct(const __grid_constant__ TileParams P,
+__global__ void __launch_bounds__(1024) k_direct(const __grid_constant__ TileParams P,
                                                 const void *__restrict__ Av,
                                                 void *__restrict__ Bv) {
   using T = typename Vec<W>::T;
@@ -258,7 +258,7 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
 // Loop trip counts are warp-uniform and the bodies predicated, so no
 // divergence/reconvergence bookkeeping is generated in the hot loops.
 template <int W, int NJ, bool GA32, bool GB32>
-__global__ void __launch_bounds__(256) k_pipe(const __grid_constant__ TileParams P,
+__global__ void __launch_bounds__(1024) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
   using T = typename Vec<W>::T;

@@ -345,7 +345,11 @@ static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) 
 // `pre` access elements (Alg. 3 enumerates limits in steps of WS and blocks the
 // slowest dim of the group; reading R12 enumerates block factors
 // directly, including the balanced ceil(n/ceil(n/t)) variants).
-static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forced) {
+static const int64_t kRunTargets[] = {64, 128, 256, 512, 1024, 2048, 4096, 0};
+static const int64_t kTileTargets[] = {4096, 8192, 16384, 32768, 65536, 131072, 0};
+
+static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forced,
+                       const int64_t *targets) {
   int c = 0;
   if (forced > 0) {
     if (forced > n) return 0;
@@ -360,8 +364,8 @@ static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forc
     out[c++] = t;
   };
   add(n);
-  static const int64_t targets[] = {64, 128, 256, 512, 1024, 2048};
-  for (int64_t R : targets) {
+  for (int i = 0; targets[i]; i++) {
+    const int64_t R = targets[i];
     int64_t t = ceil_div(R, pre * W);
     if (t >= n) continue;
     add(t);
@@ -502,7 +506,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // ---- direct (FML / COPY): input run = dims 0..a (contiguous), output run = dim 0
     int64_t pre = 1;
     for (int a = 0; a < P.d; a++) {
-      const int nb = cand_blocks(P.n[a], pre, P.W, blocksA, hints ? hints->in_block : 0);
+      const int nb = cand_blocks(P.n[a], pre, P.W, blocksA, hints ? hints->in_block : 0,
+                                 kTileTargets);
       for (int i = 0; i < nb; i++) {
         const int64_t ta = blocksA[i];
         if (pre * ta * P.W < 1024 && ta < P.n[a] && !(hints && hints->in_block))
@@ -518,11 +523,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
     for (int a = 0; a < P.d; a++) {
-      const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0);
+      const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0,
+                                  kRunTargets);
       int64_t preB = 1;
       for (int b = 0; b < P.d; b++) {
         const int pb = P.p[b];
-        const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0);
+        const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0,
+                                    kRunTargets);
         for (int i = 0; i < nbA; i++) {
           for (int j = 0; j < nbB; j++) {
             consider(staged_kind, a, blocksA[i], b, blocksB[j]);

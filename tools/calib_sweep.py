@@ -56,6 +56,7 @@ def main():
     ap.add_argument("--max-cand", type=int, default=40)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--stride", type=int, default=1)
+    ap.add_argument("--threads", default="", help="comma list of block sizes to try per candidate")
     args = ap.parse_args()
 
     import torch
@@ -81,9 +82,13 @@ def main():
             cands = [cands[int(i * step)] for i in range(args.max_cand)]
         A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
         B = torch.empty_like(A)
-        for cd in cands:
+        thr = [int(x) for x in args.threads.split(",") if x] or [0]
+        for cd, th in [(cd, th) for cd in cands for th in thr]:
+            h = dict(cd["hints"])
+            if th:
+                h["threads"] = th
             try:
-                p = ttlg.plan(dt, c.extents, c.perm, **cd["hints"])
+                p = ttlg.plan(dt, c.extents, c.perm, **h)
             except ttlg.TtlgError:
                 continue
             info = p.describe()
@@ -99,7 +104,8 @@ def main():
             t = statistics.median(ts)
             print(json.dumps({
                 "case": c.label(), "group": c.group, "bytes": c.alg_bytes, "W": info["access_bytes"],
-                "schema": info["schema"], "kernel": info["kernel"], "hints": cd["hints"],
+                "schema": info["schema"], "kernel": info["kernel"], "hints": h,
+                "threads": info["threads"],
                 "tile": info["tile_extents"], "LA": info["in_run"], "LB": info["out_run"],
                 "V": info["tile_volume"], "tiles": info["num_tiles"], "grid": info["grid"],
                 "occ": info["occupancy"], "features": info["features"],
