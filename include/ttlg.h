@@ -109,7 +109,7 @@ typedef struct {
   double predicted_seconds;               /* performance-model prediction                */
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
-  int32_t kernel;                         /* 0 direct (FML/COPY), 1 staged cp.async pipe  */
+  int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile (OD/OA/FMS)  */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[8];

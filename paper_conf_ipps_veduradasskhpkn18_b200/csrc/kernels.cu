@@ -8,27 +8,26 @@
 //            written straight to their output row (output run = the matching
 //            FVI, dim 0).  No shared memory for data, only the row table.
 //
-//  k_pipe    (OD / OA / FMS; Alg. 2, Alg. 4/5 L868-1020, Alg. 6
+//  k_tile    (OD / OA / FMS; Alg. 2, Alg. 4/5 L868-1020, Alg. 6
 //            L1022-1107): the tile (the paper's "slice") is the union of an
 //            input-prefix group and an output-prefix group.  Load phase: A-rows
-//            of LA contiguous elements are copied global -> shared with
-//            cp.async (LDGSTS), one tile ahead into the other of two buffers
-//            (S = 2), so a whole tile of loads is in flight while the previous
-//            tile is written out.  Store phase: B-rows of LB contiguous elements
-//            are read from shared memory through the column table and stored
-//            coalesced.  Rows are processed warp-wise: a warp (or a
-//            power-of-two lane group of G <= 32 lanes when the run is short)
-//            owns a row, so the row table lookup is a broadcast and the column
-//            offsets are register-resident (JREG) -- the B200 form of the
-//            paper's "compile-time constant indexing" (L1138-1155).
-//            The shared-memory layout pads every output-only dim so that output
+//            of LA contiguous elements are read coalesced (8 loads in flight per
+//            thread) and stored to shared memory; store phase: B-rows of LB
+//            contiguous elements are read from shared memory through the column
+//            offsets and written coalesced.  Rows are processed warp-wise: a
+//            warp (or a power-of-two lane group of G <= 32 lanes when the run is
+//            short) owns a row, so the row-table lookup is a broadcast and the
+//            column offsets are register-resident -- the B200 form of the
+//            paper's compile-time-constant indexing (L1138-1155).  The
+//            shared-memory layout pads every output-only dim so that output
 //            position j lands in bank j mod (128/W): conflict-free column reads
 //            (generalising the 32x33 pad, L747-749, and FMS's pad, L1104-1107).
 //
-// Both are persistent: grid = min(tiles, SMs x resident CTAs); every CTA builds
-// its row tables once in shared memory (the paper's texture-mapped offset
-// arrays, L737-745) and then strides over tiles, decoding each tile index with
-// fast-divmod (the paper's decode/compute_base, L725-737).
+// Grids: one CTA per tile (or a few consecutive tiles, `tpc`), many CTAs per
+// SM -- the skeleton that reaches the D2D copy rate on B200
+// (tools/copybench.cu).  Every CTA builds its row tables in shared memory
+// (the paper's texture-mapped offset arrays, L737-745) and decodes its tile
+// index with fast-divmod (the paper's decode/compute_base, L725-737).
 #include <cuda_runtime.h>
 
 #include <mutex>
@@ -168,7 +167,7 @@ __device__ __forceinline__ void build_rows(int R, int nr, const int32_t *ext, co
 }
 
 template <int W, int U, bool CS>
-__global__ void __launch_bounds__(1024) k_direct(const __grid_constant__ TileParams P,
+__global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TileParams P,
                                                 const void *__restrict__ Av,
                                                 void *__restrict__ Bv) {
   using T = typename Vec<W>::T;
@@ -183,7 +182,9 @@ __global__ void __launch_bounds__(1024) k_direct(const __grid_constant__ TilePar
 
   const int NT = blockDim.x, tid = threadIdx.x;
   const int r0 = tid / P.LB, j0 = tid % P.LB;
-  for (uint32_t tile = blockIdx.x; tile < P.num_tiles; tile += gridDim.x) {
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
+    if (tile >= P.num_tiles) break;
     const TileCtx c = decode_tile(P, tile);
     const int lim = P.LAunit * c.limA;  // the blocked dim a is the tile's outermost
     const T *Ab = A + c.bA;
@@ -249,24 +250,27 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
   return v;
 }
 
-// k_pipe template parameters:
-//   GA32 / GB32: the A-row / B-row lane group is a whole warp (run >= 32), so
-//                lane offsets along a row are compile-time immediates;
-//   NJ > 0:      every lane owns at most NJ output-run positions of a B-row
-//                (LB <= NJ * G_B) and keeps their shared-memory column offsets
-//                in registers; NJ = 0: column offsets read from the table.
-// Loop trip counts are warp-uniform and the bodies predicated, so no
-// divergence/reconvergence bookkeeping is generated in the hot loops.
-template <int W, int NJ, bool GA32, bool GB32>
-__global__ void __launch_bounds__(1024) k_pipe(const __grid_constant__ TileParams P,
+// k_tile template parameters (all warp-uniform, chosen at launch from the plan):
+//   KA: A-row elements per lane (ceil(LA / G_A), rounded up to a power of two);
+//       KA > 1 implies the lane group is the whole warp (G_A = 32).
+//   NJ: B-row elements per lane (ceil(LB / G_B) rounded up); NJ > 1 implies
+//       G_B = 32; NJ = 0: long output runs, column offsets read from the table.
+// Load phase: each thread loads up to 8 elements (RU = 8/KA rows x KA) into
+// registers before storing them to shared memory -- 8 independent loads in
+// flight per thread (the unrolled-copy skeleton that reaches the D2D rate on
+// B200; cp.async staging measured ~10% slower, tools/copybench.cu).
+template <int W, int KA, int NJ>
+__global__ void __launch_bounds__(512) k_tile(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
   using T = typename Vec<W>::T;
+  constexpr int RU = 8 / KA;  // A-rows per load batch
   extern __shared__ __align__(16) unsigned char smem[];
   const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
   const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
   const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
-  const uint32_t s_buf0 = s0 + P.off_data, s_buf1 = s0 + P.off_data2;
+  const uint32_t s_buf = s0 + P.off_data;
+  T *sdata = reinterpret_cast<T *>(smem + P.off_data);
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
@@ -288,15 +292,14 @@ __global__ void __launch_bounds__(1024) k_pipe(const __grid_constant__ TileParam
   __syncthreads();
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int lgA = GA32 ? 5 : P.lgA, lgB = GB32 ? 5 : P.lgB;
+  const int lgA = KA > 1 ? 5 : P.lgA, lgB = NJ != 1 ? 5 : P.lgB;
   const int gA = 1 << lgA, gB = 1 << lgB;
   const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> lgA) + (lane >> lgA);
   const int rAstep = nw * (32 >> lgA);
   const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
   const int rBstep = nw * (32 >> lgB);
   const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
-  const int kA = (LA + gA - 1) >> lgA;  // uniform per-row trip count (load)
-  const int kB = (LB + gB - 1) >> lgB;  // uniform per-row trip count (store)
+  const int kB = (LB + gB - 1) >> lgB;
   int jc[NJ > 0 ? NJ : 1];
   if constexpr (NJ > 0) {
 #pragma unroll
@@ -306,105 +309,116 @@ __global__ void __launch_bounds__(1024) k_pipe(const __grid_constant__ TileParam
     }
   }
 
-  // load phase of one tile: A-row r -> smem, cp.async, lanes stride the run
-  auto issue = [&](const TileCtx &c, uint32_t sbuf) {
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
+    if (tile >= P.num_tiles) break;
+    const TileCtx c = decode_tile(P, tile);
     const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? LA : P.LAunit * c.limA;
-    const T *Ab = A + c.bA + xA0;
-    const uint32_t sb = sbuf + xA0 * W;
-    for (int r = rA0; r < RA; r += rAstep) {
-      const int2 t = lds_int2(s_tabA + 8 * r);
-      const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
-      const T *src = Ab + t.x;
-      const uint32_t dst = sb + t.y * W;
-      for (int k = 0; k < kA; k++)
-        cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
-    }
-  };
-  // store phase of one tile: B-row r <- smem through the column offsets
-  auto drain = [&](const TileCtx &c, uint32_t sbuf) {
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? LB : P.LBunit * c.limB;
-    T *Bb = B + c.bB + xB0;
-    for (int r = rB0; r < RB; r += rBstep) {
-      const int2 t = lds_int2(s_tabB + 8 * r);
-      const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
-      T *dst = Bb + t.x;
-      const uint32_t src = sbuf + t.y * W;
-      if constexpr (NJ > 0) {
+    if (it > 0) __syncthreads();  // previous tile's reads of smem are done
+    // ---- load phase: global -> registers -> shared (8 loads in flight per thread)
+    {
+      const int lim = full ? LA : P.LAunit * c.limA;
+      const T *Ab = A + c.bA + xA0;
+      for (int r0 = rA0; r0 < RA; r0 += RU * rAstep) {
+        T v[RU][KA];
+        uint32_t so[RU];
+        bool ok[RU][KA];
 #pragma unroll
-        for (int i = 0; i < NJ; i++) {
-          if (i < kB)
-            stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+        for (int u = 0; u < RU; u++) {
+          const int r = r0 + u * rAstep;
+          const bool rin = r < RA;
+          const int2 t = rin ? lds_int2(s_tabA + 8 * r) : make_int2(0, 0);
+          const bool rok = rin && (full || lds_int(s_digB + 4 * r) < c.limB);
+          so[u] = (uint32_t)(t.y + xA0);
+          const T *src = Ab + t.x;
+#pragma unroll
+          for (int k = 0; k < KA; k++) {
+            ok[u][k] = rok && xA0 + (k << lgA) < lim;
+            if (ok[u][k]) v[u][k] = ld_stream<true>(src + (k << lgA));
+          }
         }
-      } else {
+#pragma unroll
+        for (int u = 0; u < RU; u++)
+#pragma unroll
+          for (int k = 0; k < KA; k++)
+            if (ok[u][k]) sdata[so[u] + (k << lgA)] = v[u][k];
+      }
+    }
+    __syncthreads();
+    // ---- store phase: shared -> coalesced B-row writes
+    {
+      const int lim = full ? LB : P.LBunit * c.limB;
+      T *Bb = B + c.bB + xB0;
+      for (int r = rB0; r < RB; r += rBstep) {
+        const int2 t = lds_int2(s_tabB + 8 * r);
+        const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
+        T *dst = Bb + t.x;
+        const uint32_t src = s_buf + t.y * W;
+        if constexpr (NJ > 0) {
+#pragma unroll
+          for (int i = 0; i < NJ; i++) {
+            if (i < kB)
+              stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+          }
+        } else {
 #pragma unroll 4
-        for (int i = 0; i < kB; i++) {
-          const int j = xB0 + (i << lgB);
-          const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-          stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+          for (int i = 0; i < kB; i++) {
+            const int j = xB0 + (i << lgB);
+            const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+            stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+          }
         }
       }
     }
-  };
-
-  uint32_t tile = blockIdx.x;
-  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
-  if (tile < P.num_tiles) issue(cur, s_buf0);
-  cp_async_commit();
-  for (int k = 0; tile < P.num_tiles; k++) {
-    const uint32_t next = tile + gridDim.x;
-    TileCtx nx = cur;
-    if (next < P.num_tiles) {
-      nx = decode_tile(P, next);
-      issue(nx, (k & 1) ? s_buf0 : s_buf1);
-    }
-    cp_async_commit();
-    cp_async_wait<1>();
-    __syncthreads();
-    drain(cur, (k & 1) ? s_buf1 : s_buf0);
-    __syncthreads();
-    cur = nx;
-    tile = next;
   }
-  cp_async_wait<0>();
 }
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W, bool GA32>
-static const void *kernel_ptr_g(int nj, bool gb32) {
-  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false>;  // LB < 32: one slot
+template <int W, int KA>
+static const void *kernel_ptr_ka(int nj) {
   switch (nj) {
-    case 1: return (const void *)k_pipe<W, 1, GA32, true>;
-    case 2: return (const void *)k_pipe<W, 2, GA32, true>;
-    case 4: return (const void *)k_pipe<W, 4, GA32, true>;
-    case 8: return (const void *)k_pipe<W, 8, GA32, true>;
-    case 16: return (const void *)k_pipe<W, 16, GA32, true>;
+    case 1: return (const void *)k_tile<W, KA, 1>;
+    case 2: return (const void *)k_tile<W, KA, 2>;
+    case 4: return (const void *)k_tile<W, KA, 4>;
+    case 8: return (const void *)k_tile<W, KA, 8>;
+    case 16: return (const void *)k_tile<W, KA, 16>;
   }
-  return (const void *)k_pipe<W, 0, GA32, true>;
+  return (const void *)k_tile<W, KA, 0>;
 }
 
 template <int W>
-static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr_w(int kind, int ka, int nj) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
-  return ga32 ? kernel_ptr_g<W, true>(nj, gb32) : kernel_ptr_g<W, false>(nj, gb32);
+  switch (ka) {
+    case 1: return kernel_ptr_ka<W, 1>(nj);
+    case 2: return kernel_ptr_ka<W, 2>(nj);
+    case 4: return kernel_ptr_ka<W, 4>(nj);
+  }
+  return kernel_ptr_ka<W, 8>(nj);
 }
 
-// register column slots needed for a B-row: ceil(LB / G_B) rounded up to a power of two
+static int pow2_at_least(int k) {
+  int p = 1;
+  while (p < k) p <<= 1;
+  return p;
+}
+
+// per-lane elements of an A-row (KA, <= 8) and of a B-row (NJ, 0 = table path)
+static int ka_of(const TileParams &K) {
+  const int k = pow2_at_least((K.LA + (1 << K.lgA) - 1) >> K.lgA);
+  return k <= 8 ? k : 8;
+}
 static int nj_of(const TileParams &K) {
-  const int g = 1 << K.lgB;
-  const int k = (K.LB + g - 1) / g;
-  int nj = 1;
-  while (nj < k) nj <<= 1;
-  return nj <= 16 ? nj : 0;
+  const int k = pow2_at_least((K.LB + (1 << K.lgB) - 1) >> K.lgB);
+  return k <= 16 ? k : 0;
 }
 
-static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr(int kind, int W, int ka, int nj) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32);
-    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32);
-    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32);
+    case 4: return kernel_ptr_w<4>(kind, ka, nj);
+    case 8: return kernel_ptr_w<8>(kind, ka, nj);
+    case 16: return kernel_ptr_w<16>(kind, ka, nj);
   }
   return nullptr;
 }
@@ -418,7 +432,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, true, true)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, 4)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -429,8 +443,7 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W, nj_of(plan->kp), plan->kp.lgA == 5,
-                              plan->kp.lgB == 5);
+  const void *fn = kernel_ptr(plan->kind, plan->W, ka_of(plan->kp), nj_of(plan->kp));
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

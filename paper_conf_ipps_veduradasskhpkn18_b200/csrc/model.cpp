@@ -41,16 +41,17 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   }
   write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
   const double bw = dev.hbm_gbs * 1e9;
-  // bytes in flight (Little's law with the loaded-DRAM latency): the cp.async
-  // pipeline keeps a whole tile of loads in flight per CTA; the direct kernel
-  // UNROLL access elements per thread
-  const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
-                                              : std::min<double>(mi.V, kModelUnrollDirect * mi.threads);
+  // bytes in flight (Little's law with the loaded-DRAM latency): both kernels
+  // keep up to 8 access elements per thread of loads outstanding
+  const double per_cta = std::min<double>(mi.V, kModelUnrollDirect * mi.threads);
   const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = dev.sms * inflight / kModelLatency;
   const double bw_eff = std::min(bw, bw_lat);
-  const double tiles_per_cta = std::ceil(tiles / mi.grid);
-  const double wave = tiles_per_cta / (tiles / mi.grid);
+  // wave quantisation of the grid over the resident CTA slots
+  const double slots_chip = (double)dev.sms * std::max(1, mi.occ);
+  const double waves = (double)mi.grid / slots_chip;
+  const double wave = std::ceil(waves) / waves;
+  const double tiles_per_cta = std::ceil(tiles / mi.grid) * std::ceil(waves);
   F.f[0] = 1.0;
   F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
   F.f[2] = tiles_per_cta / std::max(1, mi.occ);

@@ -440,7 +440,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   double best_t = 1e300;
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
-  const int nbuf = 2;  // k_pipe is double-buffered
+  const int nbuf = 1;  // k_tile stages one tile at a time; many CTAs per SM overlap
 
   auto consider = [&](int kind, int a, int64_t ta, int b, int64_t tb) {
     if (hints) {
@@ -478,8 +478,15 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.smem_bytes = K.smem_bytes;
     mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
     if (mi.occ < 1) return;
-    mi.grid = (int)std::min<int64_t>(K.num_tiles, (int64_t)dev.sms * mi.occ);
-    if (hints && hints->grid > 0) mi.grid = hints->grid;
+    // tiles per CTA: 1 while there are >= 4 waves of tiles, else amortise the
+    // per-CTA table build over up to 4 consecutive tiles
+    {
+      const int64_t slots = (int64_t)dev.sms * mi.occ;
+      int tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, K.num_tiles / (8 * slots)));
+      if (hints && hints->grid > 0) tpc = (int)ceil_div(K.num_tiles, hints->grid);
+      K.tpc = tpc;
+      mi.grid = (int)ceil_div(K.num_tiles, tpc);
+    }
     // effective run lengths averaged over partial tiles
     mi.fillA = (double)N / ((double)K.num_tiles * K.V);
     const double tm = predict_seconds(mi, dev);
@@ -518,7 +525,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (pre * P.W >= 256 * 1024 && !(hints && hints->in_dim > a)) break;
     }
   }
-  const int staged_kind = KK_PIPE;
+  const int staged_kind = KK_TILE;
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;

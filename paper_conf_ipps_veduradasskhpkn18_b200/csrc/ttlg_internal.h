@@ -45,7 +45,7 @@ inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
 // Kernel kinds.
 enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
-  KK_PIPE = 1,    // OD / OA / FMS: slice staged through shared memory with cp.async
+  KK_TILE = 1,    // OD / OA / FMS: slice staged through shared memory (k_tile)
   KK_NUM = 2,
 };
 
@@ -96,6 +96,7 @@ struct TileParams {
   int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
   int32_t lgA, lgB;            // log2 of the lane-group size owning one A-row / B-row
+  int32_t tpc;                 // tiles per CTA (consecutive tile indices)
 };
 
 struct Problem {
