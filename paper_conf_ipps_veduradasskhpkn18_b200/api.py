@@ -148,9 +148,12 @@ def plan_candidates(dtype, extents, perm, max_out: int = 4096, **hints) -> list:
 def candidate_hints(d: dict) -> dict:
     """Hints that reproduce a candidate returned by plan_candidates()."""
     a, b = d["in_dim"], d["out_dim"]
-    return {"schema": d["schema"] if d["schema"] != "COPY" else "FML", "in_dim": a,
-            "in_block": d["tile_extents"][a], "out_dim": b,
-            "out_block": d["tile_extents"][d["fused_perm"][b]]}
+    h = {"schema": d["schema"] if d["schema"] != "COPY" else "FML", "in_dim": a,
+         "in_block": d["tile_extents"][a], "out_dim": b,
+         "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
+    if d["kernel"] != "direct":
+        h["variant"] = 1 if d["kernel"] == "tile" else 2
+    return h
 
 
 def model_source() -> str:

@@ -250,6 +250,128 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
   return v;
 }
 
+// k_pipe template parameters:
+//   GA32 / GB32: the A-row / B-row lane group is a whole warp (run >= 32), so
+//                lane offsets along a row are compile-time immediates;
+//   NJ > 0:      every lane owns at most NJ output-run positions of a B-row
+//                (LB <= NJ * G_B) and keeps their shared-memory column offsets
+//                in registers; NJ = 0: column offsets read from the table.
+// Loop trip counts are warp-uniform and the bodies predicated, so no
+// divergence/reconvergence bookkeeping is generated in the hot loops.
+template <int W, int NJ, bool GA32, bool GB32>
+__global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams P,
+                                              const void *__restrict__ Av,
+                                              void *__restrict__ Bv) {
+  using T = typename Vec<W>::T;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_buf0 = s0 + P.off_data, s_buf1 = s0 + P.off_data2;
+  const T *A = reinterpret_cast<const T *>(Av);
+  T *B = reinterpret_cast<T *>(Bv);
+
+  build_rows(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk,
+             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB));
+  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA));
+  for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
+    int rem = j, s = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const int e = P.j_ext[k];
+      const int cq = rem / e;
+      s += (rem - cq * e) * P.j_sS[k];
+      rem = cq;
+    }
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
+  }
+  __syncthreads();
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  const int lgA = GA32 ? 5 : P.lgA, lgB = GB32 ? 5 : P.lgB;
+  const int gA = 1 << lgA, gB = 1 << lgB;
+  const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> lgA) + (lane >> lgA);
+  const int rAstep = nw * (32 >> lgA);
+  const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
+  const int rBstep = nw * (32 >> lgB);
+  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
+  const int kA = (LA + gA - 1) >> lgA;  // uniform per-row trip count (load)
+  const int kB = (LB + gB - 1) >> lgB;  // uniform per-row trip count (store)
+  int jc[NJ > 0 ? NJ : 1];
+  if constexpr (NJ > 0) {
+#pragma unroll
+    for (int i = 0; i < NJ; i++) {
+      const int j = xB0 + i * gB;
+      jc[i] = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+    }
+  }
+
+  // load phase of one tile: A-row r -> smem, cp.async, lanes stride the run
+  auto issue = [&](const TileCtx &c, uint32_t sbuf) {
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int lim = full ? LA : P.LAunit * c.limA;
+    const T *Ab = A + c.bA + xA0;
+    const uint32_t sb = sbuf + xA0 * W;
+    for (int r = rA0; r < RA; r += rAstep) {
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
+      const T *src = Ab + t.x;
+      const uint32_t dst = sb + t.y * W;
+      for (int k = 0; k < kA; k++)
+        cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
+    }
+  };
+  // store phase of one tile: B-row r <- smem through the column offsets
+  auto drain = [&](const TileCtx &c, uint32_t sbuf) {
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int lim = full ? LB : P.LBunit * c.limB;
+    T *Bb = B + c.bB + xB0;
+    for (int r = rB0; r < RB; r += rBstep) {
+      const int2 t = lds_int2(s_tabB + 8 * r);
+      const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
+      T *dst = Bb + t.x;
+      const uint32_t src = sbuf + t.y * W;
+      if constexpr (NJ > 0) {
+#pragma unroll
+        for (int i = 0; i < NJ; i++) {
+          if (i < kB)
+            stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+        }
+      } else {
+#pragma unroll 4
+        for (int i = 0; i < kB; i++) {
+          const int j = xB0 + (i << lgB);
+          const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+          stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+        }
+      }
+    }
+  };
+
+  uint32_t tile = blockIdx.x;
+  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
+  if (tile < P.num_tiles) issue(cur, s_buf0);
+  cp_async_commit();
+  for (int k = 0; tile < P.num_tiles; k++) {
+    const uint32_t next = tile + gridDim.x;
+    TileCtx nx = cur;
+    if (next < P.num_tiles) {
+      nx = decode_tile(P, next);
+      issue(nx, (k & 1) ? s_buf0 : s_buf1);
+    }
+    cp_async_commit();
+    cp_async_wait<1>();
+    __syncthreads();
+    drain(cur, (k & 1) ? s_buf1 : s_buf0);
+    __syncthreads();
+    cur = nx;
+    tile = next;
+  }
+  cp_async_wait<0>();
+}
+
+
 // k_tile template parameters (all warp-uniform, chosen at launch from the plan):
 //   KA: A-row elements per lane (ceil(LA / G_A), rounded up to a power of two);
 //       KA > 1 implies the lane group is the whole warp (G_A = 32).
@@ -320,28 +442,36 @@ __global__ void __launch_bounds__(512) k_tile(const __grid_constant__ TileParams
       const int lim = full ? LA : P.LAunit * c.limA;
       const T *Ab = A + c.bA + xA0;
       for (int r0 = rA0; r0 < RA; r0 += RU * rAstep) {
-        T v[RU][KA];
+        const T *src[RU];
         uint32_t so[RU];
-        bool ok[RU][KA];
+        bool rok[RU];
 #pragma unroll
         for (int u = 0; u < RU; u++) {
           const int r = r0 + u * rAstep;
           const bool rin = r < RA;
           const int2 t = rin ? lds_int2(s_tabA + 8 * r) : make_int2(0, 0);
-          const bool rok = rin && (full || lds_int(s_digB + 4 * r) < c.limB);
+          rok[u] = rin && (full || lds_int(s_digB + 4 * r) < c.limB);
           so[u] = (uint32_t)(t.y + xA0);
-          const T *src = Ab + t.x;
-#pragma unroll
-          for (int k = 0; k < KA; k++) {
-            ok[u][k] = rok && xA0 + (k << lgA) < lim;
-            if (ok[u][k]) v[u][k] = ld_stream<true>(src + (k << lgA));
-          }
+          src[u] = Ab + t.x;
         }
+        // runs longer than KA * 32 elements take several uniform passes
+        for (int xb = 0; xb < lim; xb += KA << lgA) {
+          T v[RU][KA];
+          bool ok[RU][KA];
 #pragma unroll
-        for (int u = 0; u < RU; u++)
+          for (int u = 0; u < RU; u++) {
 #pragma unroll
-          for (int k = 0; k < KA; k++)
-            if (ok[u][k]) sdata[so[u] + (k << lgA)] = v[u][k];
+            for (int k = 0; k < KA; k++) {
+              ok[u][k] = rok[u] && xA0 + xb + (k << lgA) < lim;
+              if (ok[u][k]) v[u][k] = ld_stream<true>(src[u] + xb + (k << lgA));
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < RU; u++)
+#pragma unroll
+            for (int k = 0; k < KA; k++)
+              if (ok[u][k]) sdata[so[u] + xb + (k << lgA)] = v[u][k];
+        }
       }
     }
     __syncthreads();
@@ -387,9 +517,24 @@ static const void *kernel_ptr_ka(int nj) {
   return (const void *)k_tile<W, KA, 0>;
 }
 
+template <int W, bool GA32>
+static const void *kernel_ptr_pipe(int nj, bool gb32) {
+  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false>;  // LB < 32: one slot
+  switch (nj) {
+    case 1: return (const void *)k_pipe<W, 1, GA32, true>;
+    case 2: return (const void *)k_pipe<W, 2, GA32, true>;
+    case 4: return (const void *)k_pipe<W, 4, GA32, true>;
+    case 8: return (const void *)k_pipe<W, 8, GA32, true>;
+    case 16: return (const void *)k_pipe<W, 16, GA32, true>;
+  }
+  return (const void *)k_pipe<W, 0, GA32, true>;
+}
+
 template <int W>
-static const void *kernel_ptr_w(int kind, int ka, int nj) {
+static const void *kernel_ptr_w(int kind, int ka, int nj, bool ga32, bool gb32) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
+  if (kind == KK_PIPE)
+    return ga32 ? kernel_ptr_pipe<W, true>(nj, gb32) : kernel_ptr_pipe<W, false>(nj, gb32);
   switch (ka) {
     case 1: return kernel_ptr_ka<W, 1>(nj);
     case 2: return kernel_ptr_ka<W, 2>(nj);
@@ -414,11 +559,11 @@ static int nj_of(const TileParams &K) {
   return k <= 16 ? k : 0;
 }
 
-static const void *kernel_ptr(int kind, int W, int ka, int nj) {
+static const void *kernel_ptr(int kind, int W, int ka, int nj, bool ga32, bool gb32) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, ka, nj);
-    case 8: return kernel_ptr_w<8>(kind, ka, nj);
-    case 16: return kernel_ptr_w<16>(kind, ka, nj);
+    case 4: return kernel_ptr_w<4>(kind, ka, nj, ga32, gb32);
+    case 8: return kernel_ptr_w<8>(kind, ka, nj, ga32, gb32);
+    case 16: return kernel_ptr_w<16>(kind, ka, nj, ga32, gb32);
   }
   return nullptr;
 }
@@ -426,13 +571,13 @@ static const void *kernel_ptr(int kind, int W, int ka, int nj) {
 static int widx(int W) { return W == 4 ? 0 : (W == 8 ? 1 : 2); }
 
 int kernel_regs(int kind, int W) {
-  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}};
+  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
   static std::mutex mu;
   std::lock_guard<std::mutex> g(mu);
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, 4)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, 4, true, true)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -443,7 +588,8 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W, ka_of(plan->kp), nj_of(plan->kp));
+  const void *fn = kernel_ptr(plan->kind, plan->W, ka_of(plan->kp), nj_of(plan->kp),
+                              plan->kp.lgA == 5, plan->kp.lgB == 5);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

@@ -41,17 +41,19 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   }
   write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
   const double bw = dev.hbm_gbs * 1e9;
-  // bytes in flight (Little's law with the loaded-DRAM latency): both kernels
-  // keep up to 8 access elements per thread of loads outstanding
-  const double per_cta = std::min<double>(mi.V, kModelUnrollDirect * mi.threads);
+  // bytes in flight (Little's law with the loaded-DRAM latency): k_direct and
+  // k_tile keep up to 8 access elements per thread of loads outstanding, the
+  // cp.async pipeline of k_pipe a whole tile per CTA
+  const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
+                                              : std::min<double>(mi.V, kModelUnroll * mi.threads);
   const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = dev.sms * inflight / kModelLatency;
   const double bw_eff = std::min(bw, bw_lat);
-  // wave quantisation of the grid over the resident CTA slots
+  // wave quantisation: tiles handed out over the resident CTA slots
   const double slots_chip = (double)dev.sms * std::max(1, mi.occ);
-  const double waves = (double)mi.grid / slots_chip;
-  const double wave = std::ceil(waves) / waves;
-  const double tiles_per_cta = std::ceil(tiles / mi.grid) * std::ceil(waves);
+  const double steps = tiles / slots_chip;
+  const double wave = std::ceil(steps) / steps;
+  const double tiles_per_cta = std::ceil(steps);
   F.f[0] = 1.0;
   F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
   F.f[2] = tiles_per_cta / std::max(1, mi.occ);
@@ -62,7 +64,9 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
 
 double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
   const ModelFeatures F = model_features(mi, dev);
-  const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect : kCoefStaged;
+  const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect
+                    : (mi.kind == KK_TILE) ? kCoefTile
+                                           : kCoefPipe;
   double t = 0.0;
   for (int i = 0; i < kModelNumFeatures; i++) t += c[i] * F.f[i];
   // the model can never beat one pass of the algorithmic bytes at copy speed

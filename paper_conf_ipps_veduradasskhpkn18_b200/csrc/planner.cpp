@@ -423,8 +423,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   }
   widen(P, forceW);
 
-  const int threads = (hints && hints->threads) ? hints->threads : 256;
-  if (threads < 32 || threads > 1024 || threads % 32) return TTLG_ERR_INVALID_VALUE;
+  if (hints && hints->threads &&
+      (hints->threads < 64 || hints->threads > 512 || hints->threads % 32))
+    return TTLG_ERR_INVALID_VALUE;
   const int force_schema = hints ? hints->schema : TTLG_SCHEMA_AUTO;
 
   int64_t N = 1;
@@ -440,9 +441,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   double best_t = 1e300;
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
-  const int nbuf = 1;  // k_tile stages one tile at a time; many CTAs per SM overlap
 
-  auto consider = [&](int kind, int a, int64_t ta, int b, int64_t tb) {
+  auto consider1 = [&](int kind, int threads, int a, int64_t ta, int b, int64_t tb) {
+    const int nbuf = (kind == KK_PIPE) ? 2 : 1;
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -478,10 +479,15 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.smem_bytes = K.smem_bytes;
     mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
     if (mi.occ < 1) return;
-    // tiles per CTA: 1 while there are >= 4 waves of tiles, else amortise the
-    // per-CTA table build over up to 4 consecutive tiles
-    {
-      const int64_t slots = (int64_t)dev.sms * mi.occ;
+    const int64_t slots = (int64_t)dev.sms * mi.occ;
+    if (kind == KK_PIPE) {
+      // persistent: one CTA per resident slot, striding over the tiles
+      K.tpc = 1;
+      mi.grid = (int)std::min<int64_t>(K.num_tiles, slots);
+      if (hints && hints->grid > 0) mi.grid = hints->grid;
+    } else {
+      // tiles per CTA: 1 while there are >= 8 waves of tiles, else amortise the
+      // per-CTA table build over up to 4 consecutive tiles
       int tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, K.num_tiles / (8 * slots)));
       if (hints && hints->grid > 0) tpc = (int)ceil_div(K.num_tiles, hints->grid);
       K.tpc = tpc;
@@ -505,6 +511,21 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       bestT = T;
       best_kind = kind;
       best_schema = schema;
+    }
+  };
+
+  // kernel variants and block sizes competing for each slice candidate
+  const int hv = hints ? hints->variant : 0;
+  const int nthr = (hints && hints->threads) ? 1 : 2;
+  const int thr_list[2] = {(hints && hints->threads) ? hints->threads : 256, 512};
+  auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
+    for (int ti = 0; ti < nthr; ti++) {
+      if (group == KK_DIRECT) {
+        consider1(KK_DIRECT, thr_list[ti], a, ta, b, tb);
+      } else {
+        if (hv != 2) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
+        if (hv != 1) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
+      }
     }
   };
 
@@ -554,7 +575,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->kind = best_kind;
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
-  plan->threads = threads;
+  plan->threads = best_mi.threads;
   plan->grid = best_mi.grid;
   plan->nbytes = N * P.W;
   plan->kp = bestK;

@@ -45,8 +45,9 @@ inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
 // Kernel kinds.
 enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
-  KK_TILE = 1,    // OD / OA / FMS: slice staged through shared memory (k_tile)
-  KK_NUM = 2,
+  KK_TILE = 1,    // OD / OA / FMS: register-staged, one tile per CTA (k_tile)
+  KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered, persistent (k_pipe)
+  KK_NUM = 3,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel

@@ -105,7 +105,7 @@ def main():
             print(json.dumps({
                 "case": c.label(), "group": c.group, "bytes": c.alg_bytes, "W": info["access_bytes"],
                 "schema": info["schema"], "kernel": info["kernel"], "hints": h,
-                "threads": info["threads"],
+                "threads": info["threads"], "kernel_hint": h.get("variant", 0),
                 "tile": info["tile_extents"], "LA": info["in_run"], "LB": info["out_run"],
                 "V": info["tile_volume"], "tiles": info["num_tiles"], "grid": info["grid"],
                 "occ": info["occupancy"], "features": info["features"],
