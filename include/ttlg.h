@@ -113,7 +113,7 @@ typedef struct {
   int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe    */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
-  double features[8];
+  double features[12];
 } ttlg_plan_info;
 
 void ttlg_plan_hints_init(ttlg_plan_hints *hints);

@@ -55,7 +55,7 @@ class PlanInfo(ctypes.Structure):
                 ("predicted_seconds", ctypes.c_double), ("candidates", ctypes.c_int32),
                 ("param_bytes", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("occupancy", ctypes.c_int32), ("num_features", ctypes.c_int32),
-                ("features", ctypes.c_double * 8)]
+                ("features", ctypes.c_double * 12)]
 
     def to_dict(self) -> dict:
         d = self.fused_rank

@@ -24,22 +24,25 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   const double W = mi.W;
   const double tiles = (double)mi.num_tiles;
   const double fill = mi.fillA;
-  double read_bytes, write_bytes, rows, slots;
+  const double sms = dev.sms;
   auto group = [](double L) { return L >= 32 ? 32.0 : std::pow(2.0, std::ceil(std::log2(L))); };
+  double read_bytes, runsA, opsA;
   if (mi.kind == KK_DIRECT) {
     read_bytes = tiles * fill * run_cost(mi.V * W);
-    rows = tiles * fill * mi.RB;
-    slots = 0.0;
+    runsA = tiles * fill;
+    opsA = tiles * mi.V / 32.0;
   } else {
     read_bytes = tiles * fill * mi.RA * run_cost(mi.LA * W);
-    rows = tiles * fill * (mi.RA + mi.RB);
-    const double gA = group(mi.LA), gB = group(mi.LB);
-    // idle lane slots of the warp-row mapping (the paper's "Cycles" feature,
-    // L1336-1353, counted per lane group instead of per 32x32 tile)
-    slots = tiles * (mi.RA * (std::ceil(mi.LA / gA) * gA - mi.LA) +
-                     mi.RB * (std::ceil(mi.LB / gB) * gB - mi.LB));
+    runsA = tiles * fill * mi.RA;
+    const double gA = group(mi.LA);
+    opsA = tiles * mi.RA * std::ceil(mi.LA / gA) / (32.0 / gA);
   }
-  write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
+  const double write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
+  const double runsB = tiles * fill * mi.RB;
+  const double gB = group(mi.LB);
+  const double opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);
+  const double sector = read_bytes + write_bytes;
+  const double alg = 2.0 * mi.N * W;
   const double bw = dev.hbm_gbs * 1e9;
   // bytes in flight (Little's law with the loaded-DRAM latency): k_direct and
   // k_tile keep up to 8 access elements per thread of loads outstanding, the
@@ -47,18 +50,26 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
                                               : std::min<double>(mi.V, kModelUnroll * mi.threads);
   const double inflight = (double)mi.occ * per_cta * W;
-  const double bw_lat = dev.sms * inflight / kModelLatency;
-  const double bw_eff = std::min(bw, bw_lat);
+  const double bw_lat = sms * inflight / kModelLatency;
   // wave quantisation: tiles handed out over the resident CTA slots
-  const double slots_chip = (double)dev.sms * std::max(1, mi.occ);
-  const double steps = tiles / slots_chip;
+  const double slots = sms * std::max(1, mi.occ);
+  const double steps = tiles / slots;
   const double wave = std::ceil(steps) / steps;
-  const double tiles_per_cta = std::ceil(steps);
-  F.f[0] = 1.0;
-  F.f[1] = (read_bytes + write_bytes) / bw_eff * wave;
-  F.f[2] = tiles_per_cta / std::max(1, mi.occ);
-  F.f[3] = slots / dev.sms;
-  F.f[4] = rows / dev.sms;
+  // shared-memory wavefronts beyond the conflict-free ideal (the paper's bank
+  // conflicts of Orthogonal-Arbitrary, L1016-1020), per SM
+  const double conf = (mi.kind == KK_DIRECT)
+                          ? 0.0
+                          : (mi.N / 32.0) * (mi.conf_load + mi.conf_store - 2.0) / sms;
+  F.f[0] = 1.0;                                                // launch + fixed costs
+  F.f[1] = alg / bw;                                           // one pass at copy speed
+  F.f[2] = (sector - alg) / bw;                                // partial-sector waste
+  F.f[3] = (runsA + runsB) / sms;                              // DRAM runs per SM
+  F.f[4] = tiles / sms;                                        // tiles per SM
+  F.f[5] = std::max(0.0, sector / std::min(bw, bw_lat) - sector / bw);  // too few bytes in flight
+  F.f[6] = (wave - 1.0) * sector / bw;                         // tail wave
+  F.f[7] = std::ceil(steps);                                   // sequential tiles per CTA slot
+  F.f[8] = conf;                                               // extra smem wavefronts per SM
+  F.f[9] = (opsA + opsB) / sms;                                // warp-level row work per SM
   return F;
 }
 

@@ -23,10 +23,11 @@ struct ModelInput {
   int64_t num_tiles;
   int threads, smem_bytes, occ, grid;
   double fillA;  // useful fraction of the tile grid (partial tiles)
+  double conf_load, conf_store;  // smem wavefronts / ideal for one warp access (>= 1)
 };
 
 struct ModelFeatures {
-  double f[8];  // see model.cpp
+  double f[12];  // see model.cpp
 };
 
 // Feature vector (units: seconds at the reference bandwidth, or counts).

@@ -4,12 +4,12 @@
 #pragma once
 
 namespace ttlg {
-constexpr int kModelNumFeatures = 5;
+constexpr int kModelNumFeatures = 10;
 constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
 constexpr double kModelUnroll = 8.0;         // loads in flight per thread (k_direct, k_tile)
-// features: [launch, memory-time, tiles-per-CTA/occ, idle-lane-slots/SM, rows/SM]
-constexpr double kCoefDirect[kModelNumFeatures] = {2.5e-6, 1.0, 0.15e-6, 0.0, 0.3e-9};
-constexpr double kCoefTile[kModelNumFeatures] = {2.5e-6, 1.0, 0.30e-6, 0.05e-9, 0.3e-9};
-constexpr double kCoefPipe[kModelNumFeatures] = {2.5e-6, 1.0, 0.30e-6, 0.05e-9, 0.3e-9};
+// features: see model.cpp model_features()
+constexpr double kCoefDirect[kModelNumFeatures] = {5e-6, 1.0, 1.0, 0, 0, 0.1, 1.0, 1e-6, 0, 0};
+constexpr double kCoefTile[kModelNumFeatures] = {10e-6, 1.0, 0.3, 1e-9, 0, 0.2, 2.0, 2e-6, 1e-9, 0};
+constexpr double kCoefPipe[kModelNumFeatures] = {10e-6, 0.6, 0.3, 0.6e-9, 1e-8, 0, 1.5, 2e-6, 1e-9, 0};
 constexpr const char *kModelSource = "default (uncalibrated)";
 }  // namespace ttlg

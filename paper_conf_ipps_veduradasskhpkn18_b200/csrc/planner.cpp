@@ -332,6 +332,64 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   return true;
 }
 
+// Shared-memory wavefronts of one warp access relative to the conflict-free
+// ideal: lanes are split in phases of 128 bytes; a phase costs the largest
+// number of distinct 4-byte words that fall into one bank.  `addr` holds the
+// 32 lanes' element offsets.
+static double wavefront_ratio(const int64_t *addr, int W) {
+  const int per_phase = 128 / W, phases = 32 / per_phase;
+  int total = 0;
+  for (int ph = 0; ph < phases; ph++) {
+    int64_t words[32 * 4];
+    int nw = 0;
+    for (int l = ph * per_phase; l < (ph + 1) * per_phase; l++)
+      for (int w = 0; w < W / 4; w++) words[nw++] = addr[l] * (W / 4) + w;
+    int worst = 1;
+    for (int bank = 0; bank < 32; bank++) {
+      int64_t seen[32 * 4];
+      int ns = 0;
+      for (int i = 0; i < nw; i++) {
+        if (((words[i] % 32) + 32) % 32 != bank) continue;
+        bool dup = false;
+        for (int s = 0; s < ns; s++) dup |= seen[s] == words[i];
+        if (!dup) seen[ns++] = words[i];
+      }
+      if (ns > worst) worst = ns;
+    }
+    total += worst;
+  }
+  return (double)total / phases;
+}
+
+// conflict ratios of the first warp of the load (A-row) and store (B-row) phases
+static void smem_conflicts(const TileParams &K, int W, double &load, double &store) {
+  auto row_off = [](int r, int n, const int32_t *ext, const int32_t *sS) {
+    int64_t s = 0;
+    for (int k = 0; k < n; k++) {
+      s += (int64_t)(r % ext[k]) * sS[k];
+      r /= ext[k];
+    }
+    return s;
+  };
+  int64_t addr[32];
+  {
+    const int g = 1 << K.lgA;
+    for (int l = 0; l < 32; l++) {
+      const int r = std::min(l >> K.lgA, K.RA - 1), x = std::min(l & (g - 1), K.LA - 1);
+      addr[l] = row_off(r, K.nra, K.ra_ext, K.ra_sS) + x;
+    }
+    load = wavefront_ratio(addr, W);
+  }
+  {
+    const int g = 1 << K.lgB;
+    for (int l = 0; l < 32; l++) {
+      const int r = std::min(l >> K.lgB, K.RB - 1), j = std::min(l & (g - 1), K.LB - 1);
+      addr[l] = row_off(r, K.nrb, K.rb_ext, K.rb_sS) + row_off(j, K.nj, K.j_ext, K.j_sS);
+    }
+    store = wavefront_ratio(addr, W);
+  }
+}
+
 static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) {
   int occ = dev.max_threads_per_sm / threads;
   const int per = smem + 1024;  // 1 KB reserved per CTA
@@ -495,6 +553,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     // effective run lengths averaged over partial tiles
     mi.fillA = (double)N / ((double)K.num_tiles * K.V);
+    mi.conf_load = mi.conf_store = 1.0;
+    if (kind != KK_DIRECT) smem_conflicts(K, P.W, mi.conf_load, mi.conf_store);
     const double tm = predict_seconds(mi, dev);
     ncand++;
     if (sink && sink->n < sink->max) {

@@ -145,7 +145,7 @@ struct CandidateSink {
   int max;
   int n;
 };
-constexpr int kModelFeatureCount = 5;
+constexpr int kModelFeatureCount = 10;
 // planner.cpp
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
