@@ -140,10 +140,15 @@ ttlg_status ttlg_plan_destroy(ttlg_plan_t plan);
 ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, const int32_t *perm,
                            const void *A, void *B, void *stream);
 
-/* Host-buffer convenience (end-to-end path): copies A_host -> A_dev, executes,
- * copies B_dev -> B_host, all asynchronous on `stream`, with the copies split in
- * chunks where the plan allows so transfers overlap.  A_host/B_host should be
- * pinned for asynchrony; A_dev/B_dev are device scratch of N*s bytes each. */
+/* Host-buffer end-to-end path: A_host -> A_dev, transpose, B_dev -> B_host.
+ * B is split along its outermost output dimension into up to 32 chunks
+ * (>= 16 MiB each); chunk k's input slab is a strided 2-D region of A copied
+ * densely (cudaMemcpy2DAsync), transposed with a sub-plan, and its contiguous
+ * output range copied back -- H2D, kernels and D2H of successive chunks run on
+ * internal streams so both PCIe directions overlap.  Ordered after prior work
+ * on `stream`; `stream` waits for completion (no host sync).  A_host/B_host
+ * should be pinned; A_dev/B_dev are device scratch of N*s bytes each (A_dev's
+ * contents are chunk slabs afterwards, not A).  Small tensors: one stream. */
 ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
                               void *B_dev, void *stream);
 

@@ -4,6 +4,7 @@
 #include <stdlib.h>
 #include <string.h>
 
+#include <algorithm>
 #include <mutex>
 #include <new>
 
@@ -141,6 +142,112 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
   return st;
 }
 
+
+// ---- host-buffer pipeline (ttlg_execute_host) --------------------------------
+// B is split along its outermost output dim o_{d-1} = input dim q into C chunks.
+// Chunk k needs the A slab i_q in [q0, q0+cq): a 2-D strided region of A
+// (outer x (inner*cq) elements, pitch inner*n_q), copied densely with
+// cudaMemcpy2DAsync; its transposition is the same permutation on extents with
+// n_q -> cq, and its output is a contiguous range of B.  H2D, kernel and D2H of
+// successive chunks run on three internal streams joined by events, so the
+// host->device and device->host PCIe directions overlap.
+namespace {
+constexpr int kMaxChunks = 32;
+struct HostPipe {
+  cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
+  cudaEvent_t start = nullptr, done = nullptr, evA[kMaxChunks], evB[kMaxChunks];
+  bool ok = false;
+  std::mutex mu;
+};
+HostPipe g_pipes[16];
+
+HostPipe *host_pipe(int dev) {
+  if (dev < 0 || dev >= 16) return nullptr;
+  HostPipe &p = g_pipes[dev];
+  if (!p.ok) {
+    bool good = cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking) == cudaSuccess &&
+                cudaStreamCreateWithFlags(&p.comp, cudaStreamNonBlocking) == cudaSuccess &&
+                cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking) == cudaSuccess &&
+                cudaEventCreateWithFlags(&p.start, cudaEventDisableTiming) == cudaSuccess &&
+                cudaEventCreateWithFlags(&p.done, cudaEventDisableTiming) == cudaSuccess;
+    for (int i = 0; good && i < kMaxChunks; i++)
+      good = cudaEventCreateWithFlags(&p.evA[i], cudaEventDisableTiming) == cudaSuccess &&
+             cudaEventCreateWithFlags(&p.evB[i], cudaEventDisableTiming) == cudaSuccess;
+    if (!good) return nullptr;
+    p.ok = true;
+  }
+  return &p;
+}
+}  // namespace
+
+static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *B_host,
+                                void *A_dev, void *B_dev, cudaStream_t s) {
+  const int esize = p->dt == TTLG_F64 ? 8 : 4;
+  const int d = p->rank;
+  const int q = p->perm[d - 1];
+  int64_t inner = 1, outer = 1, N = 1;
+  for (int k = 0; k < d; k++) N *= p->ext[k];
+  for (int k = 0; k < q; k++) inner *= p->ext[k];
+  for (int k = q + 1; k < d; k++) outer *= p->ext[k];
+  const int64_t nq = p->ext[q];
+  const int64_t nbytes = N * esize;
+  int64_t C = std::min<int64_t>({nq, (int64_t)kMaxChunks, nbytes / (16ll << 20)});
+  if (p->device < 0) return TTLG_ERR_DEVICE;
+  HostPipe *hp = C >= 2 ? host_pipe(p->device) : nullptr;
+  if (!hp) {  // small or unsplittable: one stream, in order
+    if (cudaMemcpyAsync(A_dev, A_host, (size_t)nbytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      return TTLG_ERR_CUDA;
+    ttlg_status st = execute(p, A_dev, B_dev, s);
+    if (st != TTLG_OK) return st;
+    if (cudaMemcpyAsync(B_host, B_dev, (size_t)nbytes, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+      return TTLG_ERR_CUDA;
+    return TTLG_OK;
+  }
+  std::lock_guard<std::mutex> g(hp->mu);
+  const int64_t M = N / nq;  // B elements per index of its outermost dim
+  // at most two distinct chunk extents -> two sub-plans
+  const int64_t base = nq / C, rem = nq % C;
+  ttlg_plan_s sub[2];
+  int64_t subq[2] = {base, base + 1};
+  for (int v = 0; v < 2; v++) {
+    if (subq[v] == 0 || (v == 1 && rem == 0)) continue;
+    int64_t e[TTLG_MAXD];
+    for (int k = 0; k < d; k++) e[k] = p->ext[k];
+    e[q] = subq[v];
+    ttlg_status st = plan_into(&sub[v], (ttlg_dtype)p->dt, d, e, p->perm,
+                               p->has_hints ? &p->hints : nullptr);
+    if (st != TTLG_OK) return st;
+  }
+  if (cudaEventRecord(hp->start, s) != cudaSuccess) return TTLG_ERR_CUDA;
+  cudaStreamWaitEvent(hp->h2d, hp->start, 0);
+  cudaStreamWaitEvent(hp->comp, hp->start, 0);
+  cudaStreamWaitEvent(hp->d2h, hp->start, 0);
+  int64_t q0 = 0;
+  for (int64_t k = 0; k < C; k++) {
+    const int v = k < rem ? 1 : 0;
+    const int64_t cq = subq[v];
+    const size_t width = (size_t)(inner * cq * esize), spitch = (size_t)(inner * nq * esize);
+    unsigned char *a_slab = (unsigned char *)A_dev + q0 * inner * outer * esize;
+    unsigned char *b_chunk = (unsigned char *)B_dev + q0 * M * esize;
+    if (cudaMemcpy2DAsync(a_slab, width, (const unsigned char *)A_host + q0 * inner * esize, spitch,
+                          width, (size_t)outer, cudaMemcpyHostToDevice, hp->h2d) != cudaSuccess)
+      return TTLG_ERR_CUDA;
+    cudaEventRecord(hp->evA[k], hp->h2d);
+    cudaStreamWaitEvent(hp->comp, hp->evA[k], 0);
+    ttlg_status st = execute(&sub[v], a_slab, b_chunk, hp->comp);
+    if (st != TTLG_OK) return st;
+    cudaEventRecord(hp->evB[k], hp->comp);
+    cudaStreamWaitEvent(hp->d2h, hp->evB[k], 0);
+    if (cudaMemcpyAsync((unsigned char *)B_host + q0 * M * esize, b_chunk, (size_t)(cq * M * esize),
+                        cudaMemcpyDeviceToHost, hp->d2h) != cudaSuccess)
+      return TTLG_ERR_CUDA;
+    q0 += cq;
+  }
+  if (cudaEventRecord(hp->done, hp->d2h) != cudaSuccess) return TTLG_ERR_CUDA;
+  if (cudaStreamWaitEvent(s, hp->done, 0) != cudaSuccess) return TTLG_ERR_CUDA;
+  return TTLG_OK;
+}
+
 }  // namespace ttlg
 
 using namespace ttlg;
@@ -195,16 +302,7 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
 ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
                               void *B_dev, void *stream) {
   if (!plan || !A_host || !B_host || !A_dev || !B_dev) return TTLG_ERR_INVALID_VALUE;
-  cudaStream_t s = (cudaStream_t)stream;
-  if (cudaMemcpyAsync(A_dev, A_host, (size_t)plan->nbytes, cudaMemcpyHostToDevice, s) !=
-      cudaSuccess)
-    return TTLG_ERR_CUDA;
-  ttlg_status st = execute(plan, A_dev, B_dev, stream);
-  if (st != TTLG_OK) return st;
-  if (cudaMemcpyAsync(B_host, B_dev, (size_t)plan->nbytes, cudaMemcpyDeviceToHost, s) !=
-      cudaSuccess)
-    return TTLG_ERR_CUDA;
-  return TTLG_OK;
+  return execute_host(plan, A_host, B_host, A_dev, B_dev, (cudaStream_t)stream);
 }
 
 ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,

@@ -261,3 +261,24 @@ def test_full_exactly_once_index_encoding():
         exp = oracle.source_index(case.extents, case.perm, np.arange(n, dtype=np.int64))
         assert np.array_equal(got, exp), case.label()
         del A, B
+
+
+@pytest.mark.parametrize("ext,perm,eb", [([320, 320, 256], [2, 1, 0], 8),      # 25 chunks
+                                         ([64, 64, 64, 130], [3, 1, 0, 2], 4),  # q != d-1
+                                         ([40, 50, 60], [0, 2, 1], 8),          # small: 1 stream
+                                         ([33, 17, 2048, 9], [2, 3, 0, 1], 4)])
+def test_execute_host_pipeline(ext, perm, eb):
+    """ttlg_execute_host: chunked H2D / kernel / D2H over internal streams."""
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(77, n, eb, device="cpu").pin_memory()
+    B = torch.empty_like(A).pin_memory()
+    Ad = torch.empty(n, dtype=A.dtype, device=DEV)
+    Bd = torch.empty_like(Ad)
+    p = ttlg.plan(_dt(eb), ext, perm)
+    p.execute_host(A.data_ptr(), B.data_ptr(), Ad.data_ptr(), Bd.data_ptr(),
+                   torch.cuda.current_stream().cuda_stream)
+    torch.cuda.current_stream().synchronize()
+    iv = torch.int64 if eb == 8 else torch.int32
+    uv = np.uint64 if eb == 8 else np.uint32
+    _assert_equal(B.view(iv).numpy().view(uv),
+                  oracle.transpose(A.view(iv).numpy().view(uv), ext, perm), "execute_host")
