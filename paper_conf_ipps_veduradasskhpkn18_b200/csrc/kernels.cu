@@ -250,58 +250,6 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
   return v;
 }
 
-// Store phase shared by k_tile and k_pipe: B-row r <- shared memory through
-// the column offsets -> coalesced streaming stores.  With register column
-// offsets (NJ > 0) RBU = 8/NJ rows are processed per step so that up to eight
-// independent shared-memory loads per thread are in flight before their
-// global stores (the LDS -> STG latency otherwise dominates, ncu
-// short_scoreboard stalls).
-template <int W, int NJ>
-__device__ __forceinline__ void store_rows(typename Vec<W>::T *Bb, uint32_t sbuf, uint32_t s_tabB,
-                                           uint32_t s_digA, uint32_t s_jcol, const int *jc,
-                                           int rB0, int rBstep, int RB, int kB, int lgB, int xB0,
-                                           int lim, int LB, bool full, int limA) {
-  using T = typename Vec<W>::T;
-  if constexpr (NJ > 0) {
-    constexpr int RBU = NJ >= 8 ? 1 : 8 / NJ;
-    for (int r0 = rB0; r0 < RB; r0 += RBU * rBstep) {
-      int2 t[RBU];
-      bool rok[RBU];
-#pragma unroll
-      for (int u = 0; u < RBU; u++) {
-        const int r = r0 + u * rBstep;
-        const bool rin = r < RB;
-        t[u] = rin ? lds_int2(s_tabB + 8 * r) : make_int2(0, 0);
-        rok[u] = rin && (full || lds_int(s_digA + 4 * r) < limA);
-      }
-      T v[RBU][NJ];
-#pragma unroll
-      for (int u = 0; u < RBU; u++)
-#pragma unroll
-        for (int i = 0; i < NJ; i++) v[u][i] = lds_T<T>(sbuf + t[u].y * W + jc[i]);
-#pragma unroll
-      for (int u = 0; u < RBU; u++)
-#pragma unroll
-        for (int i = 0; i < NJ; i++)
-          if (i < kB)
-            stcs_p(Bb + t[u].x + (i << lgB), v[u][i], rok[u] && xB0 + (i << lgB) < lim);
-    }
-  } else {
-    for (int r = rB0; r < RB; r += rBstep) {
-      const int2 t = lds_int2(s_tabB + 8 * r);
-      const bool rok = full || lds_int(s_digA + 4 * r) < limA;
-      T *dst = Bb + t.x;
-      const uint32_t src = sbuf + t.y * W;
-#pragma unroll 4
-      for (int i = 0; i < kB; i++) {
-        const int j = xB0 + (i << lgB);
-        const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-        stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
-      }
-    }
-  }
-}
-
 // k_pipe template parameters:
 //   GA32 / GB32: the A-row / B-row lane group is a whole warp (run >= 32), so
 //                lane offsets along a row are compile-time immediates;
@@ -365,32 +313,40 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
     const int lim = full ? LA : P.LAunit * c.limA;
     const T *Ab = A + c.bA + xA0;
     const uint32_t sb = sbuf + xA0 * W;
-    constexpr int RAU = 4;  // A-rows whose table entries are fetched together
-    for (int r0 = rA0; r0 < RA; r0 += RAU * rAstep) {
-      int2 t[RAU];
-      bool rok[RAU];
-#pragma unroll
-      for (int u = 0; u < RAU; u++) {
-        const int r = r0 + u * rAstep;
-        const bool rin = r < RA;
-        t[u] = rin ? lds_int2(s_tabA + 8 * r) : make_int2(0, 0);
-        rok[u] = rin && (full || lds_int(s_digB + 4 * r) < c.limB);
-      }
-#pragma unroll
-      for (int u = 0; u < RAU; u++) {
-        const T *src = Ab + t[u].x;
-        const uint32_t dst = sb + t[u].y * W;
-        for (int k = 0; k < kA; k++)
-          cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok[u] && xA0 + (k << lgA) < lim);
-      }
+    for (int r = rA0; r < RA; r += rAstep) {
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
+      const T *src = Ab + t.x;
+      const uint32_t dst = sb + t.y * W;
+      for (int k = 0; k < kA; k++)
+        cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
     }
   };
   // store phase of one tile: B-row r <- smem through the column offsets
   auto drain = [&](const TileCtx &c, uint32_t sbuf) {
     const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
     const int lim = full ? LB : P.LBunit * c.limB;
-    store_rows<W, NJ>(B + c.bB + xB0, sbuf, s_tabB, s_digA, s_jcol, jc, rB0, rBstep, RB, kB, lgB,
-                      xB0, lim, LB, full, c.limA);
+    T *Bb = B + c.bB + xB0;
+    for (int r = rB0; r < RB; r += rBstep) {
+      const int2 t = lds_int2(s_tabB + 8 * r);
+      const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
+      T *dst = Bb + t.x;
+      const uint32_t src = sbuf + t.y * W;
+      if constexpr (NJ > 0) {
+#pragma unroll
+        for (int i = 0; i < NJ; i++) {
+          if (i < kB)
+            stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+        }
+      } else {
+#pragma unroll 4
+        for (int i = 0; i < kB; i++) {
+          const int j = xB0 + (i << lgB);
+          const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+          stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+        }
+      }
+    }
   };
 
   uint32_t tile = blockIdx.x;
@@ -520,8 +476,30 @@ __global__ void __launch_bounds__(512) k_tile(const __grid_constant__ TileParams
     }
     __syncthreads();
     // ---- store phase: shared -> coalesced B-row writes
-    store_rows<W, NJ>(B + c.bB + xB0, s_buf, s_tabB, s_digA, s_jcol, jc, rB0, rBstep, RB, kB, lgB,
-                      xB0, full ? LB : P.LBunit * c.limB, LB, full, c.limA);
+    {
+      const int lim = full ? LB : P.LBunit * c.limB;
+      T *Bb = B + c.bB + xB0;
+      for (int r = rB0; r < RB; r += rBstep) {
+        const int2 t = lds_int2(s_tabB + 8 * r);
+        const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
+        T *dst = Bb + t.x;
+        const uint32_t src = s_buf + t.y * W;
+        if constexpr (NJ > 0) {
+#pragma unroll
+          for (int i = 0; i < NJ; i++) {
+            if (i < kB)
+              stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+          }
+        } else {
+#pragma unroll 4
+          for (int i = 0; i < kB; i++) {
+            const int j = xB0 + (i << lgB);
+            const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
+            stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+          }
+        }
+      }
+    }
   }
 }
 
