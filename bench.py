@@ -213,8 +213,7 @@ def main():
     step_bytes = sum(c.alg_bytes for c in cases)
 
     def kname(info):
-        return f"{'k_direct' if info['schema'] in ('FML', 'COPY') else 'k_staged'}" \
-               f"<W={info['access_bytes']}>[{info['schema']}]"
+        return f"k_{info['kernel']}"
 
     def one_step(evs=None):
         with torch.cuda.stream(stream):

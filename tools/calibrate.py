@@ -47,16 +47,24 @@ def main():
     ap.add_argument("files", nargs="+")
     ap.add_argument("--write", action="store_true")
     ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--rel-max", type=float, default=1.5,
+                    help="fit only candidates within this factor of their case's best "
+                         "(the model's job is ranking the good region)")
     args = ap.parse_args()
     rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
+    best = collections.defaultdict(lambda: float("inf"))
+    for r in rows:
+        best[r["case"]] = min(best[r["case"]], r["meas"])
+    for r in rows:
+        r["rel"] = r["meas"] / best[r["case"]]
     cases = sorted({r["case"] for r in rows})
     rng = random.Random(args.seed)
     test_cases = set(rng.sample(cases, max(1, len(cases) // 5)))
     coefs, report = {}, {}
     for k in KINDS:
         rk = [r for r in rows if r["kernel"] == k]
-        tr = [r for r in rk if r["case"] not in test_cases]
-        te = [r for r in rk if r["case"] in test_cases]
+        tr = [r for r in rk if r["case"] not in test_cases and r["rel"] <= args.rel_max]
+        te = [r for r in rk if r["case"] in test_cases and r["rel"] <= args.rel_max]
         if not tr:
             continue
         c = fit(tr)
@@ -102,7 +110,8 @@ def main():
                 tag = "; ".join(f"{k}: train {v['err_train']:.1f}% test {v['err_test']:.1f}% "
                                 f"(n={v['n_train']}+{v['n_test']})" for k, v in report.items())
                 out.append(f'constexpr const char *kModelSource = "B200 fit ({len(cases)} cases, '
-                           f'{len(rows)} points): {tag}";')
+                           f'{len(rows)} points, rel<={args.rel_max}): {tag}; '
+                           f'regret {100 * np.mean(reg):.1f}%";')
             else:
                 out.append(line)
         with open(COEFF_H, "w") as f:
