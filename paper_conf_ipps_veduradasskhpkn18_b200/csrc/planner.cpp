@@ -309,7 +309,11 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.off_digB = take((int64_t)K.RA * 4);
     K.off_digA = take((int64_t)K.RB * 4);
     K.off_data = take(smem_elems * P.W);
-    K.off_data2 = (nbuf == 2) ? take(smem_elems * P.W) : K.off_data;
+    K.off_data2 = K.off_data;
+    for (int s = 1; s < nbuf; s++) {
+      const int32_t o = take(smem_elems * P.W);
+      if (s == 1) K.off_data2 = o;
+    }
   } else {
     K.off_tabB = take((int64_t)K.RB * 8);
     K.off_jcol = 0;
@@ -501,7 +505,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
 
   auto consider1 = [&](int kind, int threads, int a, int64_t ta, int b, int64_t tb) {
-    const int nbuf = (kind == KK_PIPE) ? 2 : 1;
+    const int nbuf = (kind == KK_PIPE) ? 2 : (kind == KK_PIPE3) ? 3 : 1;
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -518,6 +522,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int64_t V = 1;
     for (int k = 0; k < P.d; k++) V *= T.t[k];
     if (kind != KK_DIRECT && V * P.W > max_tile_bytes) return;
+    if (kind != KK_DIRECT) {
+      // output runs longer than 16 x 32 access elements gain nothing and would
+      // need per-element column-table reads (register column offsets, NJ <= 16)
+      int64_t LBc = 1;
+      for (int i = 0; i <= b; i++) LBc *= T.t[P.p[i]];
+      if (LBc > 512) return;
+    }
     if (kind == KK_DIRECT && V * P.W > 256 * 1024) return;
     TileParams K;
     if (!build_params(P, T, kind, threads, nbuf, K)) return;
@@ -538,7 +549,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
     if (mi.occ < 1) return;
     const int64_t slots = (int64_t)dev.sms * mi.occ;
-    if (kind == KK_PIPE) {
+    if (kind == KK_PIPE || kind == KK_PIPE3) {
       // persistent: one CTA per resident slot, striding over the tiles
       K.tpc = 1;
       mi.grid = (int)std::min<int64_t>(K.num_tiles, slots);
@@ -583,8 +594,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (group == KK_DIRECT) {
         consider1(KK_DIRECT, thr_list[ti], a, ta, b, tb);
       } else {
-        if (hv != 2) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
-        if (hv != 1) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
+        if (hv == 0 || hv == 1) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
+        if (hv == 0 || hv == 2 || hv == 3) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
+        if (hv == 0 || hv == 2 || hv == 4) consider1(KK_PIPE3, thr_list[ti], a, ta, b, tb);
       }
     }
   };
