@@ -88,8 +88,7 @@ typedef struct {
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
   int32_t variant;                       /* staged kernel: 0 = model choice, 1 = k_tile
-                                            (register-staged), 2 = k_pipe (either ring),
-                                            3 = k_pipe 2 buffers, 4 = k_pipe 3 buffers    */
+                                            (register-staged), 2 = k_pipe (cp.async)      */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -111,7 +110,7 @@ typedef struct {
   double predicted_seconds;               /* performance-model prediction                */
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
-  int32_t kernel;                         /* 0 k_direct, 1 k_tile, 2 k_pipe, 3 k_pipe(S=3) */
+  int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe    */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[12];

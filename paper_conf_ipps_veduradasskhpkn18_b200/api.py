@@ -152,7 +152,7 @@ def candidate_hints(d: dict) -> dict:
          "in_block": d["tile_extents"][a], "out_dim": b,
          "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
     if d["kernel"] != "direct":
-        h["variant"] = {"tile": 1, "pipe": 3, "pipe3": 4}[d["kernel"]]
+        h["variant"] = 1 if d["kernel"] == "tile" else 2
     return h
 
 

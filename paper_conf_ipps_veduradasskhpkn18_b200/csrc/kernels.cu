@@ -258,7 +258,7 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
 //                in registers; NJ = 0: column offsets read from the table.
 // Loop trip counts are warp-uniform and the bodies predicated, so no
 // divergence/reconvergence bookkeeping is generated in the hot loops.
-template <int W, int NJ, bool GA32, bool GB32, int S>
+template <int W, int NJ, bool GA32, bool GB32>
 __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
@@ -267,7 +267,7 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
   const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
   const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
   const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
-  const uint32_t s_buf0 = s0 + P.off_data, s_bstride = P.off_data2 - P.off_data;
+  const uint32_t s_buf0 = s0 + P.off_data, s_buf1 = s0 + P.off_data2;
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
@@ -349,26 +349,24 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
     }
   };
 
-  // S-stage ring of shared-memory buffers: tiles k+1 .. k+S-1 stream in while
-  // tile k is written out (S - 1 tiles of loads in flight per CTA)
-  const uint32_t G = gridDim.x;
-#pragma unroll
-  for (int s = 0; s < S - 1; s++) {
-    const uint32_t t = blockIdx.x + s * G;
-    if (t < P.num_tiles) issue(decode_tile(P, t), s_buf0 + s * s_bstride);
+  uint32_t tile = blockIdx.x;
+  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
+  if (tile < P.num_tiles) issue(cur, s_buf0);
+  cp_async_commit();
+  for (int k = 0; tile < P.num_tiles; k++) {
+    const uint32_t next = tile + gridDim.x;
+    TileCtx nx = cur;
+    if (next < P.num_tiles) {
+      nx = decode_tile(P, next);
+      issue(nx, (k & 1) ? s_buf0 : s_buf1);
+    }
     cp_async_commit();
-  }
-  int slot = 0;  // buffer of tile k
-  for (uint32_t tile = blockIdx.x; tile < P.num_tiles; tile += G) {
-    const uint32_t ahead = tile + (S - 1) * G;
-    const int aslot = (slot + S - 1) % S;
-    if (ahead < P.num_tiles) issue(decode_tile(P, ahead), s_buf0 + aslot * s_bstride);
-    cp_async_commit();
-    cp_async_wait<S - 1>();
+    cp_async_wait<1>();
     __syncthreads();
-    drain(decode_tile(P, tile), s_buf0 + slot * s_bstride);
+    drain(cur, (k & 1) ? s_buf1 : s_buf0);
     __syncthreads();
-    slot = (slot + 1) % S;
+    cur = nx;
+    tile = next;
   }
   cp_async_wait<0>();
 }
@@ -515,28 +513,26 @@ static const void *kernel_ptr_ka(int nj) {
     case 4: return (const void *)k_tile<W, KA, 4>;
     case 8: return (const void *)k_tile<W, KA, 8>;
   }
-  return (const void *)k_tile<W, KA, 16>;
+  return (const void *)k_tile<W, KA, 16>;  // LB <= 512 (planner cap)
 }
 
-template <int W, bool GA32, int S>
+template <int W, bool GA32>
 static const void *kernel_ptr_pipe(int nj, bool gb32) {
-  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false, S>;  // LB < 32: one slot
+  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false>;  // LB < 32: one slot
   switch (nj) {
-    case 1: return (const void *)k_pipe<W, 1, GA32, true, S>;
-    case 2: return (const void *)k_pipe<W, 2, GA32, true, S>;
-    case 4: return (const void *)k_pipe<W, 4, GA32, true, S>;
-    case 8: return (const void *)k_pipe<W, 8, GA32, true, S>;
+    case 1: return (const void *)k_pipe<W, 1, GA32, true>;
+    case 2: return (const void *)k_pipe<W, 2, GA32, true>;
+    case 4: return (const void *)k_pipe<W, 4, GA32, true>;
+    case 8: return (const void *)k_pipe<W, 8, GA32, true>;
   }
-  return (const void *)k_pipe<W, 16, GA32, true, S>;
+  return (const void *)k_pipe<W, 16, GA32, true>;  // LB <= 512 (planner cap)
 }
 
 template <int W>
 static const void *kernel_ptr_w(int kind, int ka, int nj, bool ga32, bool gb32) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
   if (kind == KK_PIPE)
-    return ga32 ? kernel_ptr_pipe<W, true, 2>(nj, gb32) : kernel_ptr_pipe<W, false, 2>(nj, gb32);
-  if (kind == KK_PIPE3)
-    return ga32 ? kernel_ptr_pipe<W, true, 3>(nj, gb32) : kernel_ptr_pipe<W, false, 3>(nj, gb32);
+    return ga32 ? kernel_ptr_pipe<W, true>(nj, gb32) : kernel_ptr_pipe<W, false>(nj, gb32);
   switch (ka) {
     case 1: return kernel_ptr_ka<W, 1>(nj);
     case 2: return kernel_ptr_ka<W, 2>(nj);
@@ -573,7 +569,7 @@ static const void *kernel_ptr(int kind, int W, int ka, int nj, bool ga32, bool g
 static int widx(int W) { return W == 4 ? 0 : (W == 8 ? 1 : 2); }
 
 int kernel_regs(int kind, int W) {
-  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
+  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
   static std::mutex mu;
   std::lock_guard<std::mutex> g(mu);
   int &r = regs[kind][widx(W)];

@@ -47,9 +47,8 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   // bytes in flight (Little's law with the loaded-DRAM latency): k_direct and
   // k_tile keep up to 8 access elements per thread of loads outstanding, the
   // cp.async pipeline of k_pipe a whole tile per CTA
-  const double per_cta = (mi.kind == KK_PIPE)    ? (double)mi.V
-                         : (mi.kind == KK_PIPE3) ? 2.0 * mi.V
-                                                 : std::min<double>(mi.V, kModelUnroll * mi.threads);
+  const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
+                                              : std::min<double>(mi.V, kModelUnroll * mi.threads);
   const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = sms * inflight / kModelLatency;
   // wave quantisation: tiles handed out over the resident CTA slots
@@ -78,8 +77,7 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
   const ModelFeatures F = model_features(mi, dev);
   const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect
                     : (mi.kind == KK_TILE) ? kCoefTile
-                    : (mi.kind == KK_PIPE) ? kCoefPipe
-                                           : kCoefPipe3;
+                                           : kCoefPipe;
   double t = 0.0;
   for (int i = 0; i < kModelNumFeatures; i++) t += c[i] * F.f[i];
   // the model can never beat one pass of the algorithmic bytes at copy speed

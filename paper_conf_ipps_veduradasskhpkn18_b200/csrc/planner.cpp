@@ -505,7 +505,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
 
   auto consider1 = [&](int kind, int threads, int a, int64_t ta, int b, int64_t tb) {
-    const int nbuf = (kind == KK_PIPE) ? 2 : (kind == KK_PIPE3) ? 3 : 1;
+    const int nbuf = (kind == KK_PIPE) ? 2 : 1;
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -549,7 +549,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
     if (mi.occ < 1) return;
     const int64_t slots = (int64_t)dev.sms * mi.occ;
-    if (kind == KK_PIPE || kind == KK_PIPE3) {
+    if (kind == KK_PIPE) {
       // persistent: one CTA per resident slot, striding over the tiles
       K.tpc = 1;
       mi.grid = (int)std::min<int64_t>(K.num_tiles, slots);
@@ -594,9 +594,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (group == KK_DIRECT) {
         consider1(KK_DIRECT, thr_list[ti], a, ta, b, tb);
       } else {
-        if (hv == 0 || hv == 1) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
-        if (hv == 0 || hv == 2 || hv == 3) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
-        if (hv == 0 || hv == 2 || hv == 4) consider1(KK_PIPE3, thr_list[ti], a, ta, b, tb);
+        if (hv != 2) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
+        if (hv != 1) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
       }
     }
   };

@@ -46,9 +46,8 @@ inline uint32_t fastdiv_host(uint32_t n, const FastDiv &f) {
 enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
   KK_TILE = 1,    // OD / OA / FMS: register-staged, one tile per CTA (k_tile)
-  KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered, persistent (k_pipe, S = 2)
-  KK_PIPE3 = 3,   // as KK_PIPE with a 3-buffer ring (two tiles of loads in flight)
-  KK_NUM = 4,
+  KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered, persistent (k_pipe)
+  KK_NUM = 3,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -95,7 +94,7 @@ struct TileParams {
   int32_t j_sS[TTLG_MAXD];
   // ---- shared-memory layout (bytes) and per-thread stepping
   int32_t smem_elems;      // data tile elements incl. padding
-  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;  // data buffers at off_data + s*(off_data2-off_data)
+  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
   int32_t lgA, lgB;            // log2 of the lane-group size owning one A-row / B-row
   int32_t tpc;                 // tiles per CTA (consecutive tile indices)
