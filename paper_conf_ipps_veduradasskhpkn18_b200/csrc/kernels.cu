@@ -8,11 +8,11 @@
 //            written straight to their output row (output run = the matching
 //            FVI, dim 0).  No shared memory for data, only the row table.
 //
-//  k_tile    (OD / OA / FMS; Alg. 2, Alg. 4/5 L868-1020, Alg. 6
+//  k_pipe    (OD / OA / FMS; Alg. 2, Alg. 4/5 L868-1020, Alg. 6
 //            L1022-1107): the tile (the paper's "slice") is the union of an
 //            input-prefix group and an output-prefix group.  Load phase: A-rows
-//            of LA contiguous elements are read coalesced (8 loads in flight per
-//            thread) and stored to shared memory; store phase: B-rows of LB
+//            of LA contiguous elements are copied global -> shared with cp.async
+//            (LDGSTS, predicated PTX); store phase: B-rows of LB
 //            contiguous elements are read from shared memory through the column
 //            offsets and written coalesced.  Rows are processed warp-wise: a
 //            warp (or a power-of-two lane group of G <= 32 lanes when the run is
@@ -23,9 +23,10 @@
 //            position j lands in bank j mod (128/W): conflict-free column reads
 //            (generalising the 32x33 pad, L747-749, and FMS's pad, L1104-1107).
 //
-// Grids: one CTA per tile (or a few consecutive tiles, `tpc`), many CTAs per
-// SM -- the skeleton that reaches the D2D copy rate on B200
-// (tools/copybench.cu).  Every CTA builds its row tables in shared memory
+// Two grid strategies compete per candidate: PERSIST = false ("k_tile"): one
+// CTA per tile (or a few consecutive tiles, `tpc`), single buffer, many CTAs
+// per SM; PERSIST = true ("k_pipe"): persistent CTAs with a double-buffered
+// cp.async ring.  k_direct uses one CTA per tile.  Every CTA builds its row tables in shared memory
 // (the paper's texture-mapped offset arrays, L737-745) and decodes its tile
 // index with fast-divmod (the paper's decode/compute_base, L725-737).
 #include <cuda_runtime.h>
@@ -258,7 +259,7 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
 //                in registers; NJ = 0: column offsets read from the table.
 // Loop trip counts are warp-uniform and the bodies predicated, so no
 // divergence/reconvergence bookkeeping is generated in the hot loops.
-template <int W, int NJ, bool GA32, bool GB32>
+template <int W, int NJ, bool GA32, bool GB32, bool PERSIST>
 __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
@@ -349,196 +350,67 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
     }
   };
 
-  uint32_t tile = blockIdx.x;
-  TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
-  if (tile < P.num_tiles) issue(cur, s_buf0);
-  cp_async_commit();
-  for (int k = 0; tile < P.num_tiles; k++) {
-    const uint32_t next = tile + gridDim.x;
-    TileCtx nx = cur;
-    if (next < P.num_tiles) {
-      nx = decode_tile(P, next);
-      issue(nx, (k & 1) ? s_buf0 : s_buf1);
+  if constexpr (!PERSIST) {
+    // k_tile: one tile (or tpc consecutive tiles) per CTA, single buffer, many
+    // CTAs per SM -- the cp.async skeleton that reaches the D2D copy rate
+    // (tools/copybench.cu: 6.4-6.6 TB/s vs 5.4-5.8 TB/s persistent)
+    for (int it = 0; it < P.tpc; it++) {
+      const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
+      if (tile >= P.num_tiles) break;
+      const TileCtx c = decode_tile(P, tile);
+      if (it > 0) __syncthreads();
+      issue(c, s_buf0);
+      cp_async_commit();
+      cp_async_wait<0>();
+      __syncthreads();
+      drain(c, s_buf0);
     }
+  } else {
+    uint32_t tile = blockIdx.x;
+    TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
+    if (tile < P.num_tiles) issue(cur, s_buf0);
     cp_async_commit();
-    cp_async_wait<1>();
-    __syncthreads();
-    drain(cur, (k & 1) ? s_buf1 : s_buf0);
-    __syncthreads();
-    cur = nx;
-    tile = next;
-  }
-  cp_async_wait<0>();
-}
-
-
-// k_tile template parameters (all warp-uniform, chosen at launch from the plan):
-//   KA: A-row elements per lane (ceil(LA / G_A), rounded up to a power of two);
-//       KA > 1 implies the lane group is the whole warp (G_A = 32).
-//   NJ: B-row elements per lane (ceil(LB / G_B) rounded up); NJ > 1 implies
-//       G_B = 32; NJ = 0: long output runs, column offsets read from the table.
-// Load phase: each thread loads up to 8 elements (RU = 8/KA rows x KA) into
-// registers before storing them to shared memory -- 8 independent loads in
-// flight per thread (the unrolled-copy skeleton that reaches the D2D rate on
-// B200; cp.async staging measured ~10% slower, tools/copybench.cu).
-template <int W, int KA, int NJ>
-__global__ void __launch_bounds__(512) k_tile(const __grid_constant__ TileParams P,
-                                              const void *__restrict__ Av,
-                                              void *__restrict__ Bv) {
-  using T = typename Vec<W>::T;
-  constexpr int RU = 8 / KA;  // A-rows per load batch
-  extern __shared__ __align__(16) unsigned char smem[];
-  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
-  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
-  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
-  const uint32_t s_buf = s0 + P.off_data;
-  T *sdata = reinterpret_cast<T *>(smem + P.off_data);
-  const T *A = reinterpret_cast<const T *>(Av);
-  T *B = reinterpret_cast<T *>(Bv);
-
-  build_rows(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk,
-             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB));
-  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk,
-             reinterpret_cast<int2 *>(smem + P.off_tabB),
-             reinterpret_cast<int *>(smem + P.off_digA));
-  for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
-    int rem = j, s = 0;
-    for (int k = 0; k < P.nj; k++) {
-      const int e = P.j_ext[k];
-      const int cq = rem / e;
-      s += (rem - cq * e) * P.j_sS[k];
-      rem = cq;
-    }
-    reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
-  }
-  __syncthreads();
-
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int lgA = KA > 1 ? 5 : P.lgA, lgB = NJ != 1 ? 5 : P.lgB;
-  const int gA = 1 << lgA, gB = 1 << lgB;
-  const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> lgA) + (lane >> lgA);
-  const int rAstep = nw * (32 >> lgA);
-  const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
-  const int rBstep = nw * (32 >> lgB);
-  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
-  const int kB = (LB + gB - 1) >> lgB;
-  int jc[NJ > 0 ? NJ : 1];
-  if constexpr (NJ > 0) {
-#pragma unroll
-    for (int i = 0; i < NJ; i++) {
-      const int j = xB0 + i * gB;
-      jc[i] = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-    }
-  }
-
-  for (int it = 0; it < P.tpc; it++) {
-    const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
-    if (tile >= P.num_tiles) break;
-    const TileCtx c = decode_tile(P, tile);
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    if (it > 0) __syncthreads();  // previous tile's reads of smem are done
-    // ---- load phase: global -> registers -> shared (8 loads in flight per thread)
-    {
-      const int lim = full ? LA : P.LAunit * c.limA;
-      const T *Ab = A + c.bA + xA0;
-      for (int r0 = rA0; r0 < RA; r0 += RU * rAstep) {
-        const T *src[RU];
-        uint32_t so[RU];
-        bool rok[RU];
-#pragma unroll
-        for (int u = 0; u < RU; u++) {
-          const int r = r0 + u * rAstep;
-          const bool rin = r < RA;
-          const int2 t = rin ? lds_int2(s_tabA + 8 * r) : make_int2(0, 0);
-          rok[u] = rin && (full || lds_int(s_digB + 4 * r) < c.limB);
-          so[u] = (uint32_t)(t.y + xA0);
-          src[u] = Ab + t.x;
-        }
-        // runs longer than KA * 32 elements take several uniform passes
-        for (int xb = 0; xb < lim; xb += KA << lgA) {
-          T v[RU][KA];
-          bool ok[RU][KA];
-#pragma unroll
-          for (int u = 0; u < RU; u++) {
-#pragma unroll
-            for (int k = 0; k < KA; k++) {
-              ok[u][k] = rok[u] && xA0 + xb + (k << lgA) < lim;
-              if (ok[u][k]) v[u][k] = ld_stream<true>(src[u] + xb + (k << lgA));
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < RU; u++)
-#pragma unroll
-            for (int k = 0; k < KA; k++)
-              if (ok[u][k]) sdata[so[u] + xb + (k << lgA)] = v[u][k];
-        }
+    for (int k = 0; tile < P.num_tiles; k++) {
+      const uint32_t next = tile + gridDim.x;
+      TileCtx nx = cur;
+      if (next < P.num_tiles) {
+        nx = decode_tile(P, next);
+        issue(nx, (k & 1) ? s_buf0 : s_buf1);
       }
+      cp_async_commit();
+      cp_async_wait<1>();
+      __syncthreads();
+      drain(cur, (k & 1) ? s_buf1 : s_buf0);
+      __syncthreads();
+      cur = nx;
+      tile = next;
     }
-    __syncthreads();
-    // ---- store phase: shared -> coalesced B-row writes
-    {
-      const int lim = full ? LB : P.LBunit * c.limB;
-      T *Bb = B + c.bB + xB0;
-      for (int r = rB0; r < RB; r += rBstep) {
-        const int2 t = lds_int2(s_tabB + 8 * r);
-        const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
-        T *dst = Bb + t.x;
-        const uint32_t src = s_buf + t.y * W;
-        if constexpr (NJ > 0) {
-#pragma unroll
-          for (int i = 0; i < NJ; i++) {
-            if (i < kB)
-              stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
-          }
-        } else {
-#pragma unroll 4
-          for (int i = 0; i < kB; i++) {
-            const int j = xB0 + (i << lgB);
-            const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-            stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
-          }
-        }
-      }
-    }
+    cp_async_wait<0>();
   }
 }
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W, int KA>
-static const void *kernel_ptr_ka(int nj) {
-  switch (nj) {
-    case 1: return (const void *)k_tile<W, KA, 1>;
-    case 2: return (const void *)k_tile<W, KA, 2>;
-    case 4: return (const void *)k_tile<W, KA, 4>;
-    case 8: return (const void *)k_tile<W, KA, 8>;
-  }
-  return (const void *)k_tile<W, KA, 16>;  // LB <= 512 (planner cap)
-}
-
-template <int W, bool GA32>
+template <int W, bool GA32, bool PERSIST>
 static const void *kernel_ptr_pipe(int nj, bool gb32) {
-  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false>;  // LB < 32: one slot
+  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false, PERSIST>;  // LB < 32: one slot
   switch (nj) {
-    case 1: return (const void *)k_pipe<W, 1, GA32, true>;
-    case 2: return (const void *)k_pipe<W, 2, GA32, true>;
-    case 4: return (const void *)k_pipe<W, 4, GA32, true>;
-    case 8: return (const void *)k_pipe<W, 8, GA32, true>;
+    case 1: return (const void *)k_pipe<W, 1, GA32, true, PERSIST>;
+    case 2: return (const void *)k_pipe<W, 2, GA32, true, PERSIST>;
+    case 4: return (const void *)k_pipe<W, 4, GA32, true, PERSIST>;
+    case 8: return (const void *)k_pipe<W, 8, GA32, true, PERSIST>;
   }
-  return (const void *)k_pipe<W, 16, GA32, true>;  // LB <= 512 (planner cap)
+  return (const void *)k_pipe<W, 16, GA32, true, PERSIST>;  // LB <= 512 (planner cap)
 }
 
 template <int W>
-static const void *kernel_ptr_w(int kind, int ka, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
   if (kind == KK_PIPE)
-    return ga32 ? kernel_ptr_pipe<W, true>(nj, gb32) : kernel_ptr_pipe<W, false>(nj, gb32);
-  switch (ka) {
-    case 1: return kernel_ptr_ka<W, 1>(nj);
-    case 2: return kernel_ptr_ka<W, 2>(nj);
-    case 4: return kernel_ptr_ka<W, 4>(nj);
-  }
-  return kernel_ptr_ka<W, 8>(nj);
+    return ga32 ? kernel_ptr_pipe<W, true, true>(nj, gb32)
+                : kernel_ptr_pipe<W, false, true>(nj, gb32);
+  return ga32 ? kernel_ptr_pipe<W, true, false>(nj, gb32)
+              : kernel_ptr_pipe<W, false, false>(nj, gb32);
 }
 
 static int pow2_at_least(int k) {
@@ -547,21 +419,17 @@ static int pow2_at_least(int k) {
   return p;
 }
 
-// per-lane elements of an A-row (KA, <= 8) and of a B-row (NJ, 0 = table path)
-static int ka_of(const TileParams &K) {
-  const int k = pow2_at_least((K.LA + (1 << K.lgA) - 1) >> K.lgA);
-  return k <= 8 ? k : 8;
-}
+// per-lane elements of a B-row (NJ <= 16)
 static int nj_of(const TileParams &K) {
   const int k = pow2_at_least((K.LB + (1 << K.lgB) - 1) >> K.lgB);
   return k <= 16 ? k : 0;
 }
 
-static const void *kernel_ptr(int kind, int W, int ka, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, ka, nj, ga32, gb32);
-    case 8: return kernel_ptr_w<8>(kind, ka, nj, ga32, gb32);
-    case 16: return kernel_ptr_w<16>(kind, ka, nj, ga32, gb32);
+    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32);
+    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32);
+    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32);
   }
   return nullptr;
 }
@@ -575,7 +443,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 8, 4, true, true)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 4, true, true)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -586,8 +454,8 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W, ka_of(plan->kp), nj_of(plan->kp),
-                              plan->kp.lgA == 5, plan->kp.lgB == 5);
+  const void *fn = kernel_ptr(plan->kind, plan->W, nj_of(plan->kp), plan->kp.lgA == 5,
+                              plan->kp.lgB == 5);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

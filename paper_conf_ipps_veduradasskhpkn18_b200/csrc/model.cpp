@@ -44,11 +44,12 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   const double sector = read_bytes + write_bytes;
   const double alg = 2.0 * mi.N * W;
   const double bw = dev.hbm_gbs * 1e9;
-  // bytes in flight (Little's law with the loaded-DRAM latency): k_direct and
-  // k_tile keep up to 8 access elements per thread of loads outstanding, the
-  // cp.async pipeline of k_pipe a whole tile per CTA
-  const double per_cta = (mi.kind == KK_PIPE) ? (double)mi.V
-                                              : std::min<double>(mi.V, kModelUnroll * mi.threads);
+  // bytes in flight (Little's law with the loaded-DRAM latency): the staged
+  // kernels keep a whole tile of cp.async loads in flight per CTA, k_direct up
+  // to 8 access elements per thread
+  const double per_cta = (mi.kind == KK_DIRECT)
+                             ? std::min<double>(mi.V, kModelUnroll * mi.threads)
+                             : (double)mi.V;
   const double inflight = (double)mi.occ * per_cta * W;
   const double bw_lat = sms * inflight / kModelLatency;
   // wave quantisation: tiles handed out over the resident CTA slots

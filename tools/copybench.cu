@@ -77,6 +77,47 @@ __global__ void pipe_copy(const uint4 *__restrict__ a, uint4 *__restrict__ b, si
   asm volatile("cp.async.wait_group 0;\n" ::: "memory");
 }
 
+// k_tile skeleton for a plain copy: one tile per CTA, LDG -> regs -> STS,
+// sync, LDS -> STG (smem round trip), many CTAs (non-persistent)
+template <int U>
+__global__ void smem_copy(const uint4 *__restrict__ a, uint4 *__restrict__ b, size_t n) {
+  extern __shared__ uint4 sm[];
+  const int tile = blockDim.x * U;
+  size_t base = (size_t)blockIdx.x * tile;
+  uint4 v[U];
+#pragma unroll
+  for (int u = 0; u < U; u++) {
+    size_t i = base + u * blockDim.x + threadIdx.x;
+    if (i < n) v[u] = __ldcs(a + i);
+  }
+#pragma unroll
+  for (int u = 0; u < U; u++) sm[u * blockDim.x + threadIdx.x] = v[u];
+  __syncthreads();
+#pragma unroll
+  for (int u = 0; u < U; u++) {
+    int k = (u * blockDim.x + threadIdx.x + 17 * (threadIdx.x >> 5)) % tile;  // shuffled read
+    size_t i = base + k;
+    if (i < n) __stcs(b + i, sm[k]);
+  }
+}
+
+// cp.async single-tile-per-CTA copy (non-persistent)
+__global__ void cpasync_copy(const uint4 *__restrict__ a, uint4 *__restrict__ b, size_t n, int tile) {
+  extern __shared__ uint4 sm[];
+  size_t base = (size_t)blockIdx.x * tile;
+  for (int i = threadIdx.x; i < tile; i += blockDim.x) {
+    if (base + i < n) {
+      unsigned s = (unsigned)__cvta_generic_to_shared(sm + i);
+      asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(a + base + i));
+    }
+  }
+  asm volatile("cp.async.commit_group;\n" ::: "memory");
+  asm volatile("cp.async.wait_group 0;\n" ::: "memory");
+  __syncthreads();
+  for (int i = threadIdx.x; i < tile; i += blockDim.x)
+    if (base + i < n) __stcs(b + base + i, sm[i]);
+}
+
 template <typename F>
 float timeit(F f, int reps) {
   cudaEvent_t e0, e1;
@@ -123,6 +164,23 @@ int main(int argc, char **argv) {
       printf("chunked U%d nc   t%-4d g%-7d %.0f\n", U, threads, grid, gbs(ms));
       if (U == 4) printf("chunked U4 cs   t%-4d g%-7d %.0f\n", threads, grid, gbs(timeit([&] { chunked<4, true><<<grid, threads>>>(a, b, n); }, 20)));
     }
+  }
+  for (int threads : {256, 512}) {
+    for (int U : {4, 8}) {
+      size_t tile = (size_t)threads * U;
+      int grid = (int)((n + tile - 1) / tile);
+      float ms = U == 4 ? timeit([&] { smem_copy<4><<<grid, threads, tile * 16>>>(a, b, n); }, 20)
+                        : timeit([&] { smem_copy<8><<<grid, threads, tile * 16>>>(a, b, n); }, 20);
+      printf("smem_copy U%d t%-4d tile %zuKB g%-6d %.0f\n", U, threads, tile * 16 / 1024, grid, gbs(ms));
+    }
+  }
+  cudaFuncSetAttribute(cpasync_copy, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+  for (int tileKB : {4, 8, 16, 32}) {
+    int tile = tileKB * 1024 / 16;
+    int grid = (int)((n + tile - 1) / tile);
+    for (int threads : {128, 256, 512})
+      printf("cpasync_copy tile %2dKB t%-4d g%-6d %.0f\n", tileKB, threads, grid,
+             gbs(timeit([&] { cpasync_copy<<<grid, threads, tile * 16>>>(a, b, n, tile); }, 20)));
   }
   cudaFuncSetAttribute(pipe_copy, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
   for (int tileKB : {8, 16, 32, 48}) {
