@@ -149,14 +149,14 @@ __device__ __forceinline__ TileCtx decode_tile(const TileParams &P, uint32_t til
 
 // Row tables (Alg. 4's input_offset / output_offset, separated into a per-row
 // part and a per-column part): decode row index i over the row digits.
-__device__ __forceinline__ void build_rows(int R, int nr, const int32_t *ext, const int32_t *sG,
+// Digit extents are >= 2, so the multiply-shift division applies.
+__device__ __forceinline__ void build_rows(int R, int nr, const FastDiv *ext, const int32_t *sG,
                                            const int32_t *sS, int blk, int2 *tab, int *dig) {
   for (int i = threadIdx.x; i < R; i += blockDim.x) {
     int rem = i, g = 0, s = 0, dg = 0;
     for (int k = 0; k < nr; k++) {
-      const int e = ext[k];
-      const int cq = rem / e;
-      const int c = rem - cq * e;
+      const int cq = (int)fdiv((uint32_t)rem, ext[k]);
+      const int c = rem - cq * (int)ext[k].div;
       rem = cq;
       g += c * sG[k];
       s += c * sS[k];
@@ -178,7 +178,7 @@ __global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TilePara
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
-  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
   __syncthreads();
 
   const int NT = blockDim.x, tid = threadIdx.x;
@@ -272,17 +272,16 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
-  build_rows(P.RA, P.nra, P.ra_ext, P.ra_sG, P.ra_sS, P.ra_blk,
+  build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
              reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB));
-  build_rows(P.RB, P.nrb, P.rb_ext, P.rb_sG, P.rb_sS, P.rb_blk,
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
              reinterpret_cast<int2 *>(smem + P.off_tabB),
              reinterpret_cast<int *>(smem + P.off_digA));
   for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
     int rem = j, s = 0;
     for (int k = 0; k < P.nj; k++) {
-      const int e = P.j_ext[k];
-      const int cq = rem / e;
-      s += (rem - cq * e) * P.j_sS[k];
+      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+      s += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
       rem = cq;
     }
     reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset

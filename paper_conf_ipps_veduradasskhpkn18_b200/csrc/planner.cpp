@@ -265,6 +265,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     if (inIS[k] || T.t[k] <= 1) continue;
     if (k == pb && K.blkB_g >= 0) K.ra_blk = K.nra;
     K.ra_ext[K.nra] = (int32_t)T.t[k];
+    K.ra_div[K.nra] = make_fastdiv((uint32_t)T.t[k]);
     K.ra_sG[K.nra] = (int32_t)S.sA[k];
     K.ra_sS[K.nra] = (int32_t)sm[k];
     maxG += (T.t[k] - 1) * S.sA[k];
@@ -278,6 +279,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     if (inOS[k] || T.t[k] <= 1) continue;
     if (k == a && K.blkA_g >= 0) K.rb_blk = K.nrb;
     K.rb_ext[K.nrb] = (int32_t)T.t[k];
+    K.rb_div[K.nrb] = make_fastdiv((uint32_t)T.t[k]);
     K.rb_sG[K.nrb] = (int32_t)S.sB[k];
     K.rb_sS[K.nrb] = (int32_t)sm[k];
     maxG += (T.t[k] - 1) * S.sB[k];
@@ -289,6 +291,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     const int k = P.p[i];
     if (T.t[k] <= 1) continue;
     K.j_ext[K.nj] = (int32_t)T.t[k];
+    K.j_div[K.nj] = make_fastdiv((uint32_t)T.t[k]);
     K.j_sS[K.nj] = (int32_t)sm[k];
     K.nj++;
   }

@@ -83,15 +83,18 @@ struct TileParams {
   int32_t ra_ext[TTLG_MAXD];
   int32_t ra_sG[TTLG_MAXD];  // stride in A
   int32_t ra_sS[TTLG_MAXD];  // stride in the smem tile
+  FastDiv ra_div[TTLG_MAXD];  // fast division by ra_ext
   // ---- B-row digits (tile dims outside the output run), input order
   int32_t nrb, rb_blk;     // rb_blk: which B-row digit is dim a (-1: none)
   int32_t rb_ext[TTLG_MAXD];
   int32_t rb_sG[TTLG_MAXD];  // stride in B
   int32_t rb_sS[TTLG_MAXD];
+  FastDiv rb_div[TTLG_MAXD];
   // ---- output-run digits, output order (-> smem column offsets)
   int32_t nj;
   int32_t j_ext[TTLG_MAXD];
   int32_t j_sS[TTLG_MAXD];
+  FastDiv j_div[TTLG_MAXD];
   // ---- shared-memory layout (bytes) and per-thread stepping
   int32_t smem_elems;      // data tile elements incl. padding
   int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
