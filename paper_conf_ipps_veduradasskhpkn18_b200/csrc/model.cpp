@@ -12,10 +12,10 @@ namespace ttlg {
 // plus half a sector on average when the run is not sector-aligned, with a
 // 64-byte floor (HBM burst) -- the B200 restatement of Table I's transaction
 // counts, which count 128-byte K40 transactions.
-static double run_cost(double R) {
-  double c = 32.0 * std::ceil(R / 32.0);
-  if (std::fmod(R, 32.0) != 0.0) c += 16.0;
-  return std::max(c, 64.0);
+static double run_cost(int64_t R) {
+  int64_t c = (R + 31) / 32 * 32;
+  if (R & 31) c += 16;
+  return (double)(c < 64 ? 64 : c);
 }
 
 ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
@@ -25,19 +25,23 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   const double tiles = (double)mi.num_tiles;
   const double fill = mi.fillA;
   const double sms = dev.sms;
-  auto group = [](double L) { return L >= 32 ? 32.0 : std::pow(2.0, std::ceil(std::log2(L))); };
+  auto group = [](double L) {  // lanes per row: next power of two, at most 32
+    double g = 1.0;
+    while (g < L && g < 32.0) g *= 2.0;
+    return g;
+  };
   double read_bytes, runsA, opsA;
   if (mi.kind == KK_DIRECT) {
-    read_bytes = tiles * fill * run_cost(mi.V * W);
+    read_bytes = tiles * fill * run_cost((int64_t)mi.V * mi.W);
     runsA = tiles * fill;
     opsA = tiles * mi.V / 32.0;
   } else {
-    read_bytes = tiles * fill * mi.RA * run_cost(mi.LA * W);
+    read_bytes = tiles * fill * mi.RA * run_cost((int64_t)mi.LA * mi.W);
     runsA = tiles * fill * mi.RA;
     const double gA = group(mi.LA);
     opsA = tiles * mi.RA * std::ceil(mi.LA / gA) / (32.0 / gA);
   }
-  const double write_bytes = tiles * fill * mi.RB * run_cost(mi.LB * W);
+  const double write_bytes = tiles * fill * mi.RB * run_cost((int64_t)mi.LB * mi.W);
   const double runsB = tiles * fill * mi.RB;
   const double gB = group(mi.LB);
   const double opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);

@@ -11,6 +11,7 @@
 //
 // No CUDA calls here: the device profile is passed in, so plans can be built
 // (and unit-tested) on a host with no GPU.
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -179,6 +180,50 @@ int64_t ceil_div(int64_t x, int64_t y) { return (x + y - 1) / y; }
 
 }  // namespace
 
+// Cheap geometry summary of a tile (what the model needs), without building
+// the parameter block: used to screen candidates before the full build.
+struct TileSummary {
+  int64_t V, LA, LB, RA, RB, tiles;
+  int smem_base;  // shared memory with one data buffer
+  int buf_bytes;  // one data buffer
+};
+
+static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S) {
+  const int d = P.d, a = T.a, b = T.b;
+  bool inIS[TTLG_MAXD] = {false};
+  for (int k = 0; k <= a; k++) inIS[k] = true;
+  S.V = 1;
+  S.LA = 1;
+  S.LB = 1;
+  S.tiles = 1;
+  for (int k = 0; k < d; k++) {
+    S.V *= T.t[k];
+    S.tiles *= ceil_div(P.n[k], T.t[k]);
+  }
+  for (int k = 0; k <= a; k++) S.LA *= T.t[k];
+  for (int i = 0; i <= b; i++) S.LB *= T.t[P.p[i]];
+  if (S.V >= (1ll << 30) || S.tiles >= (1ll << 31)) return false;
+  S.RA = S.V / S.LA;
+  S.RB = S.V / S.LB;
+  auto r16 = [](int64_t x) { return (x + 15) / 16 * 16; };
+  if (kind == KK_DIRECT) {
+    S.smem_base = (int)(r16(S.RB * 8) + r16(S.RB * 4));
+    S.buf_bytes = 0;
+    return true;
+  }
+  int64_t cur = S.LA, Q = 1;
+  const int64_t Wb = 128 / P.W;
+  for (int i = 0; i <= b; i++) {
+    const int k = P.p[i];
+    if (!inIS[k] && T.t[k] > 1) cur = (cur + (((Q - cur) % Wb) + Wb) % Wb) * T.t[k];
+    Q *= T.t[k];
+  }
+  S.buf_bytes = (int)r16(cur * P.W);
+  S.smem_base = (int)(r16(S.RA * 8) + r16(S.RB * 8) + r16(S.LB * 4) + r16(S.RA * 4) +
+                      r16(S.RB * 4) + S.buf_bytes);
+  return true;
+}
+
 // Fill TileParams for a tile; returns false if it violates a kernel limit.
 static bool build_params(const Problem &P, const Tile &T, int kind, int threads, int nbuf,
                          TileParams &K) {
@@ -344,24 +389,24 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
 // number of distinct 4-byte words that fall into one bank.  `addr` holds the
 // 32 lanes' element offsets.
 static double wavefront_ratio(const int64_t *addr, int W) {
-  const int per_phase = 128 / W, phases = 32 / per_phase;
+  const int per_phase = 128 / W, phases = 32 / per_phase, wpl = W / 4;
   int total = 0;
   for (int ph = 0; ph < phases; ph++) {
-    int64_t words[32 * 4];
-    int nw = 0;
-    for (int l = ph * per_phase; l < (ph + 1) * per_phase; l++)
-      for (int w = 0; w < W / 4; w++) words[nw++] = addr[l] * (W / 4) + w;
+    // distinct words per bank (a repeated word is a broadcast); degree capped at 8
+    uint32_t bw[32][8];
+    uint8_t cnt[32] = {0};
     int worst = 1;
-    for (int bank = 0; bank < 32; bank++) {
-      int64_t seen[32 * 4];
-      int ns = 0;
-      for (int i = 0; i < nw; i++) {
-        if (((words[i] % 32) + 32) % 32 != bank) continue;
+    for (int l = ph * per_phase; l < (ph + 1) * per_phase; l++) {
+      for (int k = 0; k < wpl; k++) {
+        const uint32_t w = (uint32_t)(addr[l] * wpl + k);
+        const int b = (int)(w & 31);
         bool dup = false;
-        for (int s = 0; s < ns; s++) dup |= seen[s] == words[i];
-        if (!dup) seen[ns++] = words[i];
+        for (int s = 0; s < cnt[b]; s++) dup |= bw[b][s] == w;
+        if (!dup && cnt[b] < 8) {
+          bw[b][cnt[b]++] = w;
+          if (cnt[b] > worst) worst = cnt[b];
+        }
       }
-      if (ns > worst) worst = ns;
     }
     total += worst;
   }
@@ -370,28 +415,44 @@ static double wavefront_ratio(const int64_t *addr, int W) {
 
 // conflict ratios of the first warp of the load (A-row) and store (B-row) phases
 static void smem_conflicts(const TileParams &K, int W, double &load, double &store) {
-  auto row_off = [](int r, int n, const int32_t *ext, const int32_t *sS) {
+  // offsets of the first `cnt` rows (or columns) of a mixed-radix digit set,
+  // by odometer (no division)
+  auto offsets = [](int cnt, int n, const int32_t *ext, const int32_t *sS, int64_t *out) {
+    int dig[TTLG_MAXD] = {0};
     int64_t s = 0;
-    for (int k = 0; k < n; k++) {
-      s += (int64_t)(r % ext[k]) * sS[k];
-      r /= ext[k];
+    for (int i = 0; i < cnt; i++) {
+      out[i] = s;
+      for (int k = 0; k < n; k++) {
+        s += sS[k];
+        if (++dig[k] < ext[k]) break;
+        s -= (int64_t)dig[k] * sS[k];
+        dig[k] = 0;
+      }
     }
-    return s;
   };
-  int64_t addr[32];
-  {
-    const int g = 1 << K.lgA;
+  int64_t addr[32], rows[32], cols[32];
+  // closed-form fast paths: a whole warp on one A-row reads consecutive words;
+  // a whole warp on one B-row whose first output digit spans the warp with an
+  // odd shared-memory stride (the padding rule) hits distinct banks
+  const bool load_free = K.lgA == 5;
+  const bool store_free = K.lgB == 5 && K.nj > 0 && K.j_ext[0] >= 32 && (K.j_sS[0] & 1);
+  load = store = 1.0;
+  if (!load_free) {
+    const int g = 1 << K.lgA, nr = std::min(32 >> K.lgA, K.RA);
+    offsets(nr, K.nra, K.ra_ext, K.ra_sS, rows);
     for (int l = 0; l < 32; l++) {
-      const int r = std::min(l >> K.lgA, K.RA - 1), x = std::min(l & (g - 1), K.LA - 1);
-      addr[l] = row_off(r, K.nra, K.ra_ext, K.ra_sS) + x;
+      const int r = std::min(l >> K.lgA, nr - 1), x = std::min(l & (g - 1), K.LA - 1);
+      addr[l] = rows[r] + x;
     }
     load = wavefront_ratio(addr, W);
   }
-  {
-    const int g = 1 << K.lgB;
+  if (!store_free) {
+    const int g = 1 << K.lgB, nr = std::min(32 >> K.lgB, K.RB), nc = std::min(g, K.LB);
+    offsets(nr, K.nrb, K.rb_ext, K.rb_sS, rows);
+    offsets(nc, K.nj, K.j_ext, K.j_sS, cols);
     for (int l = 0; l < 32; l++) {
-      const int r = std::min(l >> K.lgB, K.RB - 1), j = std::min(l & (g - 1), K.LB - 1);
-      addr[l] = row_off(r, K.nrb, K.rb_ext, K.rb_sS) + row_off(j, K.nj, K.j_ext, K.j_sS);
+      const int r = std::min(l >> K.lgB, nr - 1), j = std::min(l & (g - 1), nc - 1);
+      addr[l] = rows[r] + cols[j];
     }
     store = wavefront_ratio(addr, W);
   }
@@ -507,8 +568,15 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
 
-  auto consider1 = [&](int kind, int threads, int a, int64_t ta, int b, int64_t tb) {
-    const int nbuf = (kind == KK_PIPE) ? 2 : 1;
+  // kernel variants and block sizes competing for each slice candidate
+  const int hv = hints ? hints->variant : 0;
+  const int nthr = (hints && hints->threads) ? 1 : 2;
+  const int thr_list[2] = {(hints && hints->threads) ? hints->threads : 256, 512};
+
+  // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB): the tile,
+  // its parameter block and shared-memory conflict ratios are computed once;
+  // then every kernel variant x block size is scored by the model.
+  auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -517,90 +585,126 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     Tile T = make_tile(P, a, ta, b, tb);
     if (!T.ok) return;
-    const int schema = schema_of(P, T, kind);
+    const int schema = schema_of(P, T, group);
     if (force_schema != TTLG_SCHEMA_AUTO && force_schema != schema) {
       // COPY and FML share the direct kernel; accept FML for a rank-1 problem
       if (!(force_schema == TTLG_SCHEMA_FML && schema == TTLG_SCHEMA_COPY)) return;
     }
     int64_t V = 1;
     for (int k = 0; k < P.d; k++) V *= T.t[k];
-    if (kind != KK_DIRECT && V * P.W > max_tile_bytes) return;
-    if (kind != KK_DIRECT) {
+    if (group != KK_DIRECT) {
+      if (V * P.W > max_tile_bytes) return;
       // output runs longer than 16 x 32 access elements gain nothing and would
       // need per-element column-table reads (register column offsets, NJ <= 16)
       int64_t LBc = 1;
       for (int i = 0; i <= b; i++) LBc *= T.t[P.p[i]];
       if (LBc > 512) return;
+    } else if (V * P.W > 256 * 1024) {
+      return;
     }
-    if (kind == KK_DIRECT && V * P.W > 256 * 1024) return;
-    TileParams K;
-    if (!build_params(P, T, kind, threads, nbuf, K)) return;
-    if (K.smem_bytes > dev.smem_per_block_optin) return;
-    ModelInput mi;
-    mi.kind = kind;
-    mi.schema = schema;
-    mi.W = P.W;
-    mi.N = N;
-    mi.V = K.V;
-    mi.LA = K.LA;
-    mi.LB = K.LB;
-    mi.RA = K.RA;
-    mi.RB = K.RB;
-    mi.num_tiles = K.num_tiles;
-    mi.threads = threads;
-    mi.smem_bytes = K.smem_bytes;
-    mi.occ = occupancy(dev, threads, K.smem_bytes, kernel_regs(kind, P.W));
-    if (mi.occ < 1) return;
-    const int64_t slots = (int64_t)dev.sms * mi.occ;
-    if (kind == KK_PIPE) {
-      // persistent: one CTA per resident slot, striding over the tiles
-      K.tpc = 1;
-      mi.grid = (int)std::min<int64_t>(K.num_tiles, slots);
-      if (hints && hints->grid > 0) mi.grid = hints->grid;
+    TileSummary S;
+    if (!summarize(P, T, group, S)) return;
+    TileParams K0;
+    bool built = false;
+    double conf_load = 1.0, conf_store = 1.0;
+    const int buf_bytes = S.buf_bytes;
+    int kinds[2], nk = 0;
+    if (group == KK_DIRECT) {
+      kinds[nk++] = KK_DIRECT;
     } else {
-      // tiles per CTA: 1 while there are >= 8 waves of tiles, else amortise the
-      // per-CTA table build over up to 4 consecutive tiles
-      int tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, K.num_tiles / (8 * slots)));
-      if (hints && hints->grid > 0) tpc = (int)ceil_div(K.num_tiles, hints->grid);
-      K.tpc = tpc;
-      mi.grid = (int)ceil_div(K.num_tiles, tpc);
+      if (hv != 2) kinds[nk++] = KK_TILE;
+      if (hv != 1) kinds[nk++] = KK_PIPE;
     }
-    // effective run lengths averaged over partial tiles
-    mi.fillA = (double)N / ((double)K.num_tiles * K.V);
-    mi.conf_load = mi.conf_store = 1.0;
-    if (kind != KK_DIRECT) smem_conflicts(K, P.W, mi.conf_load, mi.conf_store);
-    const double tm = predict_seconds(mi, dev);
-    ncand++;
-    if (sink && sink->n < sink->max) {
-      ttlg_plan_info &ci = sink->out[sink->n++];
-      fill_info(ci, dt, rank, P, T, K, mi, schema, kind, tm, 0);
-      const ModelFeatures F = model_features(mi, dev);
-      ci.num_features = kModelFeatureCount;
-      for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
-    }
-    if (tm < best_t) {
-      best_t = tm;
-      best_mi = mi;
-      bestK = K;
-      bestT = T;
-      best_kind = kind;
-      best_schema = schema;
-    }
-  };
-
-  // kernel variants and block sizes competing for each slice candidate
-  const int hv = hints ? hints->variant : 0;
-  const int nthr = (hints && hints->threads) ? 1 : 2;
-  const int thr_list[2] = {(hints && hints->threads) ? hints->threads : 256, 512};
-  auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
-    for (int ti = 0; ti < nthr; ti++) {
-      if (group == KK_DIRECT) {
-        consider1(KK_DIRECT, thr_list[ti], a, ta, b, tb);
-      } else {
-        if (hv != 2) consider1(KK_TILE, thr_list[ti], a, ta, b, tb);
-        if (hv != 1) consider1(KK_PIPE, thr_list[ti], a, ta, b, tb);
+    // pass 0 screens the geometry with the cheap summary and conflict-free
+    // shared memory (bank conflicts only add time: non-negative coefficients);
+    // pass 1 builds the parameter block, analyses conflicts and scores for real
+    for (int pass = 0; pass < 2; pass++) {
+      if (pass == 1) {
+        if (!build_params(P, T, group, thr_list[0], 1, K0)) return;
+        built = true;
+        if (group != KK_DIRECT) smem_conflicts(K0, P.W, conf_load, conf_store);
       }
+      bool any_better = false;
+      for (int ki = 0; ki < nk; ki++) {
+        const int kind = kinds[ki];
+        for (int ti = 0; ti < nthr; ti++) {
+          const int threads = thr_list[ti];
+          const int smem = S.smem_base + (kind == KK_PIPE ? buf_bytes : 0);
+          if (smem > dev.smem_per_block_optin) continue;
+          ModelInput mi;
+          mi.kind = kind;
+          mi.schema = schema;
+          mi.W = P.W;
+          mi.N = N;
+          mi.V = (int)S.V;
+          mi.LA = (int)S.LA;
+          mi.LB = (int)S.LB;
+          mi.RA = (int)S.RA;
+          mi.RB = (int)S.RB;
+          mi.num_tiles = S.tiles;
+          mi.threads = threads;
+          mi.smem_bytes = smem;
+          mi.occ = occupancy(dev, threads, smem, kernel_regs(kind, P.W));
+          if (mi.occ < 1) continue;
+          const int64_t slots = (int64_t)dev.sms * mi.occ;
+          int tpc = 1;
+          if (kind == KK_PIPE) {
+            // persistent: one CTA per resident slot, striding over the tiles
+            mi.grid = (int)std::min<int64_t>(S.tiles, slots);
+            if (hints && hints->grid > 0) mi.grid = hints->grid;
+          } else {
+            // tiles per CTA: 1 while there are >= 8 waves of tiles, else
+            // amortise the per-CTA table build over up to 4 consecutive tiles
+            tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, S.tiles / (8 * slots)));
+            if (hints && hints->grid > 0) tpc = (int)ceil_div(S.tiles, hints->grid);
+            mi.grid = (int)ceil_div(S.tiles, tpc);
+          }
+          // effective run lengths averaged over partial tiles
+          mi.fillA = (double)N / ((double)S.tiles * S.V);
+          mi.conf_load = conf_load;
+          mi.conf_store = conf_store;
+          const double tm = predict_seconds(mi, dev);
+          if (pass == 0) {
+            any_better |= tm < best_t;
+            continue;
+          }
+          ncand++;
+          // a variant differs from K0 only in a few scalars (second buffer of
+          // the cp.async ring, per-thread stepping, tiles per CTA)
+          auto materialise = [&](TileParams &K) {
+            K = K0;
+            if (kind == KK_PIPE) {
+              K.off_data2 = K.off_data + buf_bytes;
+              K.smem_bytes = smem;
+            }
+            K.drA = threads / K.LA;
+            K.dxA = threads % K.LA;
+            K.drB = threads / K.LB;
+            K.dxB = threads % K.LB;
+            K.tpc = tpc;
+          };
+          if (sink && sink->n < sink->max) {
+            TileParams K;
+            materialise(K);
+            ttlg_plan_info &ci = sink->out[sink->n++];
+            fill_info(ci, dt, rank, P, T, K, mi, schema, kind, tm, 0);
+            const ModelFeatures F = model_features(mi, dev);
+            ci.num_features = kModelFeatureCount;
+            for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
+          }
+          if (tm < best_t) {
+            best_t = tm;
+            best_mi = mi;
+            materialise(bestK);
+            bestT = T;
+            best_kind = kind;
+            best_schema = schema;
+          }
+        }
+      }
+      if (pass == 0 && !any_better && !sink) return;
     }
+    (void)built;
   };
 
   int64_t blocksA[32], blocksB[32];
@@ -620,7 +724,6 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (pre * P.W >= 256 * 1024 && !(hints && hints->in_dim > a)) break;
     }
   }
-  const int staged_kind = KK_TILE;
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
@@ -634,7 +737,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                                     kRunTargets);
         for (int i = 0; i < nbA; i++) {
           for (int j = 0; j < nbB; j++) {
-            consider(staged_kind, a, blocksA[i], b, blocksB[j]);
+            consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
           }
         }
         preB *= P.n[pb];
