@@ -259,7 +259,7 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
 //                in registers; NJ = 0: column offsets read from the table.
 // Loop trip counts are warp-uniform and the bodies predicated, so no
 // divergence/reconvergence bookkeeping is generated in the hot loops.
-template <int W, int NJ, bool GA32, bool GB32, bool PERSIST>
+template <int W, int NJ, bool GA32, bool GB32, bool PERSIST, bool XT>
 __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
@@ -286,6 +286,18 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
     }
     reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
   }
+  if constexpr (XT) {
+    for (int x = threadIdx.x; x < P.LA; x += blockDim.x) {
+      int rem = x, s = 0;
+      for (int k = 0; k < P.ni; k++) {
+        const int cq = (int)fdiv((uint32_t)rem, P.i_div[k]);
+        s += (rem - cq * (int)P.i_div[k].div) * P.i_sS[k];
+        rem = cq;
+      }
+      reinterpret_cast<int *>(smem + P.off_icol)[x] = s * W;  // byte offset
+    }
+  }
+  const uint32_t s_icol = s0 + P.off_icol;
   __syncthreads();
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -317,9 +329,19 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
       const int2 t = lds_int2(s_tabA + 8 * r);
       const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
       const T *src = Ab + t.x;
-      const uint32_t dst = sb + t.y * W;
-      for (int k = 0; k < kA; k++)
-        cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
+      if constexpr (XT) {
+        // padded input run: smem offset of run position x from the icol table
+        const uint32_t rowS = sbuf + t.y * W;
+        for (int k = 0; k < kA; k++) {
+          const int x = xA0 + (k << lgA);
+          const int off = x < LA ? lds_int(s_icol + 4 * x) : 0;
+          cp_async_p<W>(rowS + off, src + (k << lgA), rok && x < lim);
+        }
+      } else {
+        const uint32_t dst = sb + t.y * W;
+        for (int k = 0; k < kA; k++)
+          cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
+      }
     }
   };
   // store phase of one tile: B-row r <- smem through the column offsets
@@ -390,26 +412,32 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W, bool GA32, bool PERSIST>
+template <int W, bool GA32, bool PERSIST, bool XT>
 static const void *kernel_ptr_pipe(int nj, bool gb32) {
-  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false, PERSIST>;  // LB < 32: one slot
+  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false, PERSIST, XT>;  // LB < 32: one slot
   switch (nj) {
-    case 1: return (const void *)k_pipe<W, 1, GA32, true, PERSIST>;
-    case 2: return (const void *)k_pipe<W, 2, GA32, true, PERSIST>;
-    case 4: return (const void *)k_pipe<W, 4, GA32, true, PERSIST>;
-    case 8: return (const void *)k_pipe<W, 8, GA32, true, PERSIST>;
+    case 1: return (const void *)k_pipe<W, 1, GA32, true, PERSIST, XT>;
+    case 2: return (const void *)k_pipe<W, 2, GA32, true, PERSIST, XT>;
+    case 4: return (const void *)k_pipe<W, 4, GA32, true, PERSIST, XT>;
+    case 8: return (const void *)k_pipe<W, 8, GA32, true, PERSIST, XT>;
   }
-  return (const void *)k_pipe<W, 16, GA32, true, PERSIST>;  // LB <= 512 (planner cap)
+  return (const void *)k_pipe<W, 16, GA32, true, PERSIST, XT>;  // LB <= 512 (planner cap)
+}
+
+template <int W, bool XT>
+static const void *kernel_ptr_x(int kind, int nj, bool ga32, bool gb32) {
+  if (kind == KK_PIPE)
+    return ga32 ? kernel_ptr_pipe<W, true, true, XT>(nj, gb32)
+                : kernel_ptr_pipe<W, false, true, XT>(nj, gb32);
+  return ga32 ? kernel_ptr_pipe<W, true, false, XT>(nj, gb32)
+              : kernel_ptr_pipe<W, false, false, XT>(nj, gb32);
 }
 
 template <int W>
-static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32, bool xt) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
-  if (kind == KK_PIPE)
-    return ga32 ? kernel_ptr_pipe<W, true, true>(nj, gb32)
-                : kernel_ptr_pipe<W, false, true>(nj, gb32);
-  return ga32 ? kernel_ptr_pipe<W, true, false>(nj, gb32)
-              : kernel_ptr_pipe<W, false, false>(nj, gb32);
+  return xt ? kernel_ptr_x<W, true>(kind, nj, ga32, gb32)
+            : kernel_ptr_x<W, false>(kind, nj, ga32, gb32);
 }
 
 static int pow2_at_least(int k) {
@@ -424,11 +452,11 @@ static int nj_of(const TileParams &K) {
   return k <= 16 ? k : 0;
 }
 
-static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32, bool xt) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32);
-    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32);
-    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32);
+    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32, xt);
+    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32, xt);
+    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32, xt);
   }
   return nullptr;
 }
@@ -442,7 +470,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 4, true, true)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 4, true, true, false)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -454,7 +482,7 @@ int kernel_regs(int kind, int W) {
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
   const void *fn = kernel_ptr(plan->kind, plan->W, nj_of(plan->kp), plan->kp.lgA == 5,
-                              plan->kp.lgB == 5);
+                              plan->kp.lgB == 5, plan->kp.xtab != 0);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

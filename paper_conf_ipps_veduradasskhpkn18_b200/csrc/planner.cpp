@@ -226,7 +226,7 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
 
 // Fill TileParams for a tile; returns false if it violates a kernel limit.
 static bool build_params(const Problem &P, const Tile &T, int kind, int threads, int nbuf,
-                         TileParams &K) {
+                         TileParams &K, const int *isdelta = nullptr) {
   memset(&K, 0, sizeof(K));
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
@@ -282,12 +282,20 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   // in output order with a pad so that the output-run position j maps to
   // bank j mod (128/W) -- the generalisation of the 32x33 pad (L747-749) and of
   // FMS's "row 1 starts at bank N0" rule (L1104-1107).
+  // `isdelta` (optional) pads input-run dims k >= 1 by isdelta[k] elements:
+  // the input run is then no longer contiguous in shared memory and the
+  // kernel reads per-position offsets from the icol table (overlapping
+  // groups whose output-run digits would otherwise share banks, the
+  // Orthogonal-Arbitrary conflicts of L1016-1020).
   int64_t sm[TTLG_MAXD];
   for (int k = 0; k < d; k++) sm[k] = 0;
   int64_t cur = 1;
+  bool xtab = false;
   for (int k = 0; k <= a; k++) {
-    sm[k] = cur;
-    cur *= T.t[k];
+    const int64_t pad = (isdelta && k > 0 && T.t[k] > 1) ? isdelta[k] : 0;
+    xtab |= pad != 0;
+    sm[k] = cur + pad;
+    cur = sm[k] * T.t[k];
   }
   const int64_t Wb = 128 / P.W;
   int64_t Q = 1;
@@ -342,6 +350,17 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   }
   if (smem_elems >= (1ll << 30)) return false;
   K.smem_elems = (int32_t)smem_elems;
+  // input-run digits (input order) -> icol table when the run is padded
+  K.xtab = xtab ? 1 : 0;
+  K.ni = 0;
+  if (xtab) {
+    for (int k = 0; k <= a; k++) {
+      if (T.t[k] <= 1) continue;
+      K.i_div[K.ni] = make_fastdiv((uint32_t)T.t[k]);
+      K.i_sS[K.ni] = (int32_t)sm[k];
+      K.ni++;
+    }
+  }
 
   // shared-memory carve-up (bytes)
   int64_t off = 0;
@@ -356,6 +375,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.off_jcol = take((int64_t)K.LB * 4);
     K.off_digB = take((int64_t)K.RA * 4);
     K.off_digA = take((int64_t)K.RB * 4);
+    K.off_icol = xtab ? take((int64_t)K.LA * 4) : 0;
     K.off_data = take(smem_elems * P.W);
     K.off_data2 = K.off_data;
     for (int s = 1; s < nbuf; s++) {
@@ -434,15 +454,20 @@ static void smem_conflicts(const TileParams &K, int W, double &load, double &sto
   // closed-form fast paths: a whole warp on one A-row reads consecutive words;
   // a whole warp on one B-row whose first output digit spans the warp with an
   // odd shared-memory stride (the padding rule) hits distinct banks
-  const bool load_free = K.lgA == 5;
+  const bool load_free = K.lgA == 5 && !K.xtab;
   const bool store_free = K.lgB == 5 && K.nj > 0 && K.j_ext[0] >= 32 && (K.j_sS[0] & 1);
   load = store = 1.0;
   if (!load_free) {
     const int g = 1 << K.lgA, nr = std::min(32 >> K.lgA, K.RA);
     offsets(nr, K.nra, K.ra_ext, K.ra_sS, rows);
+    if (K.xtab) {
+      int32_t iext[TTLG_MAXD];
+      for (int k = 0; k < K.ni; k++) iext[k] = (int32_t)K.i_div[k].div;
+      offsets(std::min(g, K.LA), K.ni, iext, K.i_sS, cols);
+    }
     for (int l = 0; l < 32; l++) {
       const int r = std::min(l >> K.lgA, nr - 1), x = std::min(l & (g - 1), K.LA - 1);
-      addr[l] = rows[r] + x;
+      addr[l] = rows[r] + (K.xtab ? cols[x] : x);
     }
     load = wavefront_ratio(addr, W);
   }
@@ -607,7 +632,6 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     TileParams K0;
     bool built = false;
     double conf_load = 1.0, conf_store = 1.0;
-    const int buf_bytes = S.buf_bytes;
     int kinds[2], nk = 0;
     if (group == KK_DIRECT) {
       kinds[nk++] = KK_DIRECT;
@@ -622,13 +646,42 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (pass == 1) {
         if (!build_params(P, T, group, thr_list[0], 1, K0)) return;
         built = true;
-        if (group != KK_DIRECT) smem_conflicts(K0, P.W, conf_load, conf_store);
+        if (group != KK_DIRECT) {
+          smem_conflicts(K0, P.W, conf_load, conf_store);
+          if (conf_load + conf_store > 2.0) {
+            // greedy padding of the input-run dims (k >= 1) to remove conflicts
+            int delta[TTLG_MAXD] = {0};
+            const int lp = 128 / P.W;
+            const int opts[6] = {1, 2, 3, lp / 2, lp / 2 + 1, lp - 1};
+            for (int k = 1; k <= a && conf_load + conf_store > 2.0; k++) {
+              if (T.t[k] <= 1) continue;
+              int best_d = 0;
+              for (int o = 0; o < 6; o++) {
+                delta[k] = opts[o];
+                TileParams Kt;
+                if (!build_params(P, T, group, thr_list[0], 1, Kt, delta)) continue;
+                double cl, cs;
+                smem_conflicts(Kt, P.W, cl, cs);
+                if (cl + cs < conf_load + conf_store - 1e-9) {
+                  conf_load = cl;
+                  conf_store = cs;
+                  best_d = opts[o];
+                }
+              }
+              delta[k] = best_d;
+            }
+            if (!build_params(P, T, group, thr_list[0], 1, K0, delta)) return;
+          }
+          S.smem_base = K0.smem_bytes;
+          S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
+        }
       }
       bool any_better = false;
       for (int ki = 0; ki < nk; ki++) {
         const int kind = kinds[ki];
         for (int ti = 0; ti < nthr; ti++) {
           const int threads = thr_list[ti];
+          const int buf_bytes = S.buf_bytes;
           const int smem = S.smem_base + (kind == KK_PIPE ? buf_bytes : 0);
           if (smem > dev.smem_per_block_optin) continue;
           ModelInput mi;
@@ -735,9 +788,16 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         const int pb = P.p[b];
         const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0,
                                     kRunTargets);
-        for (int i = 0; i < nbA; i++) {
-          for (int j = 0; j < nbB; j++) {
-            consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
+        if (pb == a) {
+          // the same dim closes both groups (overlap): one shared blocking
+          // factor, drawn from both candidate lists
+          for (int i = 0; i < nbA; i++) consider(KK_TILE, a, blocksA[i], b, blocksA[i]);
+          for (int j = 0; j < nbB; j++) consider(KK_TILE, a, blocksB[j], b, blocksB[j]);
+        } else {
+          for (int i = 0; i < nbA; i++) {
+            for (int j = 0; j < nbB; j++) {
+              consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
+            }
           }
         }
         preB *= P.n[pb];

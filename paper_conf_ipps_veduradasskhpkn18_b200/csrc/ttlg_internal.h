@@ -95,6 +95,11 @@ struct TileParams {
   int32_t j_ext[TTLG_MAXD];
   int32_t j_sS[TTLG_MAXD];
   FastDiv j_div[TTLG_MAXD];
+  // ---- input-run digits, input order (-> smem offsets when the run is padded)
+  int32_t xtab, ni;        // xtab: 1 = input run padded in smem, read icol table
+  FastDiv i_div[TTLG_MAXD];
+  int32_t i_sS[TTLG_MAXD];
+  int32_t off_icol;
   // ---- shared-memory layout (bytes) and per-thread stepping
   int32_t smem_elems;      // data tile elements incl. padding
   int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
