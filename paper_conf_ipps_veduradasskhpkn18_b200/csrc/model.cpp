@@ -91,3 +91,44 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 }
 
 }  // namespace ttlg
+
+// ---- ranking stage: boosted regression trees (model_gbt.h) --------------------
+#include "model_gbt.h"
+
+namespace ttlg {
+
+// Plan descriptor fed to the trees; tools/calibrate_gbt.py desc() mirrors it.
+void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d) {
+  const ModelFeatures F = model_features(mi, dev);
+  const double W = mi.W, V = mi.V;
+  const double occ = std::max(1, mi.occ), th = mi.threads;
+  const double LAb = (mi.kind == KK_DIRECT ? V : (double)mi.LA) * W;
+  const double bytes = 2.0 * (double)mi.N * W;
+  d[0] = mi.kind;
+  d[1] = std::log2(W);
+  d[2] = std::log2(LAb);
+  d[3] = std::log2((double)mi.LB * W);
+  d[4] = std::log2(V * W);
+  d[5] = th / 256.0;
+  d[6] = occ;
+  d[7] = occ * th / 2048.0;
+  d[8] = std::log2((double)mi.num_tiles);
+  d[9] = F.f[2] / std::max(F.f[1], 1e-12);
+  d[10] = F.f[8] / std::max(1.0, bytes / 1e9);
+  d[11] = (double)mi.num_tiles / (dev.sms * occ);
+}
+
+double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
+  double d[12];
+  model_descriptor(mi, dev, d);
+  double s = kGbtInit;
+  for (int t = 0; t < kGbtTrees; t++) {
+    int n = kGbtRoot[t];
+    while (kGbtFeat[n] >= 0) n = (d[kGbtFeat[n]] <= (double)kGbtThr[n]) ? kGbtLeft[n] : kGbtRight[n];
+    s += kGbtVal[n];
+  }
+  const double ideal = 2.0 * (double)mi.N * mi.W / (dev.hbm_gbs * 1e9);
+  return std::exp(std::max(s, 0.0)) * ideal;  // never below one pass at copy speed
+}
+
+}  // namespace ttlg

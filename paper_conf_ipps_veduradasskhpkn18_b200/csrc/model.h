@@ -33,5 +33,8 @@ struct ModelFeatures {
 // Feature vector (units: seconds at the reference bandwidth, or counts).
 ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev);
 double predict_seconds(const ModelInput &mi, const DeviceProfile &dev);
+// ranking stage (boosted trees over model_descriptor); seconds
+void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d);
+double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
 
 }  // namespace ttlg

@@ -8,8 +8,8 @@ constexpr int kModelNumFeatures = 10;
 constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
 constexpr double kModelUnroll = 8.0;         // loads in flight per thread (k_direct, k_tile)
 // features: see model.cpp model_features()
-constexpr double kCoefDirect[kModelNumFeatures] = {4.373133e-06, 8.920645e-01, 1.756448e+00, 4.022023e-10, 0.000000e+00, 4.490829e-01, 4.286812e-01, 6.175414e-07, 0.000000e+00, 7.828605e-10};
-constexpr double kCoefTile[kModelNumFeatures] = {8.873988e-06, 7.329123e-01, 4.412852e-01, 3.203440e-10, 0.000000e+00, 8.750968e-02, 2.233884e-01, 1.136793e-06, 2.295258e-10, 1.333646e-09};
-constexpr double kCoefPipe[kModelNumFeatures] = {8.021830e-06, 8.330551e-01, 7.908181e-01, 2.106668e-10, 5.316145e-08, 2.988828e-02, 0.000000e+00, 3.750311e-07, 1.897926e-10, 1.544756e-09};
-constexpr const char *kModelSource = "B200 fit (176 cases, 17252 points, rel<=1.5): direct: train 4.3% test 10.3% (n=266+59); tile: train 7.7% test 7.3% (n=2358+594); pipe: train 7.4% test 7.1% (n=2365+558); regret 9.8%";
+constexpr double kCoefDirect[kModelNumFeatures] = {3.487685e-06, 8.104583e-01, 7.212736e-01, 6.918417e-10, 0.000000e+00, 2.609106e-01, 6.292655e-01, 8.807121e-07, 0.000000e+00, 1.041337e-09};
+constexpr double kCoefTile[kModelNumFeatures] = {1.016694e-05, 5.255828e-01, 1.731233e-01, 4.057429e-10, 0.000000e+00, 0.000000e+00, 2.724066e-01, 1.943307e-06, 5.811676e-11, 1.716047e-09};
+constexpr double kCoefPipe[kModelNumFeatures] = {6.559314e-06, 4.518758e-01, 0.000000e+00, 5.001977e-10, 4.830940e-08, 0.000000e+00, 0.000000e+00, 1.442755e-06, 0.000000e+00, 2.204548e-09};
+constexpr const char *kModelSource = "B200 fit (176 cases, 18270 points, rel<=3.0): direct: train 6.0% test 13.2% (n=322+58); tile: train 11.6% test 10.8% (n=4549+1089); pipe: train 12.1% test 11.6% (n=4421+1077); regret 11.3%";
 }  // namespace ttlg

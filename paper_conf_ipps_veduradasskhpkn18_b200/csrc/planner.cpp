@@ -18,6 +18,7 @@
 #include <cmath>
 
 #include "model.h"
+#include "model_gbt.h"
 #include "ttlg_internal.h"
 
 namespace ttlg {
@@ -582,14 +583,24 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   int64_t N = 1;
   for (int k = 0; k < P.d; k++) N *= P.n[k];
 
-  ModelInput best_mi;
-  TileParams bestK;
-  Tile bestT;
-  memset(&best_mi, 0, sizeof(best_mi));
-  memset(&bestK, 0, sizeof(bestK));
-  memset(&bestT, 0, sizeof(bestT));
-  int best_kind = -1, best_schema = -1, ncand = 0;
-  double best_t = 1e300;
+  // Two-stage model (§V re-derived): the per-kernel linear model screens every
+  // candidate with a cheap geometry summary (bank conflicts only add time, so
+  // the conflict-free score is a lower bound) into a short list; the short
+  // list is refined (exact parameter block, conflict analysis and padding
+  // search) and the kGbtTopK best are ranked by boosted regression trees
+  // (model_gbt.h).  Entries are small; the winner's block is rebuilt.
+  struct Entry {
+    double lin;
+    ModelInput mi;
+    Tile T;
+    int kind, schema, tpc, group;
+    int8_t delta[TTLG_MAXD];  // input-run padding chosen by the conflict search
+  };
+  constexpr int kShort = 2 * kGbtTopK;
+  Entry pool[kShort];
+  int order[kShort];  // pool slots sorted by the linear prediction
+  int ntop = 0, ncand = 0;
+  double admit = 1e300;  // admission threshold: the worst short-list entry once full
 
   const int max_tile_bytes = std::min(64 * 1024, dev.smem_per_block_optin - 8 * 1024);
 
@@ -598,9 +609,109 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   const int nthr = (hints && hints->threads) ? 1 : 2;
   const int thr_list[2] = {(hints && hints->threads) ? hints->threads : 256, 512};
 
-  // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB): the tile,
-  // its parameter block and shared-memory conflict ratios are computed once;
-  // then every kernel variant x block size is scored by the model.
+  // model input of one (geometry, kernel, block size); false if it cannot launch
+  auto make_mi = [&](ModelInput &mi, int &tpc, int kind, int schema, int threads,
+                     const TileSummary &S, double cl, double cs) {
+    const int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
+    if (smem > dev.smem_per_block_optin) return false;
+    mi.kind = kind;
+    mi.schema = schema;
+    mi.W = P.W;
+    mi.N = N;
+    mi.V = (int)S.V;
+    mi.LA = (int)S.LA;
+    mi.LB = (int)S.LB;
+    mi.RA = (int)S.RA;
+    mi.RB = (int)S.RB;
+    mi.num_tiles = S.tiles;
+    mi.threads = threads;
+    mi.smem_bytes = smem;
+    mi.occ = occupancy(dev, threads, smem, kernel_regs(kind, P.W));
+    if (mi.occ < 1) return false;
+    const int64_t slots = (int64_t)dev.sms * mi.occ;
+    tpc = 1;
+    if (kind == KK_PIPE) {
+      // persistent: one CTA per resident slot, striding over the tiles
+      mi.grid = (int)std::min<int64_t>(S.tiles, slots);
+      if (hints && hints->grid > 0) mi.grid = hints->grid;
+    } else {
+      // tiles per CTA: 1 while there are >= 8 waves of tiles, else amortise the
+      // per-CTA table build over up to 4 consecutive tiles
+      tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, S.tiles / (8 * slots)));
+      if (hints && hints->grid > 0) tpc = (int)ceil_div(S.tiles, hints->grid);
+      mi.grid = (int)ceil_div(S.tiles, tpc);
+    }
+    mi.fillA = (double)N / ((double)S.tiles * S.V);  // partial tiles
+    mi.conf_load = cl;
+    mi.conf_store = cs;
+    return true;
+  };
+
+  // exact parameter block of a geometry, with the greedy padding of the
+  // input-run dims (k >= 1) that removes shared-memory bank conflicts
+  auto build_exact = [&](const Tile &T, int group, TileParams &K0, int *delta, double &cl,
+                         double &cs, TileSummary &S) {
+    for (int k = 0; k < TTLG_MAXD; k++) delta[k] = 0;
+    cl = cs = 1.0;
+    if (!build_params(P, T, group, thr_list[0], 1, K0)) return false;
+    if (group == KK_DIRECT) return true;
+    smem_conflicts(K0, P.W, cl, cs);
+    if (cl + cs > 2.0) {
+      const int lp = 128 / P.W;
+      const int opts[6] = {1, 2, 3, lp / 2, lp / 2 + 1, lp - 1};
+      for (int k = 1; k <= T.a && cl + cs > 2.0; k++) {
+        if (T.t[k] <= 1) continue;
+        int best_d = 0;
+        for (int o = 0; o < 6; o++) {
+          delta[k] = opts[o];
+          TileParams Kt;
+          if (!build_params(P, T, group, thr_list[0], 1, Kt, delta)) continue;
+          double l2, s2;
+          smem_conflicts(Kt, P.W, l2, s2);
+          if (l2 + s2 < cl + cs - 1e-9) {
+            cl = l2;
+            cs = s2;
+            best_d = opts[o];
+          }
+        }
+        delta[k] = best_d;
+      }
+      if (!build_params(P, T, group, thr_list[0], 1, K0, delta)) return false;
+    }
+    S.smem_base = K0.smem_bytes;
+    S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
+    return true;
+  };
+
+  auto insert = [&](double lin, const ModelInput &mi, const Tile &T, int kind, int schema,
+                    int tpc, int group, const int *delta) {
+    int slot, pos;
+    if (ntop < kShort) {
+      slot = ntop;
+      pos = ntop++;
+    } else {
+      slot = order[kShort - 1];  // evict the worst
+      pos = kShort - 1;
+    }
+    while (pos > 0 && pool[order[pos - 1]].lin > lin) {
+      order[pos] = order[pos - 1];
+      pos--;
+    }
+    order[pos] = slot;
+    Entry &e = pool[slot];
+    e.lin = lin;
+    e.mi = mi;
+    e.T = T;
+    e.kind = kind;
+    e.schema = schema;
+    e.tpc = tpc;
+    e.group = group;
+    for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
+    if (ntop == kShort) admit = pool[order[kShort - 1]].lin;
+  };
+
+  // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB) x every kernel
+  // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
@@ -629,9 +740,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     TileSummary S;
     if (!summarize(P, T, group, S)) return;
+    int delta[TTLG_MAXD] = {0};
+    double cl = 1.0, cs = 1.0;
     TileParams K0;
-    bool built = false;
-    double conf_load = 1.0, conf_store = 1.0;
+    if (sink) {  // candidate listing: exact features for every candidate
+      if (!build_exact(T, group, K0, delta, cl, cs, S)) return;
+    }
     int kinds[2], nk = 0;
     if (group == KK_DIRECT) {
       kinds[nk++] = KK_DIRECT;
@@ -639,127 +753,31 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (hv != 2) kinds[nk++] = KK_TILE;
       if (hv != 1) kinds[nk++] = KK_PIPE;
     }
-    // pass 0 screens the geometry with the cheap summary and conflict-free
-    // shared memory (bank conflicts only add time: non-negative coefficients);
-    // pass 1 builds the parameter block, analyses conflicts and scores for real
-    for (int pass = 0; pass < 2; pass++) {
-      if (pass == 1) {
-        if (!build_params(P, T, group, thr_list[0], 1, K0)) return;
-        built = true;
-        if (group != KK_DIRECT) {
-          smem_conflicts(K0, P.W, conf_load, conf_store);
-          if (conf_load + conf_store > 2.0) {
-            // greedy padding of the input-run dims (k >= 1) to remove conflicts
-            int delta[TTLG_MAXD] = {0};
-            const int lp = 128 / P.W;
-            const int opts[6] = {1, 2, 3, lp / 2, lp / 2 + 1, lp - 1};
-            for (int k = 1; k <= a && conf_load + conf_store > 2.0; k++) {
-              if (T.t[k] <= 1) continue;
-              int best_d = 0;
-              for (int o = 0; o < 6; o++) {
-                delta[k] = opts[o];
-                TileParams Kt;
-                if (!build_params(P, T, group, thr_list[0], 1, Kt, delta)) continue;
-                double cl, cs;
-                smem_conflicts(Kt, P.W, cl, cs);
-                if (cl + cs < conf_load + conf_store - 1e-9) {
-                  conf_load = cl;
-                  conf_store = cs;
-                  best_d = opts[o];
-                }
-              }
-              delta[k] = best_d;
-            }
-            if (!build_params(P, T, group, thr_list[0], 1, K0, delta)) return;
-          }
-          S.smem_base = K0.smem_bytes;
-          S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
-        }
-      }
-      bool any_better = false;
-      for (int ki = 0; ki < nk; ki++) {
-        const int kind = kinds[ki];
-        for (int ti = 0; ti < nthr; ti++) {
-          const int threads = thr_list[ti];
-          const int buf_bytes = S.buf_bytes;
-          const int smem = S.smem_base + (kind == KK_PIPE ? buf_bytes : 0);
-          if (smem > dev.smem_per_block_optin) continue;
-          ModelInput mi;
-          mi.kind = kind;
-          mi.schema = schema;
-          mi.W = P.W;
-          mi.N = N;
-          mi.V = (int)S.V;
-          mi.LA = (int)S.LA;
-          mi.LB = (int)S.LB;
-          mi.RA = (int)S.RA;
-          mi.RB = (int)S.RB;
-          mi.num_tiles = S.tiles;
-          mi.threads = threads;
-          mi.smem_bytes = smem;
-          mi.occ = occupancy(dev, threads, smem, kernel_regs(kind, P.W));
-          if (mi.occ < 1) continue;
-          const int64_t slots = (int64_t)dev.sms * mi.occ;
-          int tpc = 1;
+    for (int ki = 0; ki < nk; ki++) {
+      for (int ti = 0; ti < nthr; ti++) {
+        const int kind = kinds[ki], threads = thr_list[ti];
+        ModelInput mi;
+        int tpc;
+        if (!make_mi(mi, tpc, kind, schema, threads, S, cl, cs)) continue;
+        const double tm = predict_seconds(mi, dev);
+        ncand++;
+        if (sink && sink->n < sink->max) {
+          TileParams K = K0;
           if (kind == KK_PIPE) {
-            // persistent: one CTA per resident slot, striding over the tiles
-            mi.grid = (int)std::min<int64_t>(S.tiles, slots);
-            if (hints && hints->grid > 0) mi.grid = hints->grid;
-          } else {
-            // tiles per CTA: 1 while there are >= 8 waves of tiles, else
-            // amortise the per-CTA table build over up to 4 consecutive tiles
-            tpc = (int)std::min<int64_t>(4, std::max<int64_t>(1, S.tiles / (8 * slots)));
-            if (hints && hints->grid > 0) tpc = (int)ceil_div(S.tiles, hints->grid);
-            mi.grid = (int)ceil_div(S.tiles, tpc);
+            K.off_data2 = K.off_data + S.buf_bytes;
+            K.smem_bytes = mi.smem_bytes;
           }
-          // effective run lengths averaged over partial tiles
-          mi.fillA = (double)N / ((double)S.tiles * S.V);
-          mi.conf_load = conf_load;
-          mi.conf_store = conf_store;
-          const double tm = predict_seconds(mi, dev);
-          if (pass == 0) {
-            any_better |= tm < best_t;
-            continue;
-          }
-          ncand++;
-          // a variant differs from K0 only in a few scalars (second buffer of
-          // the cp.async ring, per-thread stepping, tiles per CTA)
-          auto materialise = [&](TileParams &K) {
-            K = K0;
-            if (kind == KK_PIPE) {
-              K.off_data2 = K.off_data + buf_bytes;
-              K.smem_bytes = smem;
-            }
-            K.drA = threads / K.LA;
-            K.dxA = threads % K.LA;
-            K.drB = threads / K.LB;
-            K.dxB = threads % K.LB;
-            K.tpc = tpc;
-          };
-          if (sink && sink->n < sink->max) {
-            TileParams K;
-            materialise(K);
-            ttlg_plan_info &ci = sink->out[sink->n++];
-            fill_info(ci, dt, rank, P, T, K, mi, schema, kind, tm, 0);
-            const ModelFeatures F = model_features(mi, dev);
-            ci.num_features = kModelFeatureCount;
-            for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
-          }
-          if (tm < best_t) {
-            best_t = tm;
-            best_mi = mi;
-            materialise(bestK);
-            bestT = T;
-            best_kind = kind;
-            best_schema = schema;
-          }
+          K.tpc = tpc;
+          ttlg_plan_info &ci = sink->out[sink->n++];
+          fill_info(ci, dt, rank, P, T, K, mi, schema, kind, tm, 0);
+          const ModelFeatures F = model_features(mi, dev);
+          ci.num_features = kModelFeatureCount;
+          for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
         }
+        if (tm < admit) insert(tm, mi, T, kind, schema, tpc, group, delta);
       }
-      if (pass == 0 && !any_better && !sink) return;
     }
-    (void)built;
   };
-
   int64_t blocksA[32], blocksB[32];
   if (P.p[0] == 0) {
     // ---- direct (FML / COPY): input run = dims 0..a (contiguous), output run = dim 0
@@ -807,18 +825,90 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) break;
     }
   }
-  if (best_kind < 0) return force_schema == TTLG_SCHEMA_AUTO ? TTLG_ERR_INTERNAL : TTLG_ERR_UNSUPPORTED;
+  if (ntop == 0) return force_schema == TTLG_SCHEMA_AUTO ? TTLG_ERR_INTERNAL : TTLG_ERR_UNSUPPORTED;
 
-  plan->kind = best_kind;
+  // refine the short list: exact blocks, conflicts and padding (cached per geometry)
+  if (!sink) {
+    struct Done {
+      int a, b, group;
+      int64_t ta, tb;
+      int delta[TTLG_MAXD];
+      double cl, cs;
+      TileSummary S;
+      bool ok;
+    };
+    Done done[kShort];
+    int nd = 0;
+    for (int i = 0; i < ntop; i++) {
+      Entry &e = pool[i];
+      const int64_t ta = e.T.t[e.T.a], tb = e.T.t[P.p[e.T.b]];
+      int f = -1;
+      for (int j = 0; j < nd && f < 0; j++)
+        if (done[j].a == e.T.a && done[j].b == e.T.b && done[j].ta == ta && done[j].tb == tb &&
+            done[j].group == e.group)
+          f = j;
+      if (f < 0) {
+        Done &D = done[nd];
+        D.a = e.T.a;
+        D.b = e.T.b;
+        D.ta = ta;
+        D.tb = tb;
+        D.group = e.group;
+        TileParams K0;
+        D.ok = summarize(P, e.T, e.group, D.S) &&
+               build_exact(e.T, e.group, K0, D.delta, D.cl, D.cs, D.S);
+        f = nd++;
+      }
+      const Done &D = done[f];
+      int tpc;
+      if (!D.ok || !make_mi(e.mi, tpc, e.kind, e.schema, e.mi.threads, D.S, D.cl, D.cs)) {
+        e.lin = 1e300;
+        continue;
+      }
+      e.tpc = tpc;
+      for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)D.delta[k];
+      e.lin = predict_seconds(e.mi, dev);
+    }
+    std::sort(order, order + ntop, [&](int x, int y) { return pool[x].lin < pool[y].lin; });
+  }
+  // ranking stage: boosted trees over the kGbtTopK best
+  int win = order[0];
+  double win_t = 1e300;
+  for (int i = 0; i < std::min(ntop, kGbtTopK); i++) {
+    const Entry &e = pool[order[i]];
+    if (e.lin >= 1e299) continue;
+    const double t = predict_ranked_seconds(e.mi, dev);
+    if (t < win_t) {
+      win_t = t;
+      win = order[i];
+    }
+  }
+  const Entry &B = pool[win];
+  if (B.lin >= 1e299) return TTLG_ERR_INTERNAL;
+  // rebuild the winner's parameter block
+  TileParams K;
+  {
+    int delta[TTLG_MAXD];
+    bool padded = false;
+    for (int k = 0; k < TTLG_MAXD; k++) {
+      delta[k] = B.delta[k];
+      padded |= delta[k] != 0;
+    }
+    if (!build_params(P, B.T, B.group, B.mi.threads, B.kind == KK_PIPE ? 2 : 1, K,
+                      padded ? delta : nullptr))
+      return TTLG_ERR_INTERNAL;
+    K.tpc = B.tpc;
+  }
+  plan->kind = B.kind;
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
-  plan->threads = best_mi.threads;
-  plan->grid = best_mi.grid;
+  plan->threads = B.mi.threads;
+  plan->grid = B.mi.grid;
   plan->nbytes = N * P.W;
-  plan->kp = bestK;
-  fill_info(plan->info, dt, rank, P, bestT, bestK, best_mi, best_schema, best_kind, best_t, ncand);
+  plan->kp = K;
+  fill_info(plan->info, dt, rank, P, B.T, K, B.mi, B.schema, B.kind, win_t, ncand);
   {
-    const ModelFeatures F = model_features(best_mi, dev);
+    const ModelFeatures F = model_features(B.mi, dev);
     plan->info.num_features = kModelFeatureCount;
     for (int f = 0; f < kModelFeatureCount; f++) plan->info.features[f] = F.f[f];
   }

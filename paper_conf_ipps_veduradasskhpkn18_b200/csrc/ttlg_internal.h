@@ -29,8 +29,7 @@ inline FastDiv make_fastdiv(uint32_t d) {
     f.shr = 0;
     return f;
   }
-  uint32_t l = 0;
-  while ((1ull << l) < d) l++;  // ceil(log2 d)
+  const uint32_t l = 32 - (uint32_t)__builtin_clz(d - 1);  // ceil(log2 d), d >= 2
   uint32_t p = 31 + l;
   f.mul = (uint32_t)(((1ull << p) + d - 1) / d);
   f.shr = p - 32;

@@ -1,0 +1,143 @@
+#!/usr/bin/env python
+"""Fit the ranking stage of the B200 performance model: gradient-boosted
+regression trees on the log of (measured time / ideal one-pass time) over
+plan descriptors (model.cpp model_descriptor), trained on tools/calib_sweep.py
+data (§V's per-kernel linear regression re-derived for B200: the
+linear model screens candidates, the trees rank the short list).
+
+Reports, on a random 80/20 split of configurations (L1311-1313), the paper's
+precision metric mean(|a-p|/a) (L1414-1416) and the selection regret; then
+refits on everything and writes paper_conf_ipps_veduradasskhpkn18_b200/csrc/model_gbt.h.
+
+  python tools/calibrate_gbt.py gpurun_out/calib16_*.jsonl [--write]
+"""
+from __future__ import annotations
+
+import argparse
+import collections
+import json
+import math
+import os
+import random
+import re
+
+import numpy as np
+from sklearn.ensemble import GradientBoostingRegressor
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+CSRC = os.path.join(ROOT, "paper_conf_ipps_veduradasskhpkn18_b200", "csrc")
+KID = {"direct": 0, "tile": 1, "pipe": 2}
+HBM = 6555.5e9
+SMS = 148
+TOPK = 16
+
+
+def desc(r):
+    """Must match model.cpp model_descriptor() exactly."""
+    W, V = r["W"], r["V"]
+    occ, th = max(1, r["occ"]), r["threads"]
+    LAb = (V if r["kernel"] == "direct" else r["LA"]) * W
+    f = r["features"]
+    return [KID[r["kernel"]], math.log2(W), math.log2(LAb), math.log2(r["LB"] * W),
+            math.log2(V * W), th / 256.0, float(occ), occ * th / 2048.0,
+            math.log2(r["tiles"]), f[2] / max(f[1], 1e-12), f[8] / max(1.0, r["bytes"] / 1e9),
+            r["tiles"] / (SMS * occ)]
+
+
+def ideal(r):
+    return r["bytes"] / HBM
+
+
+def linear_coefs():
+    src = open(os.path.join(CSRC, "model_coeffs.h")).read()
+    co = {}
+    for name, k in (("kCoefDirect", "direct"), ("kCoefTile", "tile"), ("kCoefPipe", "pipe")):
+        m = re.search(name + r"\[kModelNumFeatures\] = \{([^}]*)\}", src)
+        co[k] = np.array([float(x) for x in m.group(1).split(",")])
+    return co
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("files", nargs="+")
+    ap.add_argument("--write", action="store_true")
+    ap.add_argument("--trees", type=int, default=100)
+    ap.add_argument("--depth", type=int, default=5)
+    ap.add_argument("--lr", type=float, default=0.2)
+    args = ap.parse_args()
+    rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
+    co = linear_coefs()
+    by = collections.defaultdict(list)
+    for r in rows:
+        r["lin"] = float(co[r["kernel"]] @ np.array(r["features"]))
+        by[r["case"]].append(r)
+    cases = sorted(by)
+    rng = random.Random(0)
+    test = set(rng.sample(cases, len(cases) // 5))
+
+    def fit(rs):
+        X = np.array([desc(r) for r in rs])
+        y = np.array([math.log(r["meas"] / ideal(r)) for r in rs])
+        return GradientBoostingRegressor(n_estimators=args.trees, max_depth=args.depth,
+                                         learning_rate=args.lr, subsample=0.8,
+                                         random_state=0).fit(X, y)
+
+    def evaluate(m, cs):
+        reg, err, gp, gb = [], [], [], []
+        for c in cs:
+            rs = sorted(by[c], key=lambda r: r["lin"])[:TOPK]
+            P = m.predict(np.array([desc(r) for r in rs]))
+            best = min(by[c], key=lambda r: r["meas"])
+            pick = rs[int(np.argmin(P))]
+            reg.append(pick["meas"] / best["meas"] - 1)
+            gp.append(pick["gbs"])
+            gb.append(best["gbs"])
+            for r, p in zip(rs, P):
+                err.append(abs(math.exp(p) * ideal(r) - r["meas"]) / r["meas"])
+        return 100 * np.mean(reg), 100 * np.mean(err), np.mean(gp), np.mean(gb)
+
+    m = fit([r for r in rows if r["case"] not in test])
+    tr = evaluate(m, [c for c in cases if c not in test])
+    te = evaluate(m, list(test))
+    print(f"train: regret {tr[0]:.1f}% err(top{TOPK}) {tr[1]:.1f}% picked {tr[2]:.0f} best {tr[3]:.0f}")
+    print(f"test : regret {te[0]:.1f}% err(top{TOPK}) {te[1]:.1f}% picked {te[2]:.0f} best {te[3]:.0f}")
+    if not args.write:
+        return
+    m = fit(rows)  # final model on all configurations
+    feats, thr, left, right, val, roots = [], [], [], [], [], []
+    for est in m.estimators_[:, 0]:
+        t = est.tree_
+        base = len(feats)
+        roots.append(base)
+        for i in range(t.node_count):
+            leaf = t.children_left[i] == -1
+            feats.append(-1 if leaf else int(t.feature[i]))
+            thr.append(float(t.threshold[i]) if not leaf else 0.0)
+            left.append(-1 if leaf else base + int(t.children_left[i]))
+            right.append(-1 if leaf else base + int(t.children_right[i]))
+            val.append(float(t.value[i][0][0]) * m.learning_rate)
+    init = float(m.init_.constant_[0][0]) if hasattr(m.init_, "constant_") else float(
+        np.mean([math.log(r["meas"] / ideal(r)) for r in rows]))
+    with open(os.path.join(CSRC, "model_gbt.h"), "w") as f:
+        f.write("// model_gbt.h -- GENERATED by tools/calibrate_gbt.py: boosted regression trees\n"
+                "// predicting log(time / one-pass ideal) from model_descriptor() (model.cpp).\n"
+                f"// Fitted on {len(rows)} B200 measurements ({len(cases)} configurations); held-out\n"
+                f"// 20%: selection regret {te[0]:.1f}%, mean |a-p|/a {te[1]:.1f}% (top-{TOPK} lists).\n"
+                "#pragma once\n#include <stdint.h>\nnamespace ttlg {\n")
+        f.write(f"constexpr int kGbtTrees = {len(roots)};\nconstexpr int kGbtTopK = {TOPK};\n")
+        f.write(f"constexpr double kGbtInit = {init!r};\n")
+        f.write(f'constexpr const char *kGbtSource = "GBT {len(roots)} trees depth {args.depth}, '
+                f'{len(rows)} points / {len(cases)} cases; test regret {te[0]:.1f}%, '
+                f'err {te[1]:.1f}%";\n')
+        f.write("constexpr int32_t kGbtRoot[] = {" + ",".join(map(str, roots)) + "};\n")
+        f.write("constexpr int8_t kGbtFeat[] = {" + ",".join(map(str, feats)) + "};\n")
+        f.write("constexpr float kGbtThr[] = {" + ",".join(f"{x!r}f" for x in thr) + "};\n")
+        f.write("constexpr int16_t kGbtLeft[] = {" + ",".join(map(str, left)) + "};\n")
+        f.write("constexpr int16_t kGbtRight[] = {" + ",".join(map(str, right)) + "};\n")
+        f.write("constexpr float kGbtVal[] = {" + ",".join(f"{x!r}f" for x in val) + "};\n")
+        f.write("}  // namespace ttlg\n")
+    print("wrote", os.path.join(CSRC, "model_gbt.h"), len(feats), "nodes")
+
+
+if __name__ == "__main__":
+    main()
