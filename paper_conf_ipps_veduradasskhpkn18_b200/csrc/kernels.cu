@@ -310,6 +310,7 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
   const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
   const int kA = (LA + gA - 1) >> lgA;  // uniform per-row trip count (load)
   const int kB = (LB + gB - 1) >> lgB;  // uniform per-row trip count (store)
+  const uint32_t jstrideW = (P.nj == 1 ? (uint32_t)P.j_sS[0] : 0u) * W;  // chunked long runs
   int jc[NJ > 0 ? NJ : 1];
   if constexpr (NJ > 0) {
 #pragma unroll
@@ -355,10 +356,16 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
       T *dst = Bb + t.x;
       const uint32_t src = sbuf + t.y * W;
       if constexpr (NJ > 0) {
+        // runs longer than NJ lane-slots (single output digit only, so the
+        // column offset is linear in j) take several uniform chunks
+        for (int jb = 0; jb < lim; jb += NJ << lgB) {
+          const uint32_t cb = (uint32_t)jb * jstrideW;
 #pragma unroll
-        for (int i = 0; i < NJ; i++) {
-          if (i < kB)
-            stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+          for (int i = 0; i < NJ; i++) {
+            if (i < kB)
+              stcs_p(dst + jb + (i << lgB), lds_T<T>(src + cb + jc[i]),
+                     rok && jb + xB0 + (i << lgB) < lim);
+          }
         }
       } else {
 #pragma unroll 4
@@ -449,7 +456,7 @@ static int pow2_at_least(int k) {
 // per-lane elements of a B-row (NJ <= 16)
 static int nj_of(const TileParams &K) {
   const int k = pow2_at_least((K.LB + (1 << K.lgB) - 1) >> K.lgB);
-  return k <= 16 ? k : 0;
+  return k <= 16 ? k : 16;  // longer runs: single output digit, chunked (planner rule)
 }
 
 static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32, bool xt) {

@@ -732,9 +732,15 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (V * P.W > max_tile_bytes) return;
       // output runs longer than 16 x 32 access elements gain nothing and would
       // need per-element column-table reads (register column offsets, NJ <= 16)
+      // -- except a run of a single output digit, whose offsets are linear and
+      // which the kernel walks in chunks
       int64_t LBc = 1;
-      for (int i = 0; i <= b; i++) LBc *= T.t[P.p[i]];
-      if (LBc > 512) return;
+      int ndig = 0;
+      for (int i = 0; i <= b; i++) {
+        LBc *= T.t[P.p[i]];
+        ndig += T.t[P.p[i]] > 1;
+      }
+      if (LBc > 512 && ndig > 1) return;
     } else if (V * P.W > 256 * 1024) {
       return;
     }

@@ -282,3 +282,17 @@ def test_execute_host_pipeline(ext, perm, eb):
     uv = np.uint64 if eb == 8 else np.uint32
     _assert_equal(B.view(iv).numpy().view(uv),
                   oracle.transpose(A.view(iv).numpy().view(uv), ext, perm), "execute_host")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_long_single_digit_output_runs(eb):
+    """Output runs longer than 16 x 32 lane slots (one output digit): the store
+    phase walks them in chunks; forced tile [n0, 2048] on [n0, 4096, 24] (1 0 2)."""
+    for n0 in (2, 3, 5):
+        ext, perm = [n0, 4096, 24], [1, 0, 2]
+        for variant in (1, 2):
+            got, exp, info = _run(ext, perm, eb, 300 + n0, plan_kwargs={
+                "in_dim": 1, "in_block": 2048, "out_dim": 0, "out_block": 2048,
+                "variant": variant})
+            assert info["out_run"] == 2048
+            _assert_equal(got, exp, f"long runs n0={n0} {info['kernel']}")
