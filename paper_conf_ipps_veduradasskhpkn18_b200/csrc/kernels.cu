@@ -362,9 +362,11 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
           const uint32_t cb = (uint32_t)jb * jstrideW;
 #pragma unroll
           for (int i = 0; i < NJ; i++) {
-            if (i < kB)
-              stcs_p(dst + jb + (i << lgB), lds_T<T>(src + cb + jc[i]),
-                     rok && jb + xB0 + (i << lgB) < lim);
+            if (i < kB) {
+              const bool ok = rok && jb + xB0 + (i << lgB) < lim;
+              // predicated-off lanes read a valid address (no OOB smem access)
+              stcs_p(dst + jb + (i << lgB), lds_T<T>(src + (ok ? cb + jc[i] : 0u)), ok);
+            }
           }
         }
       } else {
