@@ -831,7 +831,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) break;
     }
   }
-  if (ntop == 0) return force_schema == TTLG_SCHEMA_AUTO ? TTLG_ERR_INTERNAL : TTLG_ERR_UNSUPPORTED;
+  if (ntop == 0) {
+    const bool forced = hints && (hints->schema != TTLG_SCHEMA_AUTO || hints->in_dim >= 0 ||
+                                  hints->in_block > 0 || hints->out_dim >= 0 ||
+                                  hints->out_block > 0 || hints->variant || hints->threads);
+    return forced ? TTLG_ERR_UNSUPPORTED : TTLG_ERR_INTERNAL;
+  }
 
   // refine the short list: exact blocks, conflicts and padding (cached per geometry)
   if (!sink) {

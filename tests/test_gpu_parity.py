@@ -288,11 +288,12 @@ def test_execute_host_pipeline(ext, perm, eb):
 def test_long_single_digit_output_runs(eb):
     """Output runs longer than 16 x 32 lane slots (one output digit): the store
     phase walks them in chunks; forced tile [n0, 2048] on [n0, 4096, 24] (1 0 2)."""
+    blk = 2048 if eb == 4 else 1024   # tile <= 64 KB
     for n0 in (2, 3, 5):
         ext, perm = [n0, 4096, 24], [1, 0, 2]
         for variant in (1, 2):
             got, exp, info = _run(ext, perm, eb, 300 + n0, plan_kwargs={
-                "in_dim": 1, "in_block": 2048, "out_dim": 0, "out_block": 2048,
+                "in_dim": 1, "in_block": blk, "out_dim": 0, "out_block": blk,
                 "variant": variant})
-            assert info["out_run"] == 2048
+            assert info["out_run"] == blk
             _assert_equal(got, exp, f"long runs n0={n0} {info['kernel']}")
