@@ -356,6 +356,13 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
       T *dst = Bb + t.x;
       const uint32_t src = sbuf + t.y * W;
       if constexpr (NJ > 0) {
+        if (LB <= (NJ << lgB)) {
+#pragma unroll
+          for (int i = 0; i < NJ; i++) {
+            if (i < kB)
+              stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
+          }
+        } else
         // runs longer than NJ lane-slots (single output digit only, so the
         // column offset is linear in j) take several uniform chunks
         for (int jb = 0; jb < lim; jb += NJ << lgB) {
