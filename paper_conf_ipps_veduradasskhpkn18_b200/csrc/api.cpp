@@ -184,17 +184,32 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
                                 void *A_dev, void *B_dev, cudaStream_t s) {
   const int esize = p->dt == TTLG_F64 ? 8 : 4;
   const int d = p->rank;
-  const int q = p->perm[d - 1];
-  int64_t inner = 1, outer = 1, N = 1;
+  int64_t N = 1, m[TTLG_MAXD];
   for (int k = 0; k < d; k++) N *= p->ext[k];
-  for (int k = 0; k < q; k++) inner *= p->ext[k];
-  for (int k = q + 1; k < d; k++) outer *= p->ext[k];
-  const int64_t nq = p->ext[q];
+  for (int i = 0; i < d; i++) m[i] = p->ext[p->perm[i]];
   const int64_t nbytes = N * esize;
-  int64_t C = std::min<int64_t>({nq, (int64_t)kMaxChunks, nbytes / (16ll << 20)});
   if (p->device < 0) return TTLG_ERR_DEVICE;
-  HostPipe *hp = C >= 2 ? host_pipe(p->device) : nullptr;
-  if (!hp) {  // small or unsplittable: one stream, in order
+  // Two ways to split into chunks; each keeps one side contiguous and makes
+  // the other a 2-D strided copy.  Mode B splits B's outermost dim (input dim
+  // q = perm[d-1]): H2D rows of inner_q*c elements.  Mode A splits A's
+  // outermost dim (d-1, output position k): D2H rows of inner_B*c elements.
+  // Pick the mode with the wider rows (PCIe DMA of narrow rows is slow).
+  const int q = p->perm[d - 1];
+  int kpos = 0;
+  while (p->perm[kpos] != d - 1) kpos++;
+  int64_t inner_q = 1, inner_b = 1;
+  for (int k = 0; k < q; k++) inner_q *= p->ext[k];
+  for (int i = 0; i < kpos; i++) inner_b *= m[i];
+  const int64_t nq = p->ext[q], na = p->ext[d - 1];
+  const int64_t want = std::min<int64_t>((int64_t)kMaxChunks, nbytes / (16ll << 20));
+  const int64_t CB = std::min<int64_t>(nq, want), CA = std::min<int64_t>(na, want);
+  const double wB = CB >= 2 ? (double)inner_q * (nq / CB) * esize : 0.0;
+  const double wA = CA >= 2 ? (double)inner_b * (na / CA) * esize : 0.0;
+  const bool modeA = wA > wB;
+  const int64_t C = modeA ? CA : CB;
+  const double width_min = modeA ? wA : wB;
+  HostPipe *hp = (C >= 2 && width_min >= 2048.0) ? host_pipe(p->device) : nullptr;
+  if (!hp) {  // small, unsplittable or too narrow: one stream, in order
     if (cudaMemcpyAsync(A_dev, A_host, (size_t)nbytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
       return TTLG_ERR_CUDA;
     ttlg_status st = execute(p, A_dev, B_dev, s);
@@ -204,16 +219,17 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
     return TTLG_OK;
   }
   std::lock_guard<std::mutex> g(hp->mu);
-  const int64_t M = N / nq;  // B elements per index of its outermost dim
+  const int cd = modeA ? d - 1 : q;  // the split input dim
+  const int64_t nc = p->ext[cd];
   // at most two distinct chunk extents -> two sub-plans
-  const int64_t base = nq / C, rem = nq % C;
+  const int64_t base = nc / C, rem = nc % C;
   ttlg_plan_s sub[2];
-  int64_t subq[2] = {base, base + 1};
+  const int64_t subc[2] = {base, base + 1};
   for (int v = 0; v < 2; v++) {
-    if (subq[v] == 0 || (v == 1 && rem == 0)) continue;
+    if (subc[v] == 0 || (v == 1 && rem == 0)) continue;
     int64_t e[TTLG_MAXD];
     for (int k = 0; k < d; k++) e[k] = p->ext[k];
-    e[q] = subq[v];
+    e[cd] = subc[v];
     ttlg_status st = plan_into(&sub[v], (ttlg_dtype)p->dt, d, e, p->perm,
                                p->has_hints ? &p->hints : nullptr);
     if (st != TTLG_OK) return st;
@@ -222,26 +238,40 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
   cudaStreamWaitEvent(hp->h2d, hp->start, 0);
   cudaStreamWaitEvent(hp->comp, hp->start, 0);
   cudaStreamWaitEvent(hp->d2h, hp->start, 0);
-  int64_t q0 = 0;
+  const int64_t per = N / nc;  // elements per index of the split dim
+  unsigned char *Ah = (unsigned char *)A_host, *Bh = (unsigned char *)B_host;
+  int64_t c0 = 0;
   for (int64_t k = 0; k < C; k++) {
     const int v = k < rem ? 1 : 0;
-    const int64_t cq = subq[v];
-    const size_t width = (size_t)(inner * cq * esize), spitch = (size_t)(inner * nq * esize);
-    unsigned char *a_slab = (unsigned char *)A_dev + q0 * inner * outer * esize;
-    unsigned char *b_chunk = (unsigned char *)B_dev + q0 * M * esize;
-    if (cudaMemcpy2DAsync(a_slab, width, (const unsigned char *)A_host + q0 * inner * esize, spitch,
-                          width, (size_t)outer, cudaMemcpyHostToDevice, hp->h2d) != cudaSuccess)
-      return TTLG_ERR_CUDA;
+    const int64_t cc = subc[v];
+    unsigned char *a_slab = (unsigned char *)A_dev + c0 * per * esize;
+    unsigned char *b_chunk = (unsigned char *)B_dev + c0 * per * esize;
+    cudaError_t e;
+    if (modeA) {  // contiguous A slab
+      e = cudaMemcpyAsync(a_slab, Ah + c0 * per * esize, (size_t)(cc * per * esize),
+                          cudaMemcpyHostToDevice, hp->h2d);
+    } else {      // strided A slab: rows of inner_q*cc elements
+      const size_t w = (size_t)(inner_q * cc * esize);
+      e = cudaMemcpy2DAsync(a_slab, w, Ah + c0 * inner_q * esize, (size_t)(inner_q * nq * esize), w,
+                            (size_t)(N / (inner_q * nq)), cudaMemcpyHostToDevice, hp->h2d);
+    }
+    if (e != cudaSuccess) return TTLG_ERR_CUDA;
     cudaEventRecord(hp->evA[k], hp->h2d);
     cudaStreamWaitEvent(hp->comp, hp->evA[k], 0);
     ttlg_status st = execute(&sub[v], a_slab, b_chunk, hp->comp);
     if (st != TTLG_OK) return st;
     cudaEventRecord(hp->evB[k], hp->comp);
     cudaStreamWaitEvent(hp->d2h, hp->evB[k], 0);
-    if (cudaMemcpyAsync((unsigned char *)B_host + q0 * M * esize, b_chunk, (size_t)(cq * M * esize),
-                        cudaMemcpyDeviceToHost, hp->d2h) != cudaSuccess)
-      return TTLG_ERR_CUDA;
-    q0 += cq;
+    if (modeA) {  // the chunk's B rows are strided in B: rows of inner_b*cc elements
+      const size_t w = (size_t)(inner_b * cc * esize);
+      e = cudaMemcpy2DAsync(Bh + c0 * inner_b * esize, (size_t)(inner_b * na * esize), b_chunk, w, w,
+                            (size_t)(N / (inner_b * na)), cudaMemcpyDeviceToHost, hp->d2h);
+    } else {      // contiguous range of B
+      e = cudaMemcpyAsync(Bh + c0 * per * esize, b_chunk, (size_t)(cc * per * esize),
+                          cudaMemcpyDeviceToHost, hp->d2h);
+    }
+    if (e != cudaSuccess) return TTLG_ERR_CUDA;
+    c0 += cc;
   }
   if (cudaEventRecord(hp->done, hp->d2h) != cudaSuccess) return TTLG_ERR_CUDA;
   if (cudaStreamWaitEvent(s, hp->done, 0) != cudaSuccess) return TTLG_ERR_CUDA;
