@@ -363,7 +363,7 @@ def main():
             "cpu_baseline": cpu,
         }
         if os.environ.get("TTLG_BENCH_CASES"):
-            line["cases"] = [{"case": c.label(), "schema": inf["schema"],
+            line["cases"] = [{"case": c.label(), "schema": inf["schema"], "kernel": kname(inf),
                               "gbs": c.alg_bytes / (m * 1e-3) / 1e9,
                               "pred_gbs": c.alg_bytes / inf["predicted_seconds"] / 1e9}
                              for c, inf, m in zip(cases, infos, med)]
