@@ -159,6 +159,15 @@ ttlg_status ttlg_predict_time(ttlg_dtype dt, int rank, const int64_t *extents,
 
 ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info);
 
+/* Measure-mode refinement (the cuTT "measure" idea, PAPER.md L130-136,
+ * L1575-1579): executes up to max_candidates (<= 16) of the model's
+ * ranked short list on A -> B (B is overwritten with the correct result; A is
+ * read only), times each with CUDA events on `stream` (synchronises the
+ * stream), and replaces *plan by the fastest (the old plan is destroyed).
+ * best_seconds (may be NULL) receives the measured time. */
+ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stream,
+                           int32_t max_candidates, double *best_seconds);
+
 /* Every candidate the planner scores for this problem (Alg. 3's enumeration),
  * with its model features and predicted time -- for calibration (§V) and
  * measure-mode / model-regret studies.  Writes up to max_out entries to out and

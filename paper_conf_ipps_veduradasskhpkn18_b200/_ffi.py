@@ -23,7 +23,7 @@ STATUS = {0: "TTLG_OK", 1: "TTLG_ERR_INVALID_VALUE", 2: "TTLG_ERR_ALIASING",
 EXPORTS = ["ttlg_plan", "ttlg_plan_ex", "ttlg_plan_hints_init", "ttlg_execute",
            "ttlg_plan_destroy", "ttlg_transpose", "ttlg_execute_host", "ttlg_predict_time",
            "ttlg_plan_describe", "ttlg_status_string", "ttlg_schema_name", "ttlg_version",
-           "ttlg_model_source", "ttlg_plan_candidates"]
+           "ttlg_model_source", "ttlg_plan_candidates", "ttlg_plan_tune"]
 
 
 class TtlgError(RuntimeError):
@@ -103,6 +103,8 @@ def _load():
         "ttlg_schema_name": ([ctypes.c_int], ctypes.c_char_p),
         "ttlg_version": ([], ctypes.c_int),
         "ttlg_model_source": ([], ctypes.c_char_p),
+        "ttlg_plan_tune": ([ctypes.POINTER(P), P, P, P, ctypes.c_int32,
+                            ctypes.POINTER(ctypes.c_double)], ctypes.c_int),
         "ttlg_plan_candidates": ([ctypes.c_int, ctypes.c_int, i64p, i32p, ctypes.POINTER(PlanHints),
                                   ctypes.POINTER(PlanInfo), ctypes.c_int32,
                                   ctypes.POINTER(ctypes.c_int32)], ctypes.c_int),

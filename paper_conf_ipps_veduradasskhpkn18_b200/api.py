@@ -91,6 +91,15 @@ class Plan:
                                     ctypes.c_void_p(A_dev), ctypes.c_void_p(B_dev),
                                     ctypes.c_void_p(stream)), "ttlg_execute_host")
 
+    def tune(self, A_ptr: int, B_ptr: int, stream: int = 0, max_candidates: int = 8) -> float:
+        """Measure-mode refinement (ttlg_plan_tune): time the model's short list on
+        these buffers and keep the fastest; returns its measured seconds."""
+        out = ctypes.c_double()
+        check(lib.ttlg_plan_tune(ctypes.byref(self._h), ctypes.c_void_p(A_ptr),
+                                 ctypes.c_void_p(B_ptr), ctypes.c_void_p(stream),
+                                 max_candidates, ctypes.byref(out)), "ttlg_plan_tune")
+        return out.value
+
     def destroy(self):
         if self._h:
             lib.ttlg_plan_destroy(self._h)

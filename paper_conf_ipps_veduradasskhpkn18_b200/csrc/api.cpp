@@ -9,6 +9,7 @@
 #include <new>
 
 #include "model_coeffs.h"
+#include "model_gbt.h"
 #include "ttlg_internal.h"
 
 namespace ttlg {
@@ -350,11 +351,72 @@ ttlg_status ttlg_plan_candidates(ttlg_dtype dt, int rank, const int64_t *extents
                                  ttlg_plan_info *out, int32_t max_out, int32_t *n_out) {
   if (!out || !n_out || max_out < 0) return TTLG_ERR_INVALID_VALUE;
   ttlg_plan_s p;
-  CandidateSink sink{out, max_out, 0};
+  CandidateSink sink{out, max_out, 0, false};
   ttlg_status st = make_plan(&p, dt, rank, extents, perm, hints,
                              device_profile(current_device()), &sink);
   *n_out = sink.n;
   return st;
+}
+
+ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stream,
+                           int32_t max_candidates, double *best_seconds) {
+  if (!plan || !*plan || !A || !B || max_candidates < 1) return TTLG_ERR_INVALID_VALUE;
+  ttlg_plan_s *p = *plan;
+  if (p->device < 0) return TTLG_ERR_DEVICE;
+  // the model's ranked short list
+  ttlg_plan_info list[kGbtTopK];
+  CandidateSink sink{list, std::min<int>(max_candidates, kGbtTopK), 0, true};
+  ttlg_plan_s scratch;
+  ttlg_status st = make_plan(&scratch, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm,
+                             p->has_hints ? &p->hints : nullptr, device_profile(p->device), &sink);
+  if (st != TTLG_OK) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  cudaEvent_t e0, e1;
+  if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess)
+    return TTLG_ERR_CUDA;
+  ttlg_plan_s *best = nullptr;
+  float best_ms = 1e30f;
+  for (int i = 0; i < sink.n; i++) {
+    const ttlg_plan_info &ci = list[i];
+    ttlg_plan_hints h;
+    ttlg_plan_hints_init(&h);
+    h.schema = ci.schema == TTLG_SCHEMA_COPY ? TTLG_SCHEMA_FML : ci.schema;
+    h.in_dim = ci.in_dim;
+    h.in_block = ci.tile_extents[ci.in_dim];
+    h.out_dim = ci.out_dim;
+    h.out_block = ci.tile_extents[ci.fused_perm[ci.out_dim]];
+    h.threads = ci.threads;
+    h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : 0);
+    ttlg_plan_s *q = new (std::nothrow) ttlg_plan_s;
+    if (!q) break;
+    if (plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h) != TTLG_OK) {
+      delete q;
+      continue;
+    }
+    float ms = 1e30f;
+    bool ok = execute(q, A, B, stream) == TTLG_OK;  // warm-up
+    for (int r = 0; ok && r < 3; r++) {
+      ok = cudaEventRecord(e0, s) == cudaSuccess && execute(q, A, B, stream) == TTLG_OK &&
+           cudaEventRecord(e1, s) == cudaSuccess && cudaEventSynchronize(e1) == cudaSuccess;
+      float t = 0;
+      if (ok && cudaEventElapsedTime(&t, e0, e1) == cudaSuccess) ms = std::min(ms, t);
+    }
+    if (ok && ms < best_ms) {
+      delete best;
+      best = q;
+      best_ms = ms;
+    } else {
+      delete q;
+    }
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  if (!best) return TTLG_ERR_INTERNAL;
+  best->info.predicted_seconds = best_ms * 1e-3;  // measured
+  delete *plan;
+  *plan = best;
+  if (best_seconds) *best_seconds = best_ms * 1e-3;
+  return TTLG_OK;
 }
 
 ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info) {

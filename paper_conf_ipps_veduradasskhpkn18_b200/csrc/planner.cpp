@@ -597,6 +597,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int8_t delta[TTLG_MAXD];  // input-run padding chosen by the conflict search
   };
   constexpr int kShort = 2 * kGbtTopK;
+  // sink modes: full candidate listing (calibration) or the ranked short list
+  // (measure-mode tuning, ttlg_plan_tune)
+  const bool listing = sink && !sink->shortlist;
   Entry pool[kShort];
   int order[kShort];  // pool slots sorted by the linear prediction
   int ntop = 0, ncand = 0;
@@ -749,7 +752,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int delta[TTLG_MAXD] = {0};
     double cl = 1.0, cs = 1.0;
     TileParams K0;
-    if (sink) {  // candidate listing: exact features for every candidate
+    if (listing) {  // candidate listing: exact features for every candidate
       if (!build_exact(T, group, K0, delta, cl, cs, S)) return;
     }
     int kinds[2], nk = 0;
@@ -767,7 +770,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         if (!make_mi(mi, tpc, kind, schema, threads, S, cl, cs)) continue;
         const double tm = predict_seconds(mi, dev);
         ncand++;
-        if (sink && sink->n < sink->max) {
+        if (listing && sink->n < sink->max) {
           TileParams K = K0;
           if (kind == KK_PIPE) {
             K.off_data2 = K.off_data + S.buf_bytes;
@@ -839,7 +842,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   }
 
   // refine the short list: exact blocks, conflicts and padding (cached per geometry)
-  if (!sink) {
+  if (!listing) {
     struct Done {
       int a, b, group;
       int64_t ta, tb;
@@ -892,6 +895,26 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (t < win_t) {
       win_t = t;
       win = order[i];
+    }
+  }
+  if (sink && sink->shortlist) {
+    // the ranked short list (tree prediction in predicted_seconds)
+    for (int i = 0; i < std::min(ntop, kGbtTopK) && sink->n < sink->max; i++) {
+      const Entry &e = pool[order[i]];
+      if (e.lin >= 1e299) continue;
+      int delta[TTLG_MAXD];
+      bool padded = false;
+      for (int k = 0; k < TTLG_MAXD; k++) {
+        delta[k] = e.delta[k];
+        padded |= delta[k] != 0;
+      }
+      TileParams K;
+      if (!build_params(P, e.T, e.group, e.mi.threads, e.kind == KK_PIPE ? 2 : 1, K,
+                        padded ? delta : nullptr))
+        continue;
+      K.tpc = e.tpc;
+      fill_info(sink->out[sink->n++], dt, rank, P, e.T, K, e.mi, e.schema, e.kind,
+                predict_ranked_seconds(e.mi, dev), ncand);
     }
   }
   const Entry &B = pool[win];

@@ -151,6 +151,7 @@ struct CandidateSink {
   ttlg_plan_info *out;
   int max;
   int n;
+  bool shortlist;  // false: every scored candidate; true: the ranked short list
 };
 constexpr int kModelFeatureCount = 10;
 // planner.cpp

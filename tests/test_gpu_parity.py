@@ -299,3 +299,18 @@ def test_long_single_digit_output_runs(eb):
                 "variant": variant})
             assert info["out_run"] == blk
             _assert_equal(got, exp, f"long runs n0={n0} {info['kernel']}")
+
+
+def test_plan_tune_measure_mode():
+    """ttlg_plan_tune (N2 measure mode) keeps a correct plan and reports time."""
+    for c in configs.config1()[::6] + [configs.scaled(configs.config2()[20], 1 << 20)]:
+        n = c.n_elems
+        A = gen_tensor_torch(case_seed(c.case_id), n, c.elem_bytes, device=DEV)
+        B = torch.empty_like(A)
+        p = ttlg.plan(_dt(c.elem_bytes), c.extents, c.perm)
+        t = p.tune(A.data_ptr(), B.data_ptr(), torch.cuda.current_stream().cuda_stream, 6)
+        assert t > 0
+        B.zero_()
+        p.execute(A.data_ptr(), B.data_ptr(), torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        _assert_equal(_bits(B), oracle.transpose(_bits(A), c.extents, c.perm), "tuned plan")
