@@ -57,6 +57,8 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--stride", type=int, default=1)
     ap.add_argument("--threads", default="", help="comma list of block sizes to try per candidate")
+    ap.add_argument("--top", action="store_true",
+                    help="measure the linear screen's best candidates instead of a spread")
     args = ap.parse_args()
 
     import torch
@@ -76,10 +78,14 @@ def main():
         cands = ttlg.plan_candidates(dt, c.extents, c.perm)
         auto = ttlg.plan(dt, c.extents, c.perm).describe()
         if len(cands) > args.max_cand:
-            # keep the model's best few plus an even spread over the rest
             cands.sort(key=lambda d: d["predicted_seconds"])
-            step = len(cands) / args.max_cand
-            cands = [cands[int(i * step)] for i in range(args.max_cand)]
+            if args.top:
+                # the linear screen's best: the region the ranking stage must order
+                cands = cands[:args.max_cand]
+            else:
+                # an even spread over the whole predicted range
+                step = len(cands) / args.max_cand
+                cands = [cands[int(i * step)] for i in range(args.max_cand)]
         A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
         B = torch.empty_like(A)
         thr = [int(x) for x in args.threads.split(",") if x] or [0]
