@@ -27,6 +27,7 @@ def main():
     ap.add_argument("--reps", type=int, default=10)
     ap.add_argument("--single-k", type=int, default=50)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--check", action="store_true", help="sampled parity vs the oracle")
     args = ap.parse_args()
 
     import torch
@@ -65,13 +66,29 @@ def main():
             p = ttlg.plan(dt, c.extents, c.perm)
             info = p.describe()
             t = timed(lambda: p.execute(A.data_ptr(), B.data_ptr(), st.cuda_stream), args.reps)
+            check = None
+            if args.check:
+                # sampled parity against the oracle's definition (lin_B -> lin_A)
+                import numpy as np
+                import oracle
+                from synth import gen_at_np
+                rng = np.random.default_rng(c.case_id)
+                linB = np.unique(np.concatenate([rng.integers(0, c.n_elems, 4096),
+                                                 [0, c.n_elems - 1]]))
+                iv = torch.int64 if c.elem_bytes == 8 else torch.int32
+                got = B.view(iv)[torch.from_numpy(linB).to(dev)].cpu().numpy()
+                got = got.view(np.uint64 if c.elem_bytes == 8 else np.uint32)
+                exp = gen_at_np(case_seed(c.case_id),
+                                oracle.source_index(c.extents, c.perm, linB), c.elem_bytes)
+                check = bool(np.array_equal(got, exp))
             td = timed(lambda: B.copy_(A), args.reps)
             rec = {"group": g, "case": c.label(), "schema": info["schema"], "kernel": info["kernel"],
                    "bytes": c.alg_bytes, "ms": t * 1e3, "gbs": c.alg_bytes / t / 1e9,
                    "d2d_gbs": c.alg_bytes / td / 1e9, "frac_d2d": td / t, "frac_peak":
                    c.alg_bytes / t / 1e9 / peak, "pred_ms": info["predicted_seconds"] * 1e3,
                    "model_err": abs(info["predicted_seconds"] - t) / t,
-                   "fused_rank": info["fused_rank"], "tile": info["tile_extents"]}
+                   "fused_rank": info["fused_rank"], "tile": info["tile_extents"],
+                   "parity_sampled": check}
             if g == "c3":
                 K = args.single_k
                 ext, perm = list(c.extents), list(c.perm)
