@@ -32,6 +32,7 @@
 #include <cuda_runtime.h>
 
 #include <mutex>
+#include <type_traits>
 
 #include "ttlg_internal.h"
 
@@ -113,8 +114,27 @@ __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
 }
 
+// p + i (i unsigned 32-bit, scaled by sizeof(T)) as ONE wide multiply-add
+// (IMAD.WIDE.U32) instead of a 64-bit add + shift chain
+template <typename T>
+__device__ __forceinline__ T *wadd(T *p, uint32_t i) {
+  T *r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(i), "n"((int)sizeof(T)), "l"(p));
+  return r;
+}
+template <typename T>
+__device__ __forceinline__ const T *wadd(const T *p, uint32_t i) {
+  const T *r;
+  asm("mad.wide.u32 %0, %1, %2, %3;" : "=l"(r) : "r"(i), "n"((int)sizeof(T)), "l"(p));
+  return r;
+}
+
 __device__ __forceinline__ uint32_t fdiv(uint32_t n, const FastDiv &f) {
   return __umulhi(n, f.mul) >> f.shr;  // grid divisors are always >= 2
+}
+// any divisor >= 1 (make_fastdiv(1) has mul = 0)
+__device__ __forceinline__ uint32_t fdiv1(uint32_t n, const FastDiv &f) {
+  return f.div == 1 ? n : fdiv(n, f);
 }
 
 struct TileCtx {
@@ -151,7 +171,9 @@ __device__ __forceinline__ TileCtx decode_tile(const TileParams &P, uint32_t til
 // part and a per-column part): decode row index i over the row digits.
 // Digit extents are >= 2, so the multiply-shift division applies.
 __device__ __forceinline__ void build_rows(int R, int nr, const FastDiv *ext, const int32_t *sG,
-                                           const int32_t *sS, int blk, int2 *tab, int *dig) {
+                                           const int32_t *sS, int blk, int2 *tab, int *dig,
+                                           int sw = 1) {
+#pragma unroll 1
   for (int i = threadIdx.x; i < R; i += blockDim.x) {
     int rem = i, g = 0, s = 0, dg = 0;
     for (int k = 0; k < nr; k++) {
@@ -162,7 +184,7 @@ __device__ __forceinline__ void build_rows(int R, int nr, const FastDiv *ext, co
       s += c * sS[k];
       if (k == blk) dg = c;
     }
-    tab[i] = make_int2(g, s);
+    tab[i] = make_int2(g, s * sw);  // (global elements, shared bytes when sw = W)
     dig[i] = dg;
   }
 }
@@ -182,7 +204,7 @@ __global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TilePara
   __syncthreads();
 
   const int NT = blockDim.x, tid = threadIdx.x;
-  const int r0 = tid / P.LB, j0 = tid % P.LB;
+  const int r0 = (int)fdiv1(tid, P.fd_LB), j0 = tid - r0 * P.LB;
   for (int it = 0; it < P.tpc; it++) {
     const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
     if (tile >= P.num_tiles) break;
@@ -252,15 +274,27 @@ __device__ __forceinline__ uint4 lds_T<uint4>(uint32_t a) {
 }
 
 // k_pipe template parameters:
-//   GA32 / GB32: the A-row / B-row lane group is a whole warp (run >= 32), so
-//                lane offsets along a row are compile-time immediates;
-//   NJ > 0:      every lane owns at most NJ output-run positions of a B-row
-//                (LB <= NJ * G_B) and keeps their shared-memory column offsets
-//                in registers; NJ = 0: column offsets read from the table.
-// Loop trip counts are warp-uniform and the bodies predicated, so no
-// divergence/reconvergence bookkeeping is generated in the hot loops.
-template <int W, int NJ, bool GA32, bool GB32, bool PERSIST, bool XT>
-__global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams P,
+//   XT:      the input run is padded in shared memory (icol offset table);
+//   PERSIST: persistent grid with a double-buffered cp.async ring, else one
+//            tile (or tpc consecutive tiles) per CTA, single buffer ("k_tile");
+//   SM2:     store mapping for output runs longer than the block (LB > NT):
+//            every thread owns columns tid + m*NT of each B-row in turn.
+//            Otherwise (LB <= NT) thread t owns ONE output-run position
+//            j = t mod LB for the whole tile -- its shared-memory column offset
+//            lives in a register -- and walks the B-rows t / LB + k*(NT/LB).
+// The load phase is a flat walk over the tile's V elements (element e = tid +
+// k*NT -> A-row e / LA, run position e mod LA, stepped incrementally), so no
+// lane idles whatever LA is; per element it costs one row-table broadcast
+// read, one predicated cp.async and the index step.  The tile's base offsets
+// are decoded once per tile by one thread (the paper's decode/compute_base,
+// Alg. 2 lines 6-7) into a shared-memory slot, a tile ahead of its use.
+struct __align__(16) CtxS {
+  long long bA, bB;
+  int limA, limB, pad0, pad1;
+};
+
+template <int W, bool XT, bool PERSIST, bool SM2>
+__global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const __grid_constant__ TileParams P,
                                               const void *__restrict__ Av,
                                               void *__restrict__ Bv) {
   using T = typename Vec<W>::T;
@@ -268,16 +302,40 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
   const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
   const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
   const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_icol = s0 + P.off_icol;
   const uint32_t s_buf0 = s0 + P.off_data, s_buf1 = s0 + P.off_data2;
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
+  const int tid = threadIdx.x, NT = blockDim.x;
+  const bool decoder = tid == NT - 1;  // the last thread: idle in most table builds
+  const uint32_t first = PERSIST ? blockIdx.x : blockIdx.x * (uint32_t)P.tpc;
+  const uint32_t tstep = PERSIST ? gridDim.x : 1u;
+
+  auto put_ctx = [&](int slot, uint32_t tile) {
+    const TileCtx c = decode_tile(P, tile);
+    ctx[slot].bA = c.bA;
+    ctx[slot].bB = c.bB;
+    ctx[slot].limA = c.limA;
+    ctx[slot].limB = c.limB;
+  };
+  auto get_ctx = [&](int slot) {
+    TileCtx c;
+    c.bA = ctx[slot].bA;
+    c.bB = ctx[slot].bB;
+    c.limA = ctx[slot].limA;
+    c.limB = ctx[slot].limB;
+    return c;
+  };
+  if (decoder && first < P.num_tiles) put_ctx(0, first);
 
   build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
-             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB));
+             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB), W);
   build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
              reinterpret_cast<int2 *>(smem + P.off_tabB),
-             reinterpret_cast<int *>(smem + P.off_digA));
-  for (int j = threadIdx.x; j < P.LB; j += blockDim.x) {
+             reinterpret_cast<int *>(smem + P.off_digA), W);
+#pragma unroll 1
+  for (int j = tid; j < P.LB; j += NT) {
     int rem = j, s = 0;
     for (int k = 0; k < P.nj; k++) {
       const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
@@ -287,7 +345,8 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
     reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
   }
   if constexpr (XT) {
-    for (int x = threadIdx.x; x < P.LA; x += blockDim.x) {
+#pragma unroll 1
+    for (int x = tid; x < P.LA; x += NT) {
       int rem = x, s = 0;
       for (int k = 0; k < P.ni; k++) {
         const int cq = (int)fdiv((uint32_t)rem, P.i_div[k]);
@@ -297,128 +356,157 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
       reinterpret_cast<int *>(smem + P.off_icol)[x] = s * W;  // byte offset
     }
   }
-  const uint32_t s_icol = s0 + P.off_icol;
   __syncthreads();
 
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
-  const int lgA = GA32 ? 5 : P.lgA, lgB = GB32 ? 5 : P.lgB;
-  const int gA = 1 << lgA, gB = 1 << lgB;
-  const int xA0 = lane & (gA - 1), rA0 = warp * (32 >> lgA) + (lane >> lgA);
-  const int rAstep = nw * (32 >> lgA);
-  const int xB0 = lane & (gB - 1), rB0 = warp * (32 >> lgB) + (lane >> lgB);
-  const int rBstep = nw * (32 >> lgB);
-  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB;
-  const int kA = (LA + gA - 1) >> lgA;  // uniform per-row trip count (load)
-  const int kB = (LB + gB - 1) >> lgB;  // uniform per-row trip count (store)
-  const uint32_t jstrideW = (P.nj == 1 ? (uint32_t)P.j_sS[0] : 0u) * W;  // chunked long runs
-  int jc[NJ > 0 ? NJ : 1];
-  if constexpr (NJ > 0) {
-#pragma unroll
-    for (int i = 0; i < NJ; i++) {
-      const int j = xB0 + i * gB;
-      jc[i] = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-    }
+  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB, V = P.V;
+  // load walk: element e = tid + k*NT
+  const int rA0 = (int)fdiv1(tid, P.fd_LA), xA0 = tid - rA0 * LA;
+  const int nA = tid < V ? (int)fdiv1(V - 1 - tid, P.fd_NT) + 1 : 0;
+  const int drA = P.drA, dxA = P.dxA;
+  // store walk
+  int jB0, rB0, nB;
+  uint32_t jc0 = 0;
+  if constexpr (!SM2) {
+    rB0 = (int)fdiv1(tid, P.fd_LB);
+    jB0 = tid - rB0 * LB;
+    // threads past rsB*LB idle
+    nB = (rB0 < P.rsB && rB0 < RB) ? (int)fdiv1(RB - 1 - rB0, P.fd_rsB) + 1 : 0;
+    jc0 = lds_int(s_jcol + 4 * jB0);
+  } else {
+    jB0 = tid;
+    rB0 = 0;
+    nB = RB;
   }
 
-  // load phase of one tile: A-row r -> smem, cp.async, lanes stride the run
-  auto issue = [&](const TileCtx &c, uint32_t sbuf) {
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? LA : P.LAunit * c.limA;
-    const T *Ab = A + c.bA + xA0;
-    const uint32_t sb = sbuf + xA0 * W;
-    for (int r = rA0; r < RA; r += rAstep) {
+  // load phase of one tile: A-rows -> smem with predicated cp.async.  Row
+  // table entries hold (global element offset, shared byte offset).  FULL
+  // tiles (the common case) carry no bounds logic; when threads are a
+  // multiple of LA every thread keeps one run position for the whole tile.
+  auto issue_t = [&](auto full_c, const TileCtx &c, uint32_t sbuf) {
+    constexpr bool FULL = decltype(full_c)::value;
+    const int lim = FULL ? LA : P.LAunit * c.limA;
+    const T *Ab = A + c.bA;
+    int r = rA0, x = xA0;
+    if (!XT && dxA == 0) {
+      const T *Ax = Ab + x;
+      const uint32_t sx = sbuf + x * W;
+      const bool xok = FULL || x < lim;
+#pragma unroll 4
+      for (int k = 0; k < nA; k++) {
+        const int2 t = lds_int2(s_tabA + 8 * r);
+        if constexpr (FULL)
+          cp_async<W>(sx + t.y, wadd(Ax, (uint32_t)t.x));
+        else
+          cp_async_p<W>(sx + t.y, wadd(Ax, (uint32_t)t.x), xok && lds_int(s_digB + 4 * r) < c.limB);
+        r += drA;
+      }
+      return;
+    }
+#pragma unroll 4
+    for (int k = 0; k < nA; k++) {
       const int2 t = lds_int2(s_tabA + 8 * r);
-      const bool rok = full || lds_int(s_digB + 4 * r) < c.limB;
-      const T *src = Ab + t.x;
-      if constexpr (XT) {
-        // padded input run: smem offset of run position x from the icol table
-        const uint32_t rowS = sbuf + t.y * W;
-        for (int k = 0; k < kA; k++) {
-          const int x = xA0 + (k << lgA);
-          const int off = x < LA ? lds_int(s_icol + 4 * x) : 0;
-          cp_async_p<W>(rowS + off, src + (k << lgA), rok && x < lim);
-        }
-      } else {
-        const uint32_t dst = sb + t.y * W;
-        for (int k = 0; k < kA; k++)
-          cp_async_p<W>(dst + (k << lgA) * W, src + (k << lgA), rok && xA0 + (k << lgA) < lim);
+      uint32_t soff;
+      if constexpr (XT)
+        soff = t.y + lds_int(s_icol + 4 * x);
+      else
+        soff = t.y + x * W;
+      if constexpr (FULL)
+        cp_async<W>(sbuf + soff, wadd(Ab, (uint32_t)(t.x + x)));
+      else
+        cp_async_p<W>(sbuf + soff, wadd(Ab, (uint32_t)(t.x + x)),
+                      x < lim && lds_int(s_digB + 4 * r) < c.limB);
+      x += dxA;
+      r += drA;
+      if (x >= LA) {
+        x -= LA;
+        r++;
       }
     }
   };
-  // store phase of one tile: B-row r <- smem through the column offsets
-  auto drain = [&](const TileCtx &c, uint32_t sbuf) {
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    const int lim = full ? LB : P.LBunit * c.limB;
-    T *Bb = B + c.bB + xB0;
-    for (int r = rB0; r < RB; r += rBstep) {
-      const int2 t = lds_int2(s_tabB + 8 * r);
-      const bool rok = full || lds_int(s_digA + 4 * r) < c.limA;
-      T *dst = Bb + t.x;
-      const uint32_t src = sbuf + t.y * W;
-      if constexpr (NJ > 0) {
-        if (LB <= (NJ << lgB)) {
-#pragma unroll
-          for (int i = 0; i < NJ; i++) {
-            if (i < kB)
-              stcs_p(dst + (i << lgB), lds_T<T>(src + jc[i]), rok && xB0 + (i << lgB) < lim);
-          }
-        } else
-        // runs longer than NJ lane-slots (single output digit only, so the
-        // column offset is linear in j) take several uniform chunks
-        for (int jb = 0; jb < lim; jb += NJ << lgB) {
-          const uint32_t cb = (uint32_t)jb * jstrideW;
-#pragma unroll
-          for (int i = 0; i < NJ; i++) {
-            if (i < kB) {
-              const bool ok = rok && jb + xB0 + (i << lgB) < lim;
-              // predicated-off lanes read a valid address (no OOB smem access)
-              stcs_p(dst + jb + (i << lgB), lds_T<T>(src + (ok ? cb + jc[i] : 0u)), ok);
-            }
-          }
-        }
-      } else {
+  auto issue = [&](const TileCtx &c, uint32_t sbuf) {
+    if ((c.limA == P.blkA_t) && (c.limB == P.blkB_t))
+      issue_t(std::true_type{}, c, sbuf);
+    else
+      issue_t(std::false_type{}, c, sbuf);
+  };
+  // store phase of one tile: B-rows <- smem through the column offsets
+  auto drain_t = [&](auto full_c, const TileCtx &c, uint32_t sbuf) {
+    constexpr bool FULL = decltype(full_c)::value;
+    const int lim = FULL ? LB : P.LBunit * c.limB;
+    T *Bb = B + c.bB;
+    if constexpr (!SM2) {
+      T *Bj = Bb + jB0;
+      const uint32_t sj = sbuf + jc0;
+      const bool jok = FULL || jB0 < lim;
+      const int rs = P.rsB;
+      int r = rB0;
 #pragma unroll 4
-        for (int i = 0; i < kB; i++) {
-          const int j = xB0 + (i << lgB);
-          const int off = j < LB ? lds_int(s_jcol + 4 * j) : 0;
-          stcs_p(dst + (i << lgB), lds_T<T>(src + off), rok && j < lim);
+      for (int k = 0; k < nB; k++) {
+        const int2 t = lds_int2(s_tabB + 8 * r);
+        const T v = lds_T<T>(sj + t.y);
+        if constexpr (FULL)
+          st_stream<true>(wadd(Bj, (uint32_t)t.x), v);
+        else
+          stcs_p(wadd(Bj, (uint32_t)t.x), v, jok && lds_int(s_digA + 4 * r) < c.limA);
+        r += rs;
+      }
+    } else {
+      for (int r = 0; r < RB; r++) {
+        const int2 t = lds_int2(s_tabB + 8 * r);
+        const bool rok = FULL || lds_int(s_digA + 4 * r) < c.limA;
+        const uint32_t sr = sbuf + t.y;
+        T *Br = wadd(Bb, (uint32_t)t.x);
+#pragma unroll 2
+        for (int j = jB0; j < LB; j += NT) {
+          const int jc = lds_int(s_jcol + 4 * j);
+          stcs_p(Br + j, lds_T<T>(sr + jc), rok && (FULL || j < lim));
         }
       }
     }
+  };
+  auto drain = [&](const TileCtx &c, uint32_t sbuf) {
+    if ((c.limA == P.blkA_t) && (c.limB == P.blkB_t))
+      drain_t(std::true_type{}, c, sbuf);
+    else
+      drain_t(std::false_type{}, c, sbuf);
   };
 
   if constexpr (!PERSIST) {
     // k_tile: one tile (or tpc consecutive tiles) per CTA, single buffer, many
     // CTAs per SM -- the cp.async skeleton that reaches the D2D copy rate
-    // (tools/copybench.cu: 6.4-6.6 TB/s vs 5.4-5.8 TB/s persistent)
+    // (tools/copybench.cu)
     for (int it = 0; it < P.tpc; it++) {
-      const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
+      const uint32_t tile = first + it;
       if (tile >= P.num_tiles) break;
-      const TileCtx c = decode_tile(P, tile);
-      if (it > 0) __syncthreads();
+      if (it > 0) __syncthreads();  // buffer drained, ctx[it & 1] visible
+      const TileCtx c = get_ctx(it & 1);
       issue(c, s_buf0);
       cp_async_commit();
+      if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
       cp_async_wait<0>();
       __syncthreads();
       drain(c, s_buf0);
     }
   } else {
-    uint32_t tile = blockIdx.x;
-    TileCtx cur = decode_tile(P, tile < P.num_tiles ? tile : 0);
-    if (tile < P.num_tiles) issue(cur, s_buf0);
+    uint32_t tile = first;
+    if (tile >= P.num_tiles) return;
+    TileCtx cur = get_ctx(0);
+    issue(cur, s_buf0);
     cp_async_commit();
+    if (decoder && tile + tstep < P.num_tiles) put_ctx(1, tile + tstep);
     for (int k = 0; tile < P.num_tiles; k++) {
-      const uint32_t next = tile + gridDim.x;
+      __syncthreads();  // ctx[(k+1)&1] visible; buffer (k+1)&1 drained (iteration k-1)
+      const uint32_t next = tile + tstep;
       TileCtx nx = cur;
       if (next < P.num_tiles) {
-        nx = decode_tile(P, next);
+        nx = get_ctx((k + 1) & 1);
         issue(nx, (k & 1) ? s_buf0 : s_buf1);
       }
       cp_async_commit();
+      if (decoder && next + tstep < P.num_tiles) put_ctx(k & 1, next + tstep);
       cp_async_wait<1>();
       __syncthreads();
       drain(cur, (k & 1) ? s_buf1 : s_buf0);
-      __syncthreads();
       cur = nx;
       tile = next;
     }
@@ -428,51 +516,24 @@ __global__ void __launch_bounds__(512) k_pipe(const __grid_constant__ TileParams
 
 // ---------------------------------------------------------------------------
 // launch plumbing
-template <int W, bool GA32, bool PERSIST, bool XT>
-static const void *kernel_ptr_pipe(int nj, bool gb32) {
-  if (!gb32) return (const void *)k_pipe<W, 1, GA32, false, PERSIST, XT>;  // LB < 32: one slot
-  switch (nj) {
-    case 1: return (const void *)k_pipe<W, 1, GA32, true, PERSIST, XT>;
-    case 2: return (const void *)k_pipe<W, 2, GA32, true, PERSIST, XT>;
-    case 4: return (const void *)k_pipe<W, 4, GA32, true, PERSIST, XT>;
-    case 8: return (const void *)k_pipe<W, 8, GA32, true, PERSIST, XT>;
-  }
-  return (const void *)k_pipe<W, 16, GA32, true, PERSIST, XT>;  // LB <= 512 (planner cap)
-}
-
 template <int W, bool XT>
-static const void *kernel_ptr_x(int kind, int nj, bool ga32, bool gb32) {
+static const void *kernel_ptr_x(int kind, bool sm2) {
   if (kind == KK_PIPE)
-    return ga32 ? kernel_ptr_pipe<W, true, true, XT>(nj, gb32)
-                : kernel_ptr_pipe<W, false, true, XT>(nj, gb32);
-  return ga32 ? kernel_ptr_pipe<W, true, false, XT>(nj, gb32)
-              : kernel_ptr_pipe<W, false, false, XT>(nj, gb32);
+    return sm2 ? (const void *)k_pipe<W, XT, true, true> : (const void *)k_pipe<W, XT, true, false>;
+  return sm2 ? (const void *)k_pipe<W, XT, false, true> : (const void *)k_pipe<W, XT, false, false>;
 }
 
 template <int W>
-static const void *kernel_ptr_w(int kind, int nj, bool ga32, bool gb32, bool xt) {
+static const void *kernel_ptr_w(int kind, bool sm2, bool xt) {
   if (kind == KK_DIRECT) return (const void *)k_direct<W, 8, true>;
-  return xt ? kernel_ptr_x<W, true>(kind, nj, ga32, gb32)
-            : kernel_ptr_x<W, false>(kind, nj, ga32, gb32);
+  return xt ? kernel_ptr_x<W, true>(kind, sm2) : kernel_ptr_x<W, false>(kind, sm2);
 }
 
-static int pow2_at_least(int k) {
-  int p = 1;
-  while (p < k) p <<= 1;
-  return p;
-}
-
-// per-lane elements of a B-row (NJ <= 16)
-static int nj_of(const TileParams &K) {
-  const int k = pow2_at_least((K.LB + (1 << K.lgB) - 1) >> K.lgB);
-  return k <= 16 ? k : 16;  // longer runs: single output digit, chunked (planner rule)
-}
-
-static const void *kernel_ptr(int kind, int W, int nj, bool ga32, bool gb32, bool xt) {
+static const void *kernel_ptr(int kind, int W, bool sm2, bool xt) {
   switch (W) {
-    case 4: return kernel_ptr_w<4>(kind, nj, ga32, gb32, xt);
-    case 8: return kernel_ptr_w<8>(kind, nj, ga32, gb32, xt);
-    case 16: return kernel_ptr_w<16>(kind, nj, ga32, gb32, xt);
+    case 4: return kernel_ptr_w<4>(kind, sm2, xt);
+    case 8: return kernel_ptr_w<8>(kind, sm2, xt);
+    case 16: return kernel_ptr_w<16>(kind, sm2, xt);
   }
   return nullptr;
 }
@@ -486,7 +547,7 @@ int kernel_regs(int kind, int W) {
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, 4, true, true, false)) == cudaSuccess) {
+    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, false, false)) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -497,8 +558,7 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W, nj_of(plan->kp), plan->kp.lgA == 5,
-                              plan->kp.lgB == 5, plan->kp.xtab != 0);
+  const void *fn = kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0, plan->kp.xtab != 0);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

@@ -38,13 +38,22 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   } else {
     read_bytes = tiles * fill * mi.RA * run_cost((int64_t)mi.LA * mi.W);
     runsA = tiles * fill * mi.RA;
-    const double gA = group(mi.LA);
-    opsA = tiles * mi.RA * std::ceil(mi.LA / gA) / (32.0 / gA);
+    // flat load walk: ceil(V / threads) elements per thread
+    opsA = tiles * std::ceil((double)mi.V / mi.threads) * (mi.threads / 32.0);
   }
   const double write_bytes = tiles * fill * mi.RB * run_cost((int64_t)mi.LB * mi.W);
   const double runsB = tiles * fill * mi.RB;
-  const double gB = group(mi.LB);
-  const double opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);
+  double opsB;
+  if (mi.kind == KK_DIRECT) {
+    const double gB = group(mi.LB);
+    opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);
+  } else if (mi.LB <= mi.threads) {
+    // one output position per thread, B-rows strided by threads / LB
+    const double rs = std::floor((double)mi.threads / mi.LB);
+    opsB = tiles * std::ceil(mi.RB / rs) * (mi.threads / 32.0);
+  } else {
+    opsB = tiles * mi.RB * std::ceil((double)mi.LB / mi.threads) * (mi.threads / 32.0);
+  }
   const double sector = read_bytes + write_bytes;
   const double alg = 2.0 * mi.N * W;
   const double bw = dev.hbm_gbs * 1e9;

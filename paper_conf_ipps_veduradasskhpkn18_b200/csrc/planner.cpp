@@ -221,7 +221,7 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
   }
   S.buf_bytes = (int)r16(cur * P.W);
   S.smem_base = (int)(r16(S.RA * 8) + r16(S.RB * 8) + r16(S.LB * 4) + r16(S.RA * 4) +
-                      r16(S.RB * 4) + S.buf_bytes);
+                      r16(S.RB * 4) + 64 + S.buf_bytes);
   return true;
 }
 
@@ -377,6 +377,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.off_digB = take((int64_t)K.RA * 4);
     K.off_digA = take((int64_t)K.RB * 4);
     K.off_icol = xtab ? take((int64_t)K.LA * 4) : 0;
+    K.off_ctx = take(64);  // two decoded-tile slots (kernels.cu CtxS)
     K.off_data = take(smem_elems * P.W);
     K.off_data2 = K.off_data;
     for (int s = 1; s < nbuf; s++) {
@@ -395,13 +396,11 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   K.dxA = threads % K.LA;
   K.drB = threads / K.LB;
   K.dxB = threads % K.LB;
-  auto lg = [](int64_t L) {
-    int l = 0;
-    while ((1 << l) < L && l < 5) l++;
-    return l;
-  };
-  K.lgA = lg(K.LA);
-  K.lgB = lg(K.LB);
+  K.rsB = threads / K.LB;
+  K.fd_LA = make_fastdiv((uint32_t)K.LA);
+  K.fd_LB = make_fastdiv((uint32_t)K.LB);
+  K.fd_NT = make_fastdiv((uint32_t)threads);
+  K.fd_rsB = make_fastdiv((uint32_t)(K.rsB > 0 ? K.rsB : 1));
   return true;
 }
 
@@ -451,33 +450,33 @@ static void smem_conflicts(const TileParams &K, int W, double &load, double &sto
       }
     }
   };
-  int64_t addr[32], rows[32], cols[32];
-  // closed-form fast paths: a whole warp on one A-row reads consecutive words;
-  // a whole warp on one B-row whose first output digit spans the warp with an
-  // odd shared-memory stride (the padding rule) hits distinct banks
-  const bool load_free = K.lgA == 5 && !K.xtab;
-  const bool store_free = K.lgB == 5 && K.nj > 0 && K.j_ext[0] >= 32 && (K.j_sS[0] & 1);
+  int64_t addr[32], rows[33], cols[32];
+  // the first warp of each walk (kernels.cu k_pipe): load = flat over the tile
+  // (lane l -> A-row l / LA, run position l mod LA); store = lane l -> output
+  // position l mod LB of B-row l / LB (LB <= threads) or position l of B-row 0
+  const bool load_free = K.LA >= 32 && !K.xtab;
+  const bool store_free = K.LB >= 32 && K.nj > 0 && K.j_ext[0] >= 32 && (K.j_sS[0] & 1);
   load = store = 1.0;
   if (!load_free) {
-    const int g = 1 << K.lgA, nr = std::min(32 >> K.lgA, K.RA);
+    const int nr = std::min((31 / K.LA) + 1, K.RA);
     offsets(nr, K.nra, K.ra_ext, K.ra_sS, rows);
     if (K.xtab) {
       int32_t iext[TTLG_MAXD];
       for (int k = 0; k < K.ni; k++) iext[k] = (int32_t)K.i_div[k].div;
-      offsets(std::min(g, K.LA), K.ni, iext, K.i_sS, cols);
+      offsets(std::min(32, K.LA), K.ni, iext, K.i_sS, cols);
     }
     for (int l = 0; l < 32; l++) {
-      const int r = std::min(l >> K.lgA, nr - 1), x = std::min(l & (g - 1), K.LA - 1);
+      const int r = std::min(l / K.LA, nr - 1), x = std::min(l % K.LA, K.LA - 1);
       addr[l] = rows[r] + (K.xtab ? cols[x] : x);
     }
     load = wavefront_ratio(addr, W);
   }
   if (!store_free) {
-    const int g = 1 << K.lgB, nr = std::min(32 >> K.lgB, K.RB), nc = std::min(g, K.LB);
+    const int nr = std::min((31 / K.LB) + 1, K.RB), nc = std::min(32, K.LB);
     offsets(nr, K.nrb, K.rb_ext, K.rb_sS, rows);
     offsets(nc, K.nj, K.j_ext, K.j_sS, cols);
     for (int l = 0; l < 32; l++) {
-      const int r = std::min(l >> K.lgB, nr - 1), j = std::min(l & (g - 1), nc - 1);
+      const int r = std::min(l / K.LB, nr - 1), j = std::min(l % K.LB, nc - 1);
       addr[l] = rows[r] + cols[j];
     }
     store = wavefront_ratio(addr, W);
@@ -576,7 +575,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   widen(P, forceW);
 
   if (hints && hints->threads &&
-      (hints->threads < 64 || hints->threads > 512 || hints->threads % 32))
+      (hints->threads < 64 || hints->threads > 512 || hints->threads % 8))
     return TTLG_ERR_INVALID_VALUE;
   const int force_schema = hints ? hints->schema : TTLG_SCHEMA_AUTO;
 
@@ -762,9 +761,20 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (hv != 2) kinds[nk++] = KK_TILE;
       if (hv != 1) kinds[nk++] = KK_PIPE;
     }
+    // block sizes: 256 and 512, plus (staged kernels) the multiple of the
+    // output run LB nearest below 512 when 512 would leave >= 1/16 of the
+    // threads idle in the store walk (each thread owns one output position)
+    int tl[3] = {thr_list[0], thr_list[1], 0}, ntl = nthr;
+    if (group != KK_DIRECT && !(hints && hints->threads)) {
+      const int64_t LBc = S.LB;
+      if (LBc < 512 && (512 % LBc) * 16 >= 512) {
+        const int64_t m = (512 / LBc) * LBc;
+        if (m >= 192 && m % 8 == 0 && m != 256) tl[ntl++] = (int)m;
+      }
+    }
     for (int ki = 0; ki < nk; ki++) {
-      for (int ti = 0; ti < nthr; ti++) {
-        const int kind = kinds[ki], threads = thr_list[ti];
+      for (int ti = 0; ti < ntl; ti++) {
+        const int kind = kinds[ki], threads = tl[ti];
         ModelInput mi;
         int tpc;
         if (!make_mi(mi, tpc, kind, schema, threads, S, cl, cs)) continue;

@@ -101,9 +101,10 @@ struct TileParams {
   int32_t off_icol;
   // ---- shared-memory layout (bytes) and per-thread stepping
   int32_t smem_elems;      // data tile elements incl. padding
-  int32_t off_tabB, off_jcol, off_digB, off_digA, off_data, off_data2, smem_bytes;
+  int32_t off_tabB, off_jcol, off_digB, off_digA, off_ctx, off_data, off_data2, smem_bytes;
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
-  int32_t lgA, lgB;            // log2 of the lane-group size owning one A-row / B-row
+  int32_t rsB;                 // B-rows per pass of the store walk (threads / LB; 0: LB > threads)
+  FastDiv fd_LA, fd_LB, fd_NT, fd_rsB;  // per-thread walk setup without hardware division
   int32_t tpc;                 // tiles per CTA (consecutive tile indices)
 };
 

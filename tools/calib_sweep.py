@@ -56,6 +56,7 @@ def main():
     ap.add_argument("--max-cand", type=int, default=40)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--stride", type=int, default=1)
+    ap.add_argument("--ids", default="", help="comma list of case ids to keep")
     ap.add_argument("--threads", default="", help="comma list of block sizes to try per candidate")
     ap.add_argument("--top", action="store_true",
                     help="measure the linear screen's best candidates instead of a spread")
@@ -70,6 +71,9 @@ def main():
         cases += configs.all_configs()[args.group][::args.stride]
     if args.recipe:
         cases += recipe_cases(args.recipe, args.seed)
+    if args.ids:
+        keep = {int(x) for x in args.ids.split(",")}
+        cases = [c for c in cases if c.case_id in keep]
     dev = torch.device("cuda:0")
     stream = torch.cuda.current_stream()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
