@@ -83,12 +83,15 @@ typedef struct {
   int32_t out_dim;                       /* -1 = auto; position b of the last output dim
                                             of the output slice (Alg. 3 dimsOut)          */
   int64_t out_block;                     /* blockB, 0 = auto                             */
-  int32_t elem_bytes_override;           /* 0 = auto widening; else 4/8/16 access width  */
+  int32_t elem_bytes_override;           /* 0 = auto widening; else 4/8/16 access width
+                                            (pins the width: no k_quad 16-byte chunks)   */
   int32_t threads;                       /* 0 = auto; else threads per block             */
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
   int32_t variant;                       /* staged kernel: 0 = model choice, 1 = k_tile
-                                            (register-staged), 2 = k_pipe (cp.async)      */
+                                            (one tile per CTA), 2 = k_pipe (persistent,
+                                            double-buffered), 3 = k_quad (OD in 16-byte
+                                            chunks, K x K register transpose)            */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -110,7 +113,8 @@ typedef struct {
   double predicted_seconds;               /* performance-model prediction                */
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
-  int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe    */
+  int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe,
+                                             3 k_quad                                    */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[12];

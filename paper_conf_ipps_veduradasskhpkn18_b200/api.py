@@ -161,7 +161,7 @@ def candidate_hints(d: dict) -> dict:
          "in_block": d["tile_extents"][a], "out_dim": b,
          "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
     if d["kernel"] != "direct":
-        h["variant"] = 1 if d["kernel"] == "tile" else 2
+        h["variant"] = {"tile": 1, "pipe": 2, "quad": 3}[d["kernel"]]
     return h
 
 

@@ -122,8 +122,9 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
     cudaGetLastError();
     return TTLG_ERR_DEVICE;
   }
-  if ((a | b) % (uintptr_t)p->W) {
-    // widened access needs W-aligned pointers: re-plan at the element width
+  if ((a | b) % (uintptr_t)p->align) {
+    // widened / 16-byte-vector access needs aligned pointers: re-plan at the
+    // element width (elem_bytes_override also rules out k_quad)
     ttlg_plan_s q;
     ttlg_plan_hints h;
     if (p->has_hints) {
@@ -132,6 +133,7 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
       ttlg_plan_hints_init(&h);
     }
     h.elem_bytes_override = s;
+    if (h.variant == 3) h.variant = 0;  // k_quad needs 16-byte alignment
     ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h);
     if (st != TTLG_OK) return st;
     return launch(&q, A, B, stream);
@@ -386,7 +388,7 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
     h.out_dim = ci.out_dim;
     h.out_block = ci.tile_extents[ci.fused_perm[ci.out_dim]];
     h.threads = ci.threads;
-    h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : 0);
+    h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : (ci.kernel == KK_QUAD ? 3 : 0));
     ttlg_plan_s *q = new (std::nothrow) ttlg_plan_s;
     if (!q) break;
     if (plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h) != TTLG_OK) {

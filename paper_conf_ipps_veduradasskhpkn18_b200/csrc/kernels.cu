@@ -36,6 +36,11 @@
 
 #include "ttlg_internal.h"
 
+// 16-byte cp.async through L1 (.ca, default) or L2 only (.cg)
+#ifndef TTLG_CP16_CG
+#define TTLG_CP16_CG 0
+#endif
+
 namespace ttlg {
 
 template <int W>
@@ -74,7 +79,7 @@ __device__ __forceinline__ void st_stream(T *p, T v) {
 // registers across it.
 template <int W>
 __device__ __forceinline__ void cp_async(uint32_t s, const void *gptr) {
-  if constexpr (W == 16)
+  if constexpr (W == 16 && TTLG_CP16_CG)
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gptr));
   else
     asm volatile("cp.async.ca.shared.global [%0], [%1], %2;\n" ::"r"(s), "l"(gptr), "n"(W));
@@ -83,7 +88,7 @@ __device__ __forceinline__ void cp_async(uint32_t s, const void *gptr) {
 // lanes cost no branch / reconvergence)
 template <int W>
 __device__ __forceinline__ void cp_async_p(uint32_t s, const void *gptr, bool p) {
-  if constexpr (W == 16)
+  if constexpr (W == 16 && TTLG_CP16_CG)
     asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n"
                  " @q cp.async.cg.shared.global [%0], [%1], 16;\n}\n" ::"r"(s),
                  "l"(gptr), "r"((int)p));
@@ -514,6 +519,215 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
   }
 }
 
+// k_quad (OD in vector chunks): the
+// Orthogonal-Distinct tile (Alg. 2) moved entirely in CB-byte
+// accesses (CB = 16, or 8 for fp32 inputs whose FVIs are only even).
+// K = CB/S elements form a chunk.  Load: A-rows of LA contiguous elements ->
+// shared memory with CB-byte cp.async.  Store: a group of K lanes owns K
+// consecutive output positions j0..j0+K-1 (lane q reads the chunk of K
+// input-run positions x..x+K-1 at output position j0+q: ONE vector shared
+// load), the group transposes the K x K block in registers with
+// xor-shuffles, and lane q writes B-row x+q, positions j0..j0+K-1 as ONE
+// vector store.  Requirements (planner): OD; n0, n_perm[0], t0, t_perm[0]
+// multiples of K; whole warps; LB <= NJ * threads; CB-aligned pointers.  The
+// output-only dims of the shared tile are padded in chunk units so output
+// position j lands in chunk slot j mod (128/CB): conflict-free.
+template <int CB>
+struct Chunk;
+template <>
+struct Chunk<16> {
+  using T = uint4;
+};
+template <>
+struct Chunk<8> {
+  using T = uint2;
+};
+
+// lane q holds column q of a K x K block (rows in the chunk's element order);
+// afterwards it holds row q (columns in element order)
+template <int S, int CB>
+__device__ __forceinline__ void quad_transpose(typename Chunk<CB>::T &v, int q);
+template <>
+__device__ __forceinline__ void quad_transpose<4, 16>(uint4 &v, int q) {
+  const bool b = q & 1, h = q & 2;
+  uint32_t u0, u1, u2, u3;
+  {
+    const uint32_t r0 = __shfl_xor_sync(0xffffffffu, b ? v.x : v.y, 1);
+    const uint32_t r1 = __shfl_xor_sync(0xffffffffu, b ? v.z : v.w, 1);
+    u0 = b ? r0 : v.x;
+    u1 = b ? v.y : r0;
+    u2 = b ? r1 : v.z;
+    u3 = b ? v.w : r1;
+  }
+  const uint32_t s0 = __shfl_xor_sync(0xffffffffu, h ? u0 : u2, 2);
+  const uint32_t s1 = __shfl_xor_sync(0xffffffffu, h ? u1 : u3, 2);
+  v.x = h ? s0 : u0;
+  v.y = h ? s1 : u1;
+  v.z = h ? u2 : s0;
+  v.w = h ? u3 : s1;
+}
+template <>
+__device__ __forceinline__ void quad_transpose<8, 16>(uint4 &v, int q) {
+  // 2x2 block of 8-byte elements: (x,y) = row 0, (z,w) = row 1 of column q
+  const bool b = q & 1;
+  const uint32_t r0 = __shfl_xor_sync(0xffffffffu, b ? v.x : v.z, 1);
+  const uint32_t r1 = __shfl_xor_sync(0xffffffffu, b ? v.y : v.w, 1);
+  if (b) {
+    v.x = r0;
+    v.y = r1;
+  } else {
+    v.z = r0;
+    v.w = r1;
+  }
+}
+template <>
+__device__ __forceinline__ void quad_transpose<4, 8>(uint2 &v, int q) {
+  // 2x2 block of 4-byte elements: x = row 0, y = row 1 of column q
+  const bool b = q & 1;
+  const uint32_t r = __shfl_xor_sync(0xffffffffu, b ? v.x : v.y, 1);
+  if (b)
+    v.x = r;
+  else
+    v.y = r;
+}
+
+template <int S, int CB, int NJ>
+__global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TileParams P,
+                                                 const void *__restrict__ Av,
+                                                 void *__restrict__ Bv) {
+  constexpr int K = CB / S, LGK = K == 4 ? 2 : 1;
+  using C = typename Chunk<CB>::T;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_buf = s0 + P.off_data;
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
+  const unsigned char *A = reinterpret_cast<const unsigned char *>(Av);
+  unsigned char *B = reinterpret_cast<unsigned char *>(Bv);
+  const int tid = threadIdx.x, NT = blockDim.x;
+  const bool decoder = tid == NT - 1;
+  const uint32_t first = blockIdx.x * (uint32_t)P.tpc;
+
+  auto put_ctx = [&](int slot, uint32_t tile) {
+    const TileCtx c = decode_tile(P, tile);
+    ctx[slot].bA = c.bA;
+    ctx[slot].bB = c.bB;
+    ctx[slot].limA = c.limA;
+    ctx[slot].limB = c.limB;
+  };
+  if (decoder && first < P.num_tiles) put_ctx(0, first);
+  // row tables: (global element offset, shared byte offset)
+  build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
+             reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB), S);
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA), S);
+#pragma unroll 1
+  for (int j = tid; j < P.LB; j += NT) {
+    int rem = j, s = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+      s += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
+      rem = cq;
+    }
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * S;
+  }
+  __syncthreads();
+
+  const int LB = P.LB, LAc = P.LA / K;  // chunks per A-row
+  const int nChunks = P.V / K;
+  // load walk over chunks: chunk e = tid + k*NT -> A-row e / LAc, chunk e mod LAc
+  const int rA0 = (int)fdiv1(tid, P.fd_LA), cA0 = tid - rA0 * LAc;
+  const int nA = tid < nChunks ? (int)fdiv1(nChunks - 1 - tid, P.fd_NT) + 1 : 0;
+  const int drA = P.drA, dxA = P.dxA;
+  // store walk: output positions j0 + c*NT (c < NJ; NJ = 1 when LB <= NT),
+  // row quads m0, m0 + rsB, ...
+  int m0, j0, rs;
+  if (NJ == 1) {
+    m0 = (int)fdiv1(tid, P.fd_LB);
+    j0 = tid - m0 * LB;
+    rs = P.rsB;
+  } else {
+    m0 = 0;
+    j0 = tid;
+    rs = 1;
+  }
+  const int RBq = P.RB / K;
+  const int nB = (m0 < rs && m0 < RBq) ? (int)fdiv1(RBq - 1 - m0, P.fd_rsB) + 1 : 0;
+  const int q = j0 & (K - 1);
+  // the shuffles run warp-wide: every lane takes the warp's largest trip count
+  // (threads are a multiple of 32 for k_quad) and lanes past their own count
+  // re-read row quad 0 with the store predicated off
+  const int nBw = __reduce_max_sync(0xffffffffu, nB);
+  uint32_t jc[NJ];
+  bool jv[NJ];
+#pragma unroll
+  for (int c = 0; c < NJ; c++) {
+    const int jj = j0 + c * NT;
+    jv[c] = jj < LB;
+    jc[c] = lds_int(s_jcol + 4 * (jv[c] ? jj : j0));
+  }
+
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = first + it;
+    if (tile >= P.num_tiles) break;
+    if (it > 0) __syncthreads();
+    TileCtx c;
+    c.bA = ctx[it & 1].bA;
+    c.bB = ctx[it & 1].bB;
+    c.limA = ctx[it & 1].limA;
+    c.limB = ctx[it & 1].limB;
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    {  // load
+      const C *Ab = reinterpret_cast<const C *>(A + c.bA * S);  // chunk-aligned
+      const int limc = full ? LAc : (P.LAunit * c.limA) / K;
+      int r = rA0, cx = cA0;
+#pragma unroll 4
+      for (int k = 0; k < nA; k++) {
+        const int2 t = lds_int2(s_tabA + 8 * r);
+        const uint32_t soff = t.y + cx * CB;
+        const C *g = wadd(Ab, ((uint32_t)t.x >> LGK) + cx);
+        if (full)
+          cp_async<CB>(s_buf + soff, g);
+        else
+          cp_async_p<CB>(s_buf + soff, g, cx < limc && lds_int(s_digB + 4 * r) < c.limB);
+        cx += dxA;
+        r += drA;
+        if (cx >= LAc) {
+          cx -= LAc;
+          r++;
+        }
+      }
+    }
+    cp_async_commit();
+    if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
+    cp_async_wait<0>();
+    __syncthreads();
+    {  // store: one vector shared load, a K x K register transpose, one vector store
+      const int lim = full ? LB : P.LBunit * c.limB;
+      int m = m0;
+#pragma unroll 2
+      for (int k = 0; k < nBw; k++) {
+        const bool act = k < nB;
+        const int row = K * (act ? m : 0) + q;  // own B-row x+q after the transpose
+        const int2 t = lds_int2(s_tabB + 8 * row);
+        const bool rok = act && (full || lds_int(s_digA + 4 * row) < c.limA);
+        const uint32_t sq = s_buf + (t.y - q * S);  // chunk x..x+K-1
+#pragma unroll
+        for (int cc = 0; cc < NJ; cc++) {
+          C v = lds_T<C>(sq + jc[cc]);
+          quad_transpose<S, CB>(v, q);
+          const int jb = j0 + cc * NT - q;
+          C *dst = reinterpret_cast<C *>(B + (c.bB + jb) * S);
+          stcs_p(wadd(dst, (uint32_t)t.x >> LGK), v, rok && jv[cc] && (full || jb < lim));
+        }
+        m += rs;
+      }
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------
 // launch plumbing
 template <int W, bool XT>
@@ -530,6 +744,7 @@ static const void *kernel_ptr_w(int kind, bool sm2, bool xt) {
 }
 
 static const void *kernel_ptr(int kind, int W, bool sm2, bool xt) {
+  if (kind == KK_QUAD) return nullptr;  // quad_ptr()
   switch (W) {
     case 4: return kernel_ptr_w<4>(kind, sm2, xt);
     case 8: return kernel_ptr_w<8>(kind, sm2, xt);
@@ -540,14 +755,25 @@ static const void *kernel_ptr(int kind, int W, bool sm2, bool xt) {
 
 static int widx(int W) { return W == 4 ? 0 : (W == 8 ? 1 : 2); }
 
+template <int S, int CB>
+static const void *quad_ptr_nj(int nj) {
+  return nj <= 1 ? (const void *)k_quad<S, CB, 1>
+                 : (nj == 2 ? (const void *)k_quad<S, CB, 2> : (const void *)k_quad<S, CB, 4>);
+}
+static const void *quad_ptr(int W, int cb, int nj) {
+  if (W == 8) return quad_ptr_nj<8, 16>(nj);
+  return cb == 16 ? quad_ptr_nj<4, 16>(nj) : quad_ptr_nj<4, 8>(nj);
+}
+
 int kernel_regs(int kind, int W) {
-  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
+  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
   static std::mutex mu;
   std::lock_guard<std::mutex> g(mu);
   int &r = regs[kind][widx(W)];
   if (r < 0) {
     cudaFuncAttributes attr;
-    if (cudaFuncGetAttributes(&attr, kernel_ptr(kind, W, false, false)) == cudaSuccess) {
+    const void *fn = kind == KK_QUAD ? quad_ptr(W, 16, 1) : kernel_ptr(kind, W, false, false);
+    if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
       r = attr.numRegs;
     } else {
       cudaGetLastError();
@@ -558,7 +784,9 @@ int kernel_regs(int kind, int W) {
 }
 
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
-  const void *fn = kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0, plan->kp.xtab != 0);
+  const void *fn = plan->kind == KK_QUAD
+                       ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
+                       : kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0, plan->kp.xtab != 0);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

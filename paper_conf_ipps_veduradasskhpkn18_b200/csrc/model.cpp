@@ -38,8 +38,9 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   } else {
     read_bytes = tiles * fill * mi.RA * run_cost((int64_t)mi.LA * mi.W);
     runsA = tiles * fill * mi.RA;
-    // flat load walk: ceil(V / threads) elements per thread
-    opsA = tiles * std::ceil((double)mi.V / mi.threads) * (mi.threads / 32.0);
+    // flat load walk: ceil(V / threads) access elements (k_quad: 16-byte chunks) per thread
+    const double vk = mi.kind == KK_QUAD ? (double)mi.V / std::max(1, mi.qk) : (double)mi.V;
+    opsA = tiles * std::ceil(vk / mi.threads) * (mi.threads / 32.0);
   }
   const double write_bytes = tiles * fill * mi.RB * run_cost((int64_t)mi.LB * mi.W);
   const double runsB = tiles * fill * mi.RB;
@@ -48,9 +49,13 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
     const double gB = group(mi.LB);
     opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);
   } else if (mi.LB <= mi.threads) {
-    // one output position per thread, B-rows strided by threads / LB
+    // one output position per thread, B-rows (k_quad: groups of K B-rows) strided by threads / LB
     const double rs = std::floor((double)mi.threads / mi.LB);
-    opsB = tiles * std::ceil(mi.RB / rs) * (mi.threads / 32.0);
+    const double rows = mi.kind == KK_QUAD ? (double)mi.RB / std::max(1, mi.qk) : (double)mi.RB;
+    opsB = tiles * std::ceil(rows / rs) * (mi.threads / 32.0);
+  } else if (mi.kind == KK_QUAD) {
+    opsB = tiles * ((double)mi.RB / std::max(1, mi.qk)) * std::ceil((double)mi.LB / mi.threads) *
+           (mi.threads / 32.0);
   } else {
     opsB = tiles * mi.RB * std::ceil((double)mi.LB / mi.threads) * (mi.threads / 32.0);
   }
@@ -91,6 +96,7 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
   const ModelFeatures F = model_features(mi, dev);
   const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect
                     : (mi.kind == KK_TILE) ? kCoefTile
+                    : (mi.kind == KK_QUAD) ? kCoefQuad
                                            : kCoefPipe;
   double t = 0.0;
   for (int i = 0; i < kModelNumFeatures; i++) t += c[i] * F.f[i];
@@ -125,10 +131,15 @@ void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d)
   d[9] = F.f[2] / std::max(F.f[1], 1e-12);
   d[10] = F.f[8] / std::max(1.0, bytes / 1e9);
   d[11] = (double)mi.num_tiles / (dev.sms * occ);
+  const double RA = V / (mi.kind == KK_DIRECT ? V : (double)mi.LA), RB = V / (double)mi.LB;
+  d[12] = std::log2(V / th);                       // elements per thread
+  d[13] = (RA + RB + (double)mi.LB) / th;          // per-CTA table entries per thread
+  d[14] = mi.fillA;                                // useful fraction of the tile grid
+  d[15] = std::ceil((double)mi.num_tiles / std::max(1, mi.grid));  // tiles per CTA
 }
 
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
-  double d[12];
+  double d[kGbtDesc];
   model_descriptor(mi, dev, d);
   double s = kGbtInit;
   for (int t = 0; t < kGbtTrees; t++) {

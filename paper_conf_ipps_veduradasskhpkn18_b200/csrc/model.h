@@ -24,6 +24,7 @@ struct ModelInput {
   int threads, smem_bytes, occ, grid;
   double fillA;  // useful fraction of the tile grid (partial tiles)
   double conf_load, conf_store;  // smem wavefronts / ideal for one warp access (>= 1)
+  int qk;                        // k_quad chunk elements (0: scalar kernels)
 };
 
 struct ModelFeatures {
@@ -34,6 +35,7 @@ struct ModelFeatures {
 ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev);
 double predict_seconds(const ModelInput &mi, const DeviceProfile &dev);
 // ranking stage (boosted trees over model_descriptor); seconds
+constexpr int kGbtDesc = 16;  // descriptor length (tools/calibrate_gbt.py desc())
 void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d);
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
 

@@ -8,8 +8,9 @@ constexpr int kModelNumFeatures = 10;
 constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
 constexpr double kModelUnroll = 8.0;         // loads in flight per thread (k_direct, k_tile)
 // features: see model.cpp model_features()
-constexpr double kCoefDirect[kModelNumFeatures] = {6.864575e-06, 8.651936e-01, 9.614488e-01, 9.125569e-11, 1.499405e-10, 4.959539e-01, 2.254551e-01, 6.084763e-07, 0.000000e+00, 1.051936e-09};
-constexpr double kCoefTile[kModelNumFeatures] = {9.051371e-06, 5.877510e-01, 1.426655e-01, 5.176052e-10, 0.000000e+00, 0.000000e+00, 4.584064e-02, 1.809984e-06, 2.257271e-11, 1.886434e-09};
-constexpr double kCoefPipe[kModelNumFeatures] = {6.578404e-06, 5.461088e-01, 0.000000e+00, 4.396413e-10, 2.259999e-08, 0.000000e+00, 0.000000e+00, 1.564538e-06, 0.000000e+00, 2.021733e-09};
-constexpr const char *kModelSource = "B200 fit (402 cases, 31238 points, rel<=3.0): direct: train 5.4% test 7.9% (n=1012+117); tile: train 12.0% test 12.0% (n=10498+2869); pipe: train 11.3% test 11.9% (n=7331+2168); regret 12.5%";
+constexpr double kCoefDirect[kModelNumFeatures] = {6.347335e-06, 8.843837e-01, 0.000000e+00, 1.981821e-10, 0.000000e+00, 7.767651e-01, 2.173065e-01, 2.140969e-07, 0.000000e+00, 1.156034e-09};
+constexpr double kCoefTile[kModelNumFeatures] = {9.119138e-06, 8.575126e-01, 0.000000e+00, 4.233825e-11, 0.000000e+00, 3.127599e-01, 0.000000e+00, 3.477675e-07, 4.100381e-10, 1.423466e-09};
+constexpr double kCoefPipe[kModelNumFeatures] = {8.107715e-06, 8.890406e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.413858e-01, 2.939497e-01, 0.000000e+00, 4.139314e-10, 1.699514e-09};
+constexpr double kCoefQuad[kModelNumFeatures] = {1.022917e-05, 8.662868e-01, 0.000000e+00, 1.546947e-10, 0.000000e+00, 3.629821e-01, 3.003596e-01, 3.371972e-07, 0.000000e+00, 2.147497e-09};
+constexpr const char *kModelSource = "B200 fit (282 cases, 38128 points, rel<=1.5): direct: train 4.3% test 4.2% (n=482+62); tile: train 7.9% test 7.6% (n=5959+1653); pipe: train 7.8% test 7.6% (n=5785+1612); quad: train 7.7% test 6.7% (n=2225+678); regret 14.7%";
 }  // namespace ttlg

@@ -171,6 +171,7 @@ Tile make_tile(const Problem &P, int a, int64_t ta, int b, int64_t tb) {
 
 int schema_of(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_DIRECT) return P.d == 1 ? TTLG_SCHEMA_COPY : TTLG_SCHEMA_FML;
+  if (kind == KK_QUAD) return TTLG_SCHEMA_OD;
   if (P.p[0] == 0) return TTLG_SCHEMA_FMS;
   for (int i = 0; i <= T.b; i++)
     if (P.p[i] <= T.a) return TTLG_SCHEMA_OA;  // input and output groups overlap
@@ -179,18 +180,65 @@ int schema_of(const Problem &P, const Tile &T, int kind) {
 
 int64_t ceil_div(int64_t x, int64_t y) { return (x + y - 1) / y; }
 
+// k_quad (vector chunks in and out, K x K register transpose): an OD tile
+// whose input FVI and output FVI extents and blocks are multiples of K (so
+// every A-row, B-row and tile base is chunk-aligned).  K = 16 / W (16-byte
+// chunks); fp32 tiles whose FVIs are only even use K = 2 (8-byte chunks).
+// Returns K, or 0 when no chunking applies.
+int quad_k(const Problem &P, const Tile &T) {
+  if (P.W != P.esize || P.p[0] == 0) return 0;
+  for (int i = 0; i <= T.b; i++)
+    if (P.p[i] <= T.a) return 0;  // groups overlap: not OD
+  const int p0 = P.p[0];
+  for (int K = 16 / P.W; K >= 2; K /= 2) {
+    if (P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 && T.t[p0] % K == 0) return K;
+    if (P.W == 8) break;  // fp64: 16-byte chunks only
+  }
+  return 0;
+}
+
+// Shared-memory stride of the next output-only dim (the generalisation of the
+// 32x33 pad, L747-749, and FMS's "row 1 starts at bank N0", L1104-1107).  In
+// units u of one access element (scalar kernels, 128/W units per 128-byte
+// bank row) or one K-element chunk (k_quad, 128/(K W) chunk slots), output
+// position j must land in slot (mult * j) mod slots with mult odd: 16 or 32
+// consecutive positions then hit distinct slots.  A dim whose prefix product
+// in output order is Q gets the smallest stride >= cur that is congruent to
+// mult * Q.  OD tiles pick mult freely on the first dim (the smallest odd
+// stride >= cur: no padding at all for odd runs); tiles whose output run
+// includes input-run dims (OA/FMS) keep mult = 1, because those dims'
+// strides are fixed by the contiguous input run.
+int64_t pad_stride(int64_t cur, int64_t Q, int W, int K, bool od, int64_t &mult) {
+  const int64_t unit = K > 0 ? K : 1;
+  const int64_t slots = 128 / (unit * W);
+  const int64_t u = (cur + unit - 1) / unit;
+  if (mult == 0) {
+    if (od) {
+      const int64_t s = u | 1;  // smallest odd stride >= cur
+      mult = s % slots;
+      return s * unit;
+    }
+    mult = 1;
+  }
+  const int64_t target = (mult * Q) % slots;
+  return unit * (u + (((target - u) % slots) + slots) % slots);
+}
+
 }  // namespace
 
 // Cheap geometry summary of a tile (what the model needs), without building
 // the parameter block: used to screen candidates before the full build.
 struct TileSummary {
   int64_t V, LA, LB, RA, RB, tiles;
+  int qk;         // k_quad chunk elements (0: scalar kernels)
   int smem_base;  // shared memory with one data buffer
   int buf_bytes;  // one data buffer
 };
 
 static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S) {
   const int d = P.d, a = T.a, b = T.b;
+  const int qk = kind == KK_QUAD ? quad_k(P, T) : 0;
+  S.qk = qk;
   bool inIS[TTLG_MAXD] = {false};
   for (int k = 0; k <= a; k++) inIS[k] = true;
   S.V = 1;
@@ -212,11 +260,12 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
     S.buf_bytes = 0;
     return true;
   }
-  int64_t cur = S.LA, Q = 1;
-  const int64_t Wb = 128 / P.W;
+  int64_t cur = S.LA, Q = 1, mult = 0;
+  bool od = true;
+  for (int i = 0; i <= b; i++) od &= !inIS[P.p[i]];
   for (int i = 0; i <= b; i++) {
     const int k = P.p[i];
-    if (!inIS[k] && T.t[k] > 1) cur = (cur + (((Q - cur) % Wb) + Wb) % Wb) * T.t[k];
+    if (!inIS[k] && T.t[k] > 1) cur = pad_stride(cur, Q, P.W, qk, od, mult) * T.t[k];
     Q *= T.t[k];
   }
   S.buf_bytes = (int)r16(cur * P.W);
@@ -229,6 +278,8 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
 static bool build_params(const Problem &P, const Tile &T, int kind, int threads, int nbuf,
                          TileParams &K, const int *isdelta = nullptr) {
   memset(&K, 0, sizeof(K));
+  const int qk = kind == KK_QUAD ? quad_k(P, T) : 0;
+  if (kind == KK_QUAD && qk == 0) return false;
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
   bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
@@ -298,12 +349,13 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     sm[k] = cur + pad;
     cur = sm[k] * T.t[k];
   }
-  const int64_t Wb = 128 / P.W;
-  int64_t Q = 1;
+  int64_t Q = 1, mult = 0;
+  bool od = true;
+  for (int i = 0; i <= b; i++) od &= !inIS[P.p[i]];
   for (int i = 0; i <= b; i++) {
     const int k = P.p[i];
     if (!inIS[k] && T.t[k] > 1) {
-      int64_t s = cur + (((Q - cur) % Wb) + Wb) % Wb;
+      const int64_t s = pad_stride(cur, Q, P.W, qk, od, mult);
       sm[k] = s;
       cur = s * T.t[k];
     }
@@ -397,7 +449,16 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   K.drB = threads / K.LB;
   K.dxB = threads % K.LB;
   K.rsB = threads / K.LB;
-  K.fd_LA = make_fastdiv((uint32_t)K.LA);
+  if (kind == KK_QUAD) {  // the load walk runs over chunks
+    K.qk = qk;
+    K.qnj = K.LB <= threads ? 1 : (K.LB <= 2 * threads ? 2 : 4);
+    const int LAc = K.LA / qk;
+    K.drA = threads / LAc;
+    K.dxA = threads % LAc;
+    K.fd_LA = make_fastdiv((uint32_t)LAc);
+  } else {
+    K.fd_LA = make_fastdiv((uint32_t)K.LA);
+  }
   K.fd_LB = make_fastdiv((uint32_t)K.LB);
   K.fd_NT = make_fastdiv((uint32_t)threads);
   K.fd_rsB = make_fastdiv((uint32_t)(K.rsB > 0 ? K.rsB : 1));
@@ -616,6 +677,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                      const TileSummary &S, double cl, double cs) {
     const int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
     if (smem > dev.smem_per_block_optin) return false;
+    // k_quad: at most 4 output positions per thread, warp-wide shuffles (whole warps)
+    if (kind == KK_QUAD && (S.LB > 4 * threads || threads % 32)) return false;
+    mi.qk = kind == KK_QUAD ? S.qk : 0;
     mi.kind = kind;
     mi.schema = schema;
     mi.W = P.W;
@@ -657,6 +721,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     cl = cs = 1.0;
     if (!build_params(P, T, group, thr_list[0], 1, K0)) return false;
     if (group == KK_DIRECT) return true;
+    if (group == KK_QUAD) {  // conflict-free by construction (16-byte slot j mod 8)
+      S.smem_base = K0.smem_bytes;
+      S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
+      return true;
+    }
     smem_conflicts(K0, P.W, cl, cs);
     if (cl + cs > 2.0) {
       const int lp = 128 / P.W;
@@ -723,6 +792,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     Tile T = make_tile(P, a, ta, b, tb);
     if (!T.ok) return;
+    if (group == KK_QUAD && (!quad_k(P, T) || forceW || (hv != 0 && hv != 3))) return;
     const int schema = schema_of(P, T, group);
     if (force_schema != TTLG_SCHEMA_AUTO && force_schema != schema) {
       // COPY and FML share the direct kernel; accept FML for a rank-1 problem
@@ -757,7 +827,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int kinds[2], nk = 0;
     if (group == KK_DIRECT) {
       kinds[nk++] = KK_DIRECT;
+    } else if (group == KK_QUAD) {
+      kinds[nk++] = KK_QUAD;
     } else {
+      if (hv == 3) return;
       if (hv != 2) kinds[nk++] = KK_TILE;
       if (hv != 1) kinds[nk++] = KK_PIPE;
     }
@@ -834,6 +907,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           for (int i = 0; i < nbA; i++) {
             for (int j = 0; j < nbB; j++) {
               consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
+              consider(KK_QUAD, a, blocksA[i], b, blocksB[j]);
             }
           }
         }
@@ -946,6 +1020,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->kind = B.kind;
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
+  plan->align = B.kind == KK_QUAD ? K.qk * P.W : P.W;
   plan->threads = B.mi.threads;
   plan->grid = B.mi.grid;
   plan->nbytes = N * P.W;

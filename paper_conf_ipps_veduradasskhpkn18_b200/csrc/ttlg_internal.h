@@ -46,7 +46,8 @@ enum KernelKind : int32_t {
   KK_DIRECT = 0,  // FML / COPY: contiguous input run -> rows of the output run, no smem staging
   KK_TILE = 1,    // OD / OA / FMS: register-staged, one tile per CTA (k_tile)
   KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered, persistent (k_pipe)
-  KK_NUM = 3,
+  KK_QUAD = 3,    // OD: 16-byte chunks in and out, K x K register transpose (k_quad)
+  KK_NUM = 4,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -105,6 +106,7 @@ struct TileParams {
   int32_t drA, dxA, drB, dxB;  // divmod(threads, LA) and divmod(threads, LB)
   int32_t rsB;                 // B-rows per pass of the store walk (threads / LB; 0: LB > threads)
   FastDiv fd_LA, fd_LB, fd_NT, fd_rsB;  // per-thread walk setup without hardware division
+  int32_t qk, qnj;             // k_quad: chunk elements K (0: scalar kernels), column slots
   int32_t tpc;                 // tiles per CTA (consecutive tile indices)
 };
 
@@ -132,6 +134,7 @@ struct ttlg_plan_s {
   int device;  // -1 when planned against the virtual profile
   int kind;    // ttlg::KernelKind
   int W;       // access bytes
+  int align;   // pointer alignment the kernel needs (W, or 16 for k_quad)
   int threads;
   int grid;
   int variant;  // reserved (hints->variant)

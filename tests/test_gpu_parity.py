@@ -314,3 +314,81 @@ def test_plan_tune_measure_mode():
         p.execute(A.data_ptr(), B.data_ptr(), torch.cuda.current_stream().cuda_stream)
         torch.cuda.synchronize()
         _assert_equal(_bits(B), oracle.transpose(_bits(A), c.extents, c.perm), "tuned plan")
+
+
+# ---- every staged kernel variant forced (k_tile 1, k_pipe 2, k_quad 3), ragged tiles ----------
+_VARIANT_CASES = [
+    ([5120 // 16, 5120 // 20], [1, 0], 8),         # 2-D OD
+    ([52, 36], [1, 0], 4),                           # small 2-D, partial tiles
+    ([4, 1000, 60], [1, 2, 0], 4),                   # AoS -> SoA (fuses to [4, 60000] 1 0)
+    ([8, 44, 36], [2, 1, 0], 4),
+    ([24, 20, 12, 8], [3, 1, 0, 2], 8),
+    ([16, 6, 10, 12, 4], [2, 0, 4, 1, 3], 8),
+    ([12, 14, 16, 10], [1, 0, 3, 2], 4),
+    ([2, 1000, 60], [1, 2, 0], 4),                   # fp32 even FVI: 8-byte chunks (K = 2)
+    ([6, 44, 36], [2, 1, 0], 4),
+    ([2, 300, 40], [1, 0, 2], 4),
+]
+
+
+@pytest.mark.parametrize("variant", [1, 2, 3])
+@pytest.mark.parametrize("ext,perm,eb", _VARIANT_CASES)
+def test_kernel_variants_forced(ext, perm, eb, variant):
+    try:
+        ttlg.plan(_dt(eb), ext, perm, variant=variant)
+    except ttlg.TtlgError:
+        pytest.skip("variant not applicable")
+    got, exp, info = _run(ext, perm, eb, 77, plan_kwargs={"variant": variant}, canary=64)
+    _assert_equal(got, exp, f"variant {variant} {info}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_quad_partial_tiles_and_blocks(eb):
+    """k_quad under every block factor pair that leaves partial tiles on both sides."""
+    ext, perm = [20 * (16 // eb), 28, 3], [1, 0, 2]
+    n_ok = 0
+    for ib in (4, 8, 12):
+        for ob in (4, 8, 12, 16):
+            kw = {"variant": 3, "in_dim": 0, "in_block": ib, "out_dim": 0, "out_block": ob}
+            try:
+                ttlg.plan(_dt(eb), ext, perm, **kw)
+            except ttlg.TtlgError:
+                continue
+            got, exp, info = _run(ext, perm, eb, 91, plan_kwargs=kw, canary=32)
+            assert info["kernel"] == "quad"
+            _assert_equal(got, exp, f"quad {kw}")
+            n_ok += 1
+    assert n_ok >= 4
+
+
+def test_quad_misaligned_pointers_fall_back():
+    ext, perm = [64, 96], [1, 0]
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(5, n + 1, 4, device=DEV)
+    B = torch.empty(n + 1, dtype=torch.float32, device=DEV)
+    p = ttlg.plan("f32", ext, perm, variant=3)
+    assert p.describe()["kernel"] == "quad"
+    p.execute(A[1:].data_ptr(), B[1:].data_ptr(), torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    _assert_equal(_bits(B[1:]), oracle.transpose(_bits(A[1:]), ext, perm), "quad misaligned")
+
+
+@pytest.mark.parametrize("ext,eb,ob,threads", [([8, 3000], 4, 1024, 256), ([8, 3000], 4, 512, 256),
+                                               ([6, 2050], 4, 2048, 512), ([4, 1800], 8, 1024, 256)])
+def test_quad_multi_column(ext, eb, ob, threads):
+    """k_quad with output runs longer than the block (2 or 4 positions per thread), ragged."""
+    kw = {"variant": 3, "in_dim": 0, "in_block": ext[0], "out_dim": 0, "out_block": ob,
+          "threads": threads}
+    got, exp, info = _run(ext, [1, 0], eb, 93, plan_kwargs=kw, canary=32)
+    assert info["kernel"] == "quad" and info["out_run"] > threads
+    _assert_equal(got, exp, f"quad multi-column {kw}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_all_720_rank6_perms(eb):
+    """N3: every permutation of a rank-6 tensor (the paper's 720-perm sweep,
+    L1484-1493) at an oracle-sized shape with odd and even extents."""
+    ext = [3, 4, 2, 5, 2, 3]
+    for k, perm in enumerate(itertools.permutations(range(6))):
+        got, exp, info = _run(ext, list(perm), eb, 3000 + k)
+        _assert_equal(got, exp, f"{perm} {info['schema']} {info['kernel']}")

@@ -199,3 +199,17 @@ def test_torch_to_c_matches_numpy_transpose():
         assert np.array_equal(got, np.ascontiguousarray(X.transpose(perm_t)).ravel())
     # 2-D: (1, 0) <-> (1, 0)
     assert ttlg.torch_to_c([3, 5], [1, 0]) == ([5, 3], [1, 0])
+
+
+def test_plan_candidates_every_config_case():
+    """Listing mode (calibration) builds the exact parameter block of every
+    candidate of every kernel family: must never fault on any config case."""
+    from synth import configs
+    groups = configs.all_configs()
+    for g in ("c1", "c2", "c3", "c4"):
+        for c in groups[g]:
+            dt = "f64" if c.elem_bytes == 8 else "f32"
+            cands = ttlg.plan_candidates(dt, c.extents, c.perm)
+            assert cands, c.label()
+            kinds = {d["kernel"] for d in cands}
+            assert kinds <= {"direct", "tile", "pipe", "quad"}

@@ -24,7 +24,7 @@ from scipy.optimize import nnls
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 COEFF_H = os.path.join(ROOT, "paper_conf_ipps_veduradasskhpkn18_b200", "csrc", "model_coeffs.h")
-KINDS = ["direct", "tile", "pipe"]
+KINDS = ["direct", "tile", "pipe", "quad"]
 
 
 def fit(rows):
@@ -96,7 +96,8 @@ def main():
         with open(COEFF_H) as f:
             src = f.read()
         lines = []
-        for k, name in (("direct", "kCoefDirect"), ("tile", "kCoefTile"), ("pipe", "kCoefPipe")):
+        for k, name in (("direct", "kCoefDirect"), ("tile", "kCoefTile"), ("pipe", "kCoefPipe"),
+                        ("quad", "kCoefQuad")):
             if k in coefs:
                 vals = ", ".join(f"{v:.6e}" for v in coefs[k])
                 lines.append(f"constexpr double {name}[kModelNumFeatures] = {{{vals}}};")

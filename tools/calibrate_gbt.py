@@ -26,10 +26,10 @@ from sklearn.ensemble import GradientBoostingRegressor
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 CSRC = os.path.join(ROOT, "paper_conf_ipps_veduradasskhpkn18_b200", "csrc")
-KID = {"direct": 0, "tile": 1, "pipe": 2}
+KID = {"direct": 0, "tile": 1, "pipe": 2, "quad": 3}
 HBM = 6555.5e9
 SMS = 148
-TOPK = 16
+TOPK = int(os.environ.get("TTLG_GBT_TOPK", "16"))
 
 
 def desc(r):
@@ -38,10 +38,15 @@ def desc(r):
     occ, th = max(1, r["occ"]), r["threads"]
     LAb = (V if r["kernel"] == "direct" else r["LA"]) * W
     f = r["features"]
+    N = r["bytes"] / (2.0 * W)
+    RA = V / (V if r["kernel"] == "direct" else r["LA"])
+    RB = V / r["LB"]
     return [KID[r["kernel"]], math.log2(W), math.log2(LAb), math.log2(r["LB"] * W),
             math.log2(V * W), th / 256.0, float(occ), occ * th / 2048.0,
             math.log2(r["tiles"]), f[2] / max(f[1], 1e-12), f[8] / max(1.0, r["bytes"] / 1e9),
-            r["tiles"] / (SMS * occ)]
+            r["tiles"] / (SMS * occ),
+            math.log2(V / th), (RA + RB + r["LB"]) / th, N / (r["tiles"] * V),
+            math.ceil(r["tiles"] / r["grid"])]
 
 
 def ideal(r):
@@ -51,7 +56,8 @@ def ideal(r):
 def linear_coefs():
     src = open(os.path.join(CSRC, "model_coeffs.h")).read()
     co = {}
-    for name, k in (("kCoefDirect", "direct"), ("kCoefTile", "tile"), ("kCoefPipe", "pipe")):
+    for name, k in (("kCoefDirect", "direct"), ("kCoefTile", "tile"), ("kCoefPipe", "pipe"),
+                    ("kCoefQuad", "quad")):
         m = re.search(name + r"\[kModelNumFeatures\] = \{([^}]*)\}", src)
         co[k] = np.array([float(x) for x in m.group(1).split(",")])
     return co
