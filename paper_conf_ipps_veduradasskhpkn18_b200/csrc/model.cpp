@@ -139,16 +139,37 @@ void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d)
 }
 
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
-  double d[kGbtDesc];
-  model_descriptor(mi, dev, d);
-  double s = kGbtInit;
-  for (int t = 0; t < kGbtTrees; t++) {
-    int n = kGbtRoot[t];
-    while (kGbtFeat[n] >= 0) n = (d[kGbtFeat[n]] <= (double)kGbtThr[n]) ? kGbtLeft[n] : kGbtRight[n];
-    s += kGbtVal[n];
+  double t;
+  predict_ranked_batch(&mi, 1, dev, &t);
+  return t;
+}
+
+// The candidates' traversals of one tree are independent: interleaving them
+// (tree-major) lets the core overlap their dependent node loads.
+void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
+  constexpr int kB = 32;
+  double d[kB][kGbtDesc], s[kB];
+  for (int b0 = 0; b0 < n; b0 += kB) {
+    const int m = std::min(kB, n - b0);
+    for (int c = 0; c < m; c++) {
+      model_descriptor(mis[b0 + c], dev, d[c]);
+      s[c] = kGbtInit;
+    }
+    for (int t = 0; t < kGbtTrees; t++) {
+      const int root = kGbtRoot[t];
+      for (int c = 0; c < m; c++) {
+        int k = root;
+        while (kGbtNodes[k].f >= 0)
+          k = (d[c][kGbtNodes[k].f] <= (double)kGbtNodes[k].t) ? k + 1 : kGbtNodes[k].r;
+        s[c] += kGbtNodes[k].t;
+      }
+    }
+    for (int c = 0; c < m; c++) {
+      const ModelInput &mi = mis[b0 + c];
+      const double ideal = 2.0 * (double)mi.N * mi.W / (dev.hbm_gbs * 1e9);
+      out[b0 + c] = std::exp(std::max(s[c], 0.0)) * ideal;  // never below one pass at copy speed
+    }
   }
-  const double ideal = 2.0 * (double)mi.N * mi.W / (dev.hbm_gbs * 1e9);
-  return std::exp(std::max(s, 0.0)) * ideal;  // never below one pass at copy speed
 }
 
 }  // namespace ttlg

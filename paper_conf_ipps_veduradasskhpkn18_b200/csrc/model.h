@@ -38,5 +38,6 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev);
 constexpr int kGbtDesc = 16;  // descriptor length (tools/calibrate_gbt.py desc())
 void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d);
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
+void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
 
 }  // namespace ttlg

@@ -8,9 +8,9 @@ constexpr int kModelNumFeatures = 10;
 constexpr double kModelLatency = 1.0e-6;     // loaded DRAM latency (s)
 constexpr double kModelUnroll = 8.0;         // loads in flight per thread (k_direct, k_tile)
 // features: see model.cpp model_features()
-constexpr double kCoefDirect[kModelNumFeatures] = {6.347335e-06, 8.843837e-01, 0.000000e+00, 1.981821e-10, 0.000000e+00, 7.767651e-01, 2.173065e-01, 2.140969e-07, 0.000000e+00, 1.156034e-09};
-constexpr double kCoefTile[kModelNumFeatures] = {9.119138e-06, 8.575126e-01, 0.000000e+00, 4.233825e-11, 0.000000e+00, 3.127599e-01, 0.000000e+00, 3.477675e-07, 4.100381e-10, 1.423466e-09};
-constexpr double kCoefPipe[kModelNumFeatures] = {8.107715e-06, 8.890406e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.413858e-01, 2.939497e-01, 0.000000e+00, 4.139314e-10, 1.699514e-09};
-constexpr double kCoefQuad[kModelNumFeatures] = {1.022917e-05, 8.662868e-01, 0.000000e+00, 1.546947e-10, 0.000000e+00, 3.629821e-01, 3.003596e-01, 3.371972e-07, 0.000000e+00, 2.147497e-09};
-constexpr const char *kModelSource = "B200 fit (282 cases, 38128 points, rel<=1.5): direct: train 4.3% test 4.2% (n=482+62); tile: train 7.9% test 7.6% (n=5959+1653); pipe: train 7.8% test 7.6% (n=5785+1612); quad: train 7.7% test 6.7% (n=2225+678); regret 14.7%";
+constexpr double kCoefDirect[kModelNumFeatures] = {6.621356e-06, 8.801143e-01, 8.640416e-02, 1.966767e-10, 0.000000e+00, 8.763387e-01, 2.180839e-01, 2.113898e-07, 0.000000e+00, 1.182271e-09};
+constexpr double kCoefTile[kModelNumFeatures] = {8.564110e-06, 8.672552e-01, 4.235581e-02, 3.343247e-11, 0.000000e+00, 3.600222e-01, 8.875134e-02, 2.948236e-07, 3.549572e-10, 1.462520e-09};
+constexpr double kCoefPipe[kModelNumFeatures] = {7.472125e-06, 9.025470e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.375855e-01, 4.479036e-01, 0.000000e+00, 3.127622e-10, 1.671868e-09};
+constexpr double kCoefQuad[kModelNumFeatures] = {8.068869e-06, 8.957848e-01, 0.000000e+00, 1.501453e-10, 0.000000e+00, 3.723977e-01, 1.773548e-01, 2.590639e-07, 0.000000e+00, 2.316751e-09};
+constexpr const char *kModelSource = "B200 fit (362 cases, 43650 points, rel<=1.5): direct: train 4.7% test 7.8% (n=854+167); tile: train 7.9% test 8.0% (n=7618+1987); pipe: train 7.7% test 7.8% (n=6688+1699); quad: train 8.0% test 7.2% (n=2853+906); regret 15.9%";
 }  // namespace ttlg

@@ -972,13 +972,20 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // ranking stage: boosted trees over the kGbtTopK best
   int win = order[0];
   double win_t = 1e300;
+  ModelInput rk[kGbtTopK];
+  int rid[kGbtTopK], nrk = 0;
+  double rt[kGbtTopK];
   for (int i = 0; i < std::min(ntop, kGbtTopK); i++) {
     const Entry &e = pool[order[i]];
     if (e.lin >= 1e299) continue;
-    const double t = predict_ranked_seconds(e.mi, dev);
-    if (t < win_t) {
-      win_t = t;
-      win = order[i];
+    rk[nrk] = e.mi;
+    rid[nrk++] = order[i];
+  }
+  predict_ranked_batch(rk, nrk, dev, rt);
+  for (int i = 0; i < nrk; i++) {
+    if (rt[i] < win_t) {
+      win_t = rt[i];
+      win = rid[i];
     }
   }
   if (sink && sink->shortlist) {

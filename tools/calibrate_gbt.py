@@ -110,18 +110,25 @@ def main():
     if not args.write:
         return
     m = fit(rows)  # final model on all configurations
-    feats, thr, left, right, val, roots = [], [], [], [], [], []
+    # packed preorder layout: node i's left child is i + 1, `right` is absolute;
+    # a leaf has feat -1 and carries its (learning-rate scaled) value in thr
+    nodes, roots = [], []
     for est in m.estimators_[:, 0]:
         t = est.tree_
-        base = len(feats)
-        roots.append(base)
-        for i in range(t.node_count):
-            leaf = t.children_left[i] == -1
-            feats.append(-1 if leaf else int(t.feature[i]))
-            thr.append(float(t.threshold[i]) if not leaf else 0.0)
-            left.append(-1 if leaf else base + int(t.children_left[i]))
-            right.append(-1 if leaf else base + int(t.children_right[i]))
-            val.append(float(t.value[i][0][0]) * m.learning_rate)
+        roots.append(len(nodes))
+
+        def emit(i):
+            me = len(nodes)
+            if t.children_left[i] == -1:
+                nodes.append([-1, float(t.value[i][0][0]) * m.learning_rate, -1])
+                return
+            nodes.append([int(t.feature[i]), float(t.threshold[i]), -1])
+            emit(t.children_left[i])
+            nodes[me][2] = len(nodes)
+            emit(t.children_right[i])
+
+        emit(0)
+    assert len(nodes) < 2 ** 31
     init = float(m.init_.constant_[0][0]) if hasattr(m.init_, "constant_") else float(
         np.mean([math.log(r["meas"] / ideal(r)) for r in rows]))
     with open(os.path.join(CSRC, "model_gbt.h"), "w") as f:
@@ -129,19 +136,20 @@ def main():
                 "// predicting log(time / one-pass ideal) from model_descriptor() (model.cpp).\n"
                 f"// Fitted on {len(rows)} B200 measurements ({len(cases)} configurations); held-out\n"
                 f"// 20%: selection regret {te[0]:.1f}%, mean |a-p|/a {te[1]:.1f}% (top-{TOPK} lists).\n"
-                "#pragma once\n#include <stdint.h>\nnamespace ttlg {\n")
+                "// Nodes in preorder: left child = next node, `r` = right child, f < 0 = leaf\n"
+                "// whose value is `t`.\n"
+                "#pragma once\n#include <stdint.h>\nnamespace ttlg {\n"
+                "struct GbtNode {\n  float t;\n  int16_t f;\n  int16_t pad;\n  int32_t r;\n};\n")
         f.write(f"constexpr int kGbtTrees = {len(roots)};\nconstexpr int kGbtTopK = {TOPK};\n")
         f.write(f"constexpr double kGbtInit = {init!r};\n")
         f.write(f'constexpr const char *kGbtSource = "GBT {len(roots)} trees depth {args.depth}, '
                 f'{len(rows)} points / {len(cases)} cases; test regret {te[0]:.1f}%, '
                 f'err {te[1]:.1f}%";\n')
         f.write("constexpr int32_t kGbtRoot[] = {" + ",".join(map(str, roots)) + "};\n")
-        f.write("constexpr int8_t kGbtFeat[] = {" + ",".join(map(str, feats)) + "};\n")
-        f.write("constexpr float kGbtThr[] = {" + ",".join(f"{x!r}f" for x in thr) + "};\n")
-        f.write("constexpr int16_t kGbtLeft[] = {" + ",".join(map(str, left)) + "};\n")
-        f.write("constexpr int16_t kGbtRight[] = {" + ",".join(map(str, right)) + "};\n")
-        f.write("constexpr float kGbtVal[] = {" + ",".join(f"{x!r}f" for x in val) + "};\n")
+        f.write("constexpr GbtNode kGbtNodes[] = {\n" + ",\n".join(
+            f"{{{x[1]!r}f,{x[0]},0,{x[2]}}}" for x in nodes) + "};\n")
         f.write("}  // namespace ttlg\n")
+    feats = nodes
     print("wrote", os.path.join(CSRC, "model_gbt.h"), len(feats), "nodes")
 
 
