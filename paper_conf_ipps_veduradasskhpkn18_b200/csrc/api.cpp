@@ -82,10 +82,13 @@ static int current_device() {
   return dev;
 }
 
+constexpr double kFastPlanSeconds = 150e-6;
+
 static ttlg_status plan_into(ttlg_plan_s *p, ttlg_dtype dt, int rank, const int64_t *ext,
-                             const int32_t *perm, const ttlg_plan_hints *hints) {
+                             const int32_t *perm, const ttlg_plan_hints *hints,
+                             bool fast = false) {
   const int dev = current_device();
-  ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev));
+  ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev), nullptr, fast);
   if (st != TTLG_OK) return st;
   p->device = dev;
   p->dt = dt;
@@ -327,7 +330,15 @@ ttlg_status ttlg_plan_destroy(ttlg_plan_t plan) {
 ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, const int32_t *perm,
                            const void *A, void *B, void *stream) {
   ttlg_plan_s p;  // single use: no heap, no cache
-  ttlg_status st = plan_into(&p, dt, rank, extents, perm, nullptr);
+  // the plan must hide behind the previous launch: when one pass over the
+  // data is short (< kFastPlanSeconds at the profile's copy bandwidth) use the
+  // fast effort level
+  ttlg_status st = validate(dt, rank, extents, perm);
+  if (st != TTLG_OK) return st;
+  double bytes = 2.0 * (dt == TTLG_F64 ? 8 : 4);
+  for (int k = 0; k < rank; k++) bytes *= (double)extents[k];
+  const bool fast = bytes / (device_profile(current_device()).hbm_gbs * 1e9) < kFastPlanSeconds;
+  st = plan_into(&p, dt, rank, extents, perm, nullptr, fast);
   if (st != TTLG_OK) return st;
   return execute(&p, A, B, stream);
 }

@@ -148,20 +148,25 @@ double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 // (tree-major) lets the core overlap their dependent node loads.
 void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
   constexpr int kB = 32;
-  double d[kB][kGbtDesc], s[kB];
+  constexpr int NI = (1 << kGbtDepth) - 1;
+  float d[kB][kGbtDesc];
+  double s[kB];
   for (int b0 = 0; b0 < n; b0 += kB) {
     const int m = std::min(kB, n - b0);
     for (int c = 0; c < m; c++) {
-      model_descriptor(mis[b0 + c], dev, d[c]);
+      double dd[kGbtDesc];
+      model_descriptor(mis[b0 + c], dev, dd);
+      for (int k = 0; k < kGbtDesc; k++) d[c][k] = (float)dd[k];  // sklearn splits on float32
       s[c] = kGbtInit;
     }
     for (int t = 0; t < kGbtTrees; t++) {
-      const int root = kGbtRoot[t];
+      const int8_t *F = kGbtF[t];
+      const float *T = kGbtT[t];
       for (int c = 0; c < m; c++) {
-        int k = root;
-        while (kGbtNodes[k].f >= 0)
-          k = (d[c][kGbtNodes[k].f] <= (double)kGbtNodes[k].t) ? k + 1 : kGbtNodes[k].r;
-        s[c] += kGbtNodes[k].t;
+        int i = 0;
+#pragma GCC unroll 8
+        for (int l = 0; l < kGbtDepth; l++) i = 2 * i + 1 + (d[c][F[i]] > T[i]);
+        s[c] += kGbtV[t][i - NI];
       }
     }
     for (int c = 0; c < m; c++) {

@@ -619,7 +619,7 @@ static void fill_info(ttlg_plan_info &I, ttlg_dtype dt, int rank, const Problem 
 
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints,
-                      const DeviceProfile &dev, CandidateSink *sink) {
+                      const DeviceProfile &dev, CandidateSink *sink, bool fast) {
   ttlg_status st = validate(dt, rank, ext, perm);
   if (st != TTLG_OK) return st;
   const int s = (dt == TTLG_F64) ? 8 : 4;
@@ -727,7 +727,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       return true;
     }
     smem_conflicts(K0, P.W, cl, cs);
-    if (cl + cs > 2.0) {
+    // padding input-run dims (XT) only separates output-run digits that live
+    // in the input run, i.e. overlapping groups (OA/FMS); OD tiles skip the search
+    bool overlap = false;
+    for (int i = 0; i <= T.b; i++) overlap |= P.p[i] <= T.a;
+    if (overlap && cl + cs > 2.0) {
       const int lp = 128 / P.W;
       const int opts[6] = {1, 2, 3, lp / 2, lp / 2 + 1, lp - 1};
       for (int k = 1; k <= T.a && cl + cs > 2.0; k++) {
@@ -756,6 +760,29 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
 
   auto insert = [&](double lin, const ModelInput &mi, const Tile &T, int kind, int schema,
                     int tpc, int group, const int *delta) {
+    // different (a, ta, b, tb) can describe the same tile box: keep one entry
+    // per (box, kernel, block size) so the short list stays diverse
+    for (int i = 0; i < ntop; i++) {
+      const Entry &o = pool[i];
+      if (o.kind != kind || o.mi.threads != mi.threads) continue;
+      bool same = true;
+      for (int k = 0; k < P.d && same; k++) same = o.T.t[k] == T.t[k];
+      if (same) {
+        if (lin < o.lin) {  // same box, better score: replace in place and re-sort
+          Entry &e = pool[i];
+          e.lin = lin;
+          e.mi = mi;
+          e.T = T;
+          e.schema = schema;
+          e.tpc = tpc;
+          e.group = group;
+          for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
+          std::sort(order, order + ntop, [&](int x, int y) { return pool[x].lin < pool[y].lin; });
+          if (ntop == kShort) admit = pool[order[kShort - 1]].lin;
+        }
+        return;
+      }
+    }
     int slot, pos;
     if (ntop < kShort) {
       slot = ntop;
@@ -937,8 +964,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     };
     Done done[kShort];
     int nd = 0;
-    for (int i = 0; i < ntop; i++) {
-      Entry &e = pool[i];
+    // fast planning (single-use calls on small tensors): refine only the
+    // linear screen's best few; the rest drop out
+    const int nref = fast ? std::min(ntop, kFastRefine) : ntop;
+    for (int i = nref; i < ntop; i++) pool[order[i]].lin = 1e300;
+    for (int ii = 0; ii < nref; ii++) {
+      Entry &e = pool[order[ii]];
       const int64_t ta = e.T.t[e.T.a], tb = e.T.t[P.p[e.T.b]];
       int f = -1;
       for (int j = 0; j < nd && f < 0; j++)
@@ -975,7 +1006,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   ModelInput rk[kGbtTopK];
   int rid[kGbtTopK], nrk = 0;
   double rt[kGbtTopK];
-  for (int i = 0; i < std::min(ntop, kGbtTopK); i++) {
+  const int topk = fast ? kFastTopK : kGbtTopK;
+  for (int i = 0; i < std::min(ntop, topk); i++) {
     const Entry &e = pool[order[i]];
     if (e.lin >= 1e299) continue;
     rk[nrk] = e.mi;

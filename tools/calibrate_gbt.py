@@ -91,7 +91,11 @@ def main():
     def evaluate(m, cs):
         reg, err, gp, gb = [], [], [], []
         for c in cs:
-            rs = sorted(by[c], key=lambda r: r["lin"])[:TOPK]
+            # the planner's short list holds one entry per (tile box, kernel, block size)
+            uniq = {}
+            for r in sorted(by[c], key=lambda r: r["lin"]):
+                uniq.setdefault((tuple(r["tile"]), r["kernel"], r["threads"]), r)
+            rs = list(uniq.values())[:TOPK]
             P = m.predict(np.array([desc(r) for r in rs]))
             best = min(by[c], key=lambda r: r["meas"])
             pick = rs[int(np.argmin(P))]
@@ -110,47 +114,65 @@ def main():
     if not args.write:
         return
     m = fit(rows)  # final model on all configurations
-    # packed preorder layout: node i's left child is i + 1, `right` is absolute;
-    # a leaf has feat -1 and carries its (learning-rate scaled) value in thr
-    nodes, roots = [], []
+    # complete binary trees of depth D in implicit layout (node i -> children
+    # 2i+1, 2i+2): shallower sklearn leaves are padded with always-left dummy
+    # splits (feature 0, threshold +inf) so traversal is D branch-free steps
+    D = args.depth
+    NI, NL = 2 ** D - 1, 2 ** D
+    F, T, V = [], [], []
     for est in m.estimators_[:, 0]:
         t = est.tree_
-        roots.append(len(nodes))
+        f_ = [0] * NI
+        t_ = [float("inf")] * NI
+        v_ = [0.0] * NL
 
-        def emit(i):
-            me = len(nodes)
+        def fill(i, pos, depth):
             if t.children_left[i] == -1:
-                nodes.append([-1, float(t.value[i][0][0]) * m.learning_rate, -1])
+                val = float(t.value[i][0][0]) * m.learning_rate
+                lo, hi = pos, pos  # leaves of the complete subtree under pos
+                while lo < NI:
+                    lo, hi = 2 * lo + 1, 2 * hi + 2
+                for q in range(lo, hi + 1):
+                    v_[q - NI] = val
                 return
-            nodes.append([int(t.feature[i]), float(t.threshold[i]), -1])
-            emit(t.children_left[i])
-            nodes[me][2] = len(nodes)
-            emit(t.children_right[i])
+            assert depth < D
+            f_[pos] = int(t.feature[i])
+            t_[pos] = float(t.threshold[i])
+            fill(t.children_left[i], 2 * pos + 1, depth + 1)
+            fill(t.children_right[i], 2 * pos + 2, depth + 1)
 
-        emit(0)
-    assert len(nodes) < 2 ** 31
+        fill(0, 0, 0)
+        F.append(f_)
+        T.append(t_)
+        V.append(v_)
     init = float(m.init_.constant_[0][0]) if hasattr(m.init_, "constant_") else float(
         np.mean([math.log(r["meas"] / ideal(r)) for r in rows]))
+
+    def flt(x):
+        return "INFINITY" if x == float("inf") else f"{x!r}f"
+
     with open(os.path.join(CSRC, "model_gbt.h"), "w") as f:
         f.write("// model_gbt.h -- GENERATED by tools/calibrate_gbt.py: boosted regression trees\n"
                 "// predicting log(time / one-pass ideal) from model_descriptor() (model.cpp).\n"
                 f"// Fitted on {len(rows)} B200 measurements ({len(cases)} configurations); held-out\n"
                 f"// 20%: selection regret {te[0]:.1f}%, mean |a-p|/a {te[1]:.1f}% (top-{TOPK} lists).\n"
-                "// Nodes in preorder: left child = next node, `r` = right child, f < 0 = leaf\n"
-                "// whose value is `t`.\n"
-                "#pragma once\n#include <stdint.h>\nnamespace ttlg {\n"
-                "struct GbtNode {\n  float t;\n  int16_t f;\n  int16_t pad;\n  int32_t r;\n};\n")
-        f.write(f"constexpr int kGbtTrees = {len(roots)};\nconstexpr int kGbtTopK = {TOPK};\n")
+                f"// Complete trees of depth {D}: node i has children 2i+1 (x <= t) and 2i+2.\n"
+                "#pragma once\n#include <math.h>\n#include <stdint.h>\nnamespace ttlg {\n")
+        f.write(f"constexpr int kGbtTrees = {len(F)};\nconstexpr int kGbtDepth = {D};\n"
+                f"constexpr int kGbtTopK = {TOPK};\n")
         f.write(f"constexpr double kGbtInit = {init!r};\n")
-        f.write(f'constexpr const char *kGbtSource = "GBT {len(roots)} trees depth {args.depth}, '
+        f.write(f'constexpr const char *kGbtSource = "GBT {len(F)} trees depth {D}, '
                 f'{len(rows)} points / {len(cases)} cases; test regret {te[0]:.1f}%, '
                 f'err {te[1]:.1f}%";\n')
-        f.write("constexpr int32_t kGbtRoot[] = {" + ",".join(map(str, roots)) + "};\n")
-        f.write("constexpr GbtNode kGbtNodes[] = {\n" + ",\n".join(
-            f"{{{x[1]!r}f,{x[0]},0,{x[2]}}}" for x in nodes) + "};\n")
+        f.write(f"constexpr int8_t kGbtF[{len(F)}][{NI}] = {{\n" +
+                ",\n".join("{" + ",".join(map(str, r)) + "}" for r in F) + "};\n")
+        f.write(f"constexpr float kGbtT[{len(F)}][{NI}] = {{\n" +
+                ",\n".join("{" + ",".join(flt(x) for x in r) + "}" for r in T) + "};\n")
+        f.write(f"constexpr float kGbtV[{len(F)}][{NL}] = {{\n" +
+                ",\n".join("{" + ",".join(flt(x) for x in r) + "}" for r in V) + "};\n")
         f.write("}  // namespace ttlg\n")
-    feats = nodes
-    print("wrote", os.path.join(CSRC, "model_gbt.h"), len(feats), "nodes")
+    feats = F
+    print("wrote", os.path.join(CSRC, "model_gbt.h"), len(feats), "trees")
 
 
 if __name__ == "__main__":
