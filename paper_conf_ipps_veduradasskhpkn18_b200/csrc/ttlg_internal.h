@@ -162,7 +162,7 @@ constexpr int kModelFeatureCount = 10;
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
 // fast = the single-use effort level: refine the linear screen's best
 // kFastRefine candidates and rank kFastTopK of them with the trees
-constexpr int kFastRefine = 8, kFastTopK = 4;
+constexpr int kFastRefine = 12, kFastTopK = 8;
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev,
                       CandidateSink *sink = nullptr, bool fast = false);
