@@ -8,7 +8,9 @@ import os
 
 MAX_RANK = 15
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libttlg.so")
+# TTLG_LIB: development override (A/B builds of the same sources); the
+# product loads the in-tree build
+LIB_PATH = os.environ.get("TTLG_LIB") or os.path.join(_PKG, "libttlg.so")
 
 F32, F64 = 0, 1
 SCHEMA_AUTO, SCHEMA_COPY, SCHEMA_FML, SCHEMA_FMS, SCHEMA_OD, SCHEMA_OA = -1, 0, 1, 2, 3, 4

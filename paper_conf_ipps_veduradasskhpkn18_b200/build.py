@@ -24,14 +24,16 @@ def _stale() -> bool:
     return any(os.path.getmtime(p) > t for p in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not _stale():
+def build(force: bool = False, verbose: bool = False, out: str = None, defines=()) -> str:
+    """Build libttlg.so (or, for A/B experiments, `out` with extra -D defines)."""
+    if out is None and not force and not _stale():
         return LIB
     cmd = [NVCC, "-O3", "-std=c++17", "-lineinfo", *ARCH, "-shared", "-Xcompiler", "-fPIC",
            "-Xcompiler", "-Wall", "-cudart", "shared", "-Xptxas", "-v" if verbose else "-O3",
            "-I", os.path.join(ROOT, "include"),
            "-Xlinker", "-rpath,/usr/local/cuda/lib64",
-           "-o", LIB + ".tmp"]
+           *[f"-D{d}" for d in defines],
+           "-o", (out or LIB) + ".tmp"]
     cmd += [os.path.join(CSRC, s) for s in SOURCES]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
@@ -39,8 +41,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc build of libttlg.so failed")
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(LIB + ".tmp", LIB)
-    return LIB
+    os.replace((out or LIB) + ".tmp", out or LIB)
+    return out or LIB
 
 
 if __name__ == "__main__":

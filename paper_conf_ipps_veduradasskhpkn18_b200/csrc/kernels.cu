@@ -40,6 +40,16 @@
 #ifndef TTLG_CP16_CG
 #define TTLG_CP16_CG 0
 #endif
+// store cache policy of the staged kernels: "cs" (evict-first streaming,
+// default) or "wb" (-DTTLG_ST_WB=1, plain write-back)
+#ifndef TTLG_ST_WB
+#define TTLG_ST_WB 0
+#endif
+#if TTLG_ST_WB
+#define TTLG_STP "st.global"
+#else
+#define TTLG_STP "st.global.cs"
+#endif
 
 namespace ttlg {
 
@@ -67,7 +77,7 @@ __device__ __forceinline__ T ld_stream(const T *p) {
 }
 template <bool CS, typename T>
 __device__ __forceinline__ void st_stream(T *p, T v) {
-  if constexpr (CS)
+  if constexpr (CS && !TTLG_ST_WB)
     __stcs(p, v);
   else
     *p = v;
@@ -98,17 +108,17 @@ __device__ __forceinline__ void cp_async_p(uint32_t s, const void *gptr, bool p)
                  "l"(gptr), "r"((int)p), "n"(W));
 }
 __device__ __forceinline__ void stcs_p(unsigned int *a, unsigned int v, bool p) {
-  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q st.global.cs.u32 [%0], %1;\n}\n"
+  asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %2, 0;\n @q " TTLG_STP ".u32 [%0], %1;\n}\n"
                ::"l"(a), "r"(v), "r"((int)p) : "memory");
 }
 __device__ __forceinline__ void stcs_p(uint2 *a, uint2 v, bool p) {
   asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %3, 0;\n"
-               " @q st.global.cs.v2.u32 [%0], {%1, %2};\n}\n"
+               " @q " TTLG_STP ".v2.u32 [%0], {%1, %2};\n}\n"
                ::"l"(a), "r"(v.x), "r"(v.y), "r"((int)p) : "memory");
 }
 __device__ __forceinline__ void stcs_p(uint4 *a, uint4 v, bool p) {
   asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %5, 0;\n"
-               " @q st.global.cs.v4.u32 [%0], {%1, %2, %3, %4};\n}\n"
+               " @q " TTLG_STP ".v4.u32 [%0], {%1, %2, %3, %4};\n}\n"
                ::"l"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"((int)p) : "memory");
 }
 __device__ __forceinline__ void cp_async_commit() {
