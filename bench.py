@@ -180,6 +180,128 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def run_sharded(args, rank, world, local_rank, dev):
+    """--workload sharded: BASELINE config 5, the 8 GiB rank-5 fp32 tensor
+    [64,64,64,64,128] sharded on A's outermost dim across the ranks (one
+    process per GPU).  No-move perms: one local transposition per rank, no
+    communication.  Moved perms: the fused exchange (sub-transpositions storing
+    into the peers' B slabs over CUDA IPC / NVLink) and, for comparison, local
+    transpose -> NCCL all_to_all_single -> fold.  Also, on rank 0: the fused
+    exchange of P = 2/4/8 emulated on this one GPU (every peer slab local) --
+    the HBM-side cost of its sub-box launches."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_veduradasskhpkn18_b200.sharded import (
+        plan_shards, P2PExchange, map_peer_slabs, unmap_peer_slabs, sharded_transpose)
+    from synth import configs, gen_tensor_torch, case_seed
+
+    cases = configs.config5()
+    ext = list(cases[0].extents)
+    n = 1
+    for e in ext:
+        n *= e
+    n_local = n // world
+    stream = torch.cuda.Stream(device=dev)
+    sptr = stream.cuda_stream
+    A = gen_tensor_torch(case_seed(5000), n_local, 4, device=dev, start=rank * n_local)
+    B = torch.empty_like(A)
+    if world > 1:
+        peers, opened = map_peer_slabs(B)
+    else:
+        peers, opened = [B.data_ptr()], []
+    work = (torch.empty_like(A), torch.empty_like(A)) if world > 1 else None
+    exs = [P2PExchange(ext, c.perm, B, peer_ptrs=peers, rank=rank, world=world) for c in cases]
+    torch.cuda.synchronize()
+
+    def timed(fn, steps):
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(steps):
+            fn()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = e0.elapsed_time(e1)
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+            dist.barrier()
+        return ms
+
+    per, a2a = [], {}
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    time.sleep(0.3)
+    for c, ex in zip(cases, exs):
+        def f_p2p(ex=ex):
+            ex.run(A, sptr)
+        for _ in range(args.warmup):
+            f_p2p()
+        ms = timed(f_p2p, args.steps)
+        per.append(ms)
+        if world > 1 and ex.sp.moved:
+            def f_a2a(c=c):
+                with torch.cuda.stream(stream):
+                    sharded_transpose(A, ext, c.perm, work=work)
+            for _ in range(args.warmup):
+                f_a2a()
+            a2a["".join(map(str, c.perm))] = 2 * n * 4 * args.steps / (
+                timed(f_a2a, args.steps) / 1e3) / 1e9
+    clk = clocks.stop()
+    total_ms = sum(per)
+    value = 2 * n * 4 * len(cases) * args.steps / (total_ms / 1e3) / 1e9
+
+    emulated = {}
+    if rank == 0 and world == 1 and not args.no_emulate:
+        # the fused exchange at P = 2/4/8 with every peer slab on this GPU
+        Af = A  # world == 1: A is the whole tensor
+        for P in (2, 4, 8):
+            slabs = [B[q * (n // P):(q + 1) * (n // P)] for q in range(P)]
+            ptrs = [t.data_ptr() for t in slabs]
+            for c in cases:
+                sp = plan_shards(ext, c.perm, P)
+                if not sp.moved:
+                    continue
+                rexs = [P2PExchange(ext, c.perm, slabs[p], peer_ptrs=ptrs, rank=p, world=P)
+                        for p in range(P)]
+
+                def f_all(rexs=rexs, P=P):
+                    for p, ex in enumerate(rexs):
+                        ex.run(Af[p * (n // P):(p + 1) * (n // P)], sptr)
+                for _ in range(2):
+                    f_all()
+                ms = timed(f_all, max(2, args.steps // 2))
+                emulated[f"P{P}:{''.join(map(str, c.perm))}"] = \
+                    2 * n * 4 * max(2, args.steps // 2) / (ms / 1e3) / 1e9
+    for ex in exs:
+        ex.close()
+    unmap_peer_slabs(opened)
+    if rank == 0:
+        peak, peak_src, _ = _peaks()
+        line = {
+            "metric": "effective transpose GB/s (2*N*s/time)", "value": value, "unit": "GB/s",
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": total_ms / args.steps, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic (SplitMix64 bit patterns, generated on device)",
+            "config": {"workload": "c5-8GiB-rank5-fp32 sharded on A's outermost dim (BASELINE config 5)",
+                       "extents": ext, "perms": [list(c.perm) for c in cases],
+                       "parallelism": f"shard x{world}", "exchange": "fused p2p (CUDA IPC stores)",
+                       "l2": "no flush: 8 GiB tensors (inputs larger than L2)"},
+            "gpu_launches": sum(len(ex.subs) for ex in exs) * args.steps,
+            "per_perm_gbs": {"".join(map(str, c.perm)): 2 * n * 4 * args.steps / (m / 1e3) / 1e9
+                             for c, m in zip(cases, per)},
+            "alltoall_path_gbs": a2a or None,
+            "p2p_emulated_one_gpu_gbs": emulated or None,
+            "frac_of_peak": value / world / peak,
+            "clocks": clk,
+        }
+        print(json.dumps(line), flush=True)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -191,6 +313,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--ref-cases-per-step", type=int, default=6)
+    ap.add_argument("--no-emulate", action="store_true",
+                    help="sharded workload: skip the one-GPU emulation of P = 2/4/8")
     ap.add_argument("--tune", type=int, default=8,
                     help="measure-mode candidates per case for the 'tuned' key (0 = off)")
     args = ap.parse_args()
@@ -215,6 +339,11 @@ def main():
     import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
     from synth import gen_tensor_torch, case_seed
 
+    if args.workload == "sharded":
+        run_sharded(args, rank, world, local_rank, dev)
+        if world > 1:
+            dist.destroy_process_group()
+        return
     name, cases = _workload(args.workload)
     peak, peak_src, peaks = _peaks()
     stream = torch.cuda.Stream(device=dev)

@@ -133,6 +133,27 @@ ttlg_status ttlg_plan(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *
 ttlg_status ttlg_plan_ex(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
                          const int32_t *perm, const ttlg_plan_hints *hints);
 
+/* Sub-tensor transposition (the general strided form; used by the fused
+ * sharded exchange): the same operation as ttlg_plan on
+ * extents/perm, but element (i0..i_{d-1}) is read from
+ *     A + sum_k i_k * in_strides[k]
+ * and written to
+ *     B + sum_i o_i * out_strides[i],   o_i = i_{perm[i]},
+ * strides in ELEMENTS (in_strides per input dim, out_strides per output dim;
+ * either may be NULL = dense, which is exactly ttlg_plan_ex).  Extent-1 dims
+ * ignore their stride.  Requirements: every stride of a non-unit dim >= 1; the
+ * fastest non-unit dim of A has in_stride 1 and the first non-unit output dim
+ * has out_stride 1 (else TTLG_ERR_UNSUPPORTED: the kernels move contiguous
+ * runs along both FVIs); B must be injective -- sorted by stride, each output
+ * dim's stride >= the previous stride x extent (else TTLG_ERR_INVALID_VALUE).
+ * Index fusion (L666-685) joins two dims only where both tensors are dense
+ * across them.  Aliasing is checked on the spanned byte ranges
+ * [A, A + s*(1 + sum (n_k-1)*in_strides[k])) and likewise for B.
+ * ttlg_execute_host rejects strided plans (TTLG_ERR_UNSUPPORTED). */
+ttlg_status ttlg_plan_strided(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                              const int32_t *perm, const int64_t *in_strides,
+                              const int64_t *out_strides, const ttlg_plan_hints *hints);
+
 /* Repeated-use execution: one asynchronous kernel launch on `stream`
  * (a cudaStream_t; NULL = legacy default stream).  A and B are device
  * pointers, element-aligned, non-overlapping. */
@@ -181,6 +202,23 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
 ttlg_status ttlg_plan_candidates(ttlg_dtype dt, int rank, const int64_t *extents,
                                  const int32_t *perm, const ttlg_plan_hints *hints,
                                  ttlg_plan_info *out, int32_t max_out, int32_t *n_out);
+
+/* Peer memory for the fused sharded exchange (not in the
+ * paper): rank p's sub-tensor transpositions store straight into the B slabs
+ * of the other ranks over NVLink/NVSwitch (CUDA IPC mappings; every rank runs
+ * one process per GPU, PyTorch supplies the process group that moves the
+ * handles).
+ *   ttlg_ipc_export: handle (TTLG_IPC_HANDLE_BYTES bytes, caller-owned) of the
+ *     device allocation containing `ptr`, and ptr's byte offset in it;
+ *   ttlg_ipc_open: map another process's allocation on the current device
+ *     (peer access enabled lazily); *ptr = mapped base + offset;
+ *   ttlg_ipc_close: unmap (pass the pointer and offset ttlg_ipc_open used).
+ * Errors: TTLG_ERR_INVALID_VALUE for null arguments, TTLG_ERR_CUDA when the
+ * runtime refuses (e.g. handle opened in the exporting process itself). */
+#define TTLG_IPC_HANDLE_BYTES 64
+ttlg_status ttlg_ipc_export(const void *ptr, void *handle, int64_t *offset);
+ttlg_status ttlg_ipc_open(const void *handle, int64_t offset, void **ptr);
+ttlg_status ttlg_ipc_close(void *ptr, int64_t offset);
 
 const char *ttlg_status_string(ttlg_status s);
 const char *ttlg_schema_name(int schema);

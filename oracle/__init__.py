@@ -53,6 +53,12 @@ def _load():
                                             ctypes.POINTER(ctypes.c_int32),
                                             ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64]
         lib.oracle_source_index.restype = ctypes.c_int
+        lib.oracle_transpose_strided.argtypes = [
+            ctypes.c_int, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
+            ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int64),
+            ctypes.POINTER(ctypes.c_int64), ctypes.c_void_p, ctypes.c_int64,
+            ctypes.c_void_p, ctypes.c_int64]
+        lib.oracle_transpose_strided.restype = ctypes.c_int
         _lib = lib
     return _lib
 
@@ -84,6 +90,29 @@ def transpose(A: np.ndarray, extents: Sequence[int], perm: Sequence[int],
     ext, pr = _arrs(extents, perm)
     rc = _load().oracle_transpose(A.dtype.itemsize, len(extents), ext, pr,
                                   A.ctypes.data, B.ctypes.data, int(threads))
+    if rc != 0:
+        raise ValueError("oracle: invalid rank/extents/perm")
+    return B
+
+
+def transpose_strided(A: np.ndarray, B: np.ndarray, extents: Sequence[int],
+                      perm: Sequence[int], in_strides: Sequence[int],
+                      out_strides: Sequence[int], a_off: int = 0, b_off: int = 0) -> np.ndarray:
+    """Sub-tensor transposition into B in place (only the addressed positions
+    change): B[b_off + sum_i o_i out_strides[i]] = A[a_off + sum_k i_k in_strides[k]],
+    o_i = i_{perm[i]}.  A, B: flat contiguous arrays of the same item size."""
+    if not (A.flags.c_contiguous and B.flags.c_contiguous) or A.dtype.itemsize != B.dtype.itemsize:
+        raise ValueError("A and B must be contiguous with the same element size")
+    d = len(extents)
+    span_a = a_off + sum((int(e) - 1) * int(s) for e, s in zip(extents, in_strides))
+    span_b = b_off + sum((int(extents[p]) - 1) * int(s) for p, s in zip(perm, out_strides))
+    if span_a >= A.size or span_b >= B.size or a_off < 0 or b_off < 0:
+        raise ValueError("strided box exceeds the buffers")
+    ext, pr = _arrs(extents, perm)
+    sa = (ctypes.c_int64 * d)(*[int(x) for x in in_strides])
+    sb = (ctypes.c_int64 * d)(*[int(x) for x in out_strides])
+    rc = _load().oracle_transpose_strided(A.dtype.itemsize, d, ext, pr, sa, sb, A.ctypes.data,
+                                          int(a_off), B.ctypes.data, int(b_off))
     if rc != 0:
         raise ValueError("oracle: invalid rank/extents/perm")
     return B

@@ -133,6 +133,28 @@ int oracle_transpose(int elem_bytes, int rank, const int64_t *extents,
     return 0;
 }
 
+/* The sub-tensor form (the library's ttlg_plan_strided; used by the fused
+ * sharded exchange): the same d-nested loop with given strides (elements),
+ * lin_A = a_off + sum_k i_k in_strides[k], lin_B = b_off + sum_i
+ * i_{perm[i]} out_strides[i].  Writes only the addressed positions of B. */
+int oracle_transpose_strided(int elem_bytes, int rank, const int64_t *extents,
+                             const int32_t *perm, const int64_t *in_strides,
+                             const int64_t *out_strides, const void *A, int64_t a_off,
+                             void *B, int64_t b_off) {
+    job_t j;
+    if (setup(&j, elem_bytes, rank, extents, perm)) return 1;
+    for (int k = 0; k < rank; k++) {
+        j.sA[k] = in_strides[k];
+        j.sB[k] = out_strides[k];
+    }
+    j.A = (const char *)A + a_off * elem_bytes;
+    j.B = (char *)B + b_off * elem_bytes;
+    j.lo = 0;
+    j.hi = j.n[rank - 1];
+    run(&j);
+    return 0;
+}
+
 /* The same definition read backwards, for sampled checks at sizes the full
  * loop cannot hold: for each output linear index lin_B, decode the output
  * multi-index o (o_0 fastest, extents m[i] = n[perm[i]]), set

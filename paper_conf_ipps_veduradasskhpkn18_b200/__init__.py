@@ -5,9 +5,9 @@ Public surface (same names as the C ABI in include/ttlg.h):
 plus `sharded` (multi-GPU slab / all-to-all driver over torch.distributed).
 """
 from .api import (Plan, plan, execute, transpose, predict_time, transpose_tensor, torch_to_c,
-                  make_hints, model_source, plan_candidates, candidate_hints)
+                  make_hints, model_source, plan_candidates, candidate_hints, plan_strided)
 from ._ffi import TtlgError, F32, F64, SCHEMA_NAMES, LIB_PATH
 
 __all__ = ["Plan", "plan", "execute", "transpose", "predict_time", "transpose_tensor",
-           "torch_to_c", "make_hints", "model_source", "plan_candidates", "candidate_hints", "TtlgError", "F32", "F64",
+           "torch_to_c", "make_hints", "model_source", "plan_candidates", "candidate_hints", "plan_strided", "TtlgError", "F32", "F64",
            "SCHEMA_NAMES", "LIB_PATH"]

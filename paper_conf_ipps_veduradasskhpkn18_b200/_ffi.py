@@ -25,7 +25,9 @@ STATUS = {0: "TTLG_OK", 1: "TTLG_ERR_INVALID_VALUE", 2: "TTLG_ERR_ALIASING",
 EXPORTS = ["ttlg_plan", "ttlg_plan_ex", "ttlg_plan_hints_init", "ttlg_execute",
            "ttlg_plan_destroy", "ttlg_transpose", "ttlg_execute_host", "ttlg_predict_time",
            "ttlg_plan_describe", "ttlg_status_string", "ttlg_schema_name", "ttlg_version",
-           "ttlg_model_source", "ttlg_plan_candidates", "ttlg_plan_tune"]
+           "ttlg_model_source", "ttlg_plan_candidates", "ttlg_plan_tune", "ttlg_plan_strided",
+           "ttlg_ipc_export", "ttlg_ipc_open", "ttlg_ipc_close"]
+IPC_HANDLE_BYTES = 64
 
 
 class TtlgError(RuntimeError):
@@ -94,6 +96,11 @@ def _load():
         "ttlg_plan_ex": ([ctypes.POINTER(P), ctypes.c_int, ctypes.c_int, i64p, i32p,
                           ctypes.POINTER(PlanHints)], ctypes.c_int),
         "ttlg_plan_hints_init": ([ctypes.POINTER(PlanHints)], None),
+        "ttlg_plan_strided": ([ctypes.POINTER(P), ctypes.c_int, ctypes.c_int, i64p, i32p, i64p,
+                               i64p, ctypes.POINTER(PlanHints)], ctypes.c_int),
+        "ttlg_ipc_export": ([P, ctypes.c_char_p, i64p], ctypes.c_int),
+        "ttlg_ipc_open": ([ctypes.c_char_p, ctypes.c_int64, ctypes.POINTER(P)], ctypes.c_int),
+        "ttlg_ipc_close": ([P, ctypes.c_int64], ctypes.c_int),
         "ttlg_execute": ([P, P, P, P], ctypes.c_int),
         "ttlg_plan_destroy": ([P], ctypes.c_int),
         "ttlg_transpose": ([ctypes.c_int, ctypes.c_int, i64p, i32p, P, P, P], ctypes.c_int),

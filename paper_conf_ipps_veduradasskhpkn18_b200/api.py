@@ -59,13 +59,30 @@ def make_hints(schema=None, in_dim=None, in_block=None, out_dim=None, out_block=
 class Plan:
     """A ttlg_plan_t (repeated-use mode)."""
 
-    def __init__(self, dtype, extents: Sequence[int], perm: Sequence[int], **hints):
+    def __init__(self, dtype, extents: Sequence[int], perm: Sequence[int],
+                 in_strides: Optional[Sequence[int]] = None,
+                 out_strides: Optional[Sequence[int]] = None, **hints):
         self._h = ctypes.c_void_p()
         self.dtype = _dtype_code(dtype)
         self.extents = [int(e) for e in extents]
         self.perm = [int(p) for p in perm]
         ext, pr = arrays(self.extents, self.perm)
-        if hints:
+        if in_strides is not None or out_strides is not None:
+            # sub-tensor form (ttlg_plan_strided): strides in elements
+            d = len(self.extents)
+
+            def arr(v):
+                if v is None:
+                    return None
+                if len(v) != d:
+                    raise ValueError("strides must have one entry per dim")
+                return (ctypes.c_int64 * d)(*[int(x) for x in v])
+            hh = make_hints(**hints) if hints else None
+            check(lib.ttlg_plan_strided(ctypes.byref(self._h), self.dtype, d, ext, pr,
+                                        arr(in_strides), arr(out_strides),
+                                        ctypes.byref(hh) if hh is not None else None),
+                  "ttlg_plan_strided")
+        elif hints:
             hh = make_hints(**hints)
             check(lib.ttlg_plan_ex(ctypes.byref(self._h), self.dtype, len(self.extents), ext, pr,
                                    ctypes.byref(hh)), "ttlg_plan_ex")
@@ -114,6 +131,32 @@ class Plan:
 
 def plan(dtype, extents, perm, **hints) -> Plan:
     return Plan(dtype, extents, perm, **hints)
+
+
+def plan_strided(dtype, extents, perm, in_strides=None, out_strides=None, **hints) -> Plan:
+    """Sub-tensor transposition (ttlg_plan_strided): element strides per input
+    dim (A) and per output dim (B); None = dense."""
+    return Plan(dtype, extents, perm, in_strides=in_strides, out_strides=out_strides, **hints)
+
+
+# ---- peer memory (CUDA IPC) for the fused sharded exchange ------------------------------
+def ipc_export(ptr: int):
+    """(handle bytes, offset) of the device allocation containing ptr."""
+    h = ctypes.create_string_buffer(_ffi.IPC_HANDLE_BYTES)
+    off = ctypes.c_int64()
+    check(lib.ttlg_ipc_export(ctypes.c_void_p(ptr), h, ctypes.byref(off)), "ttlg_ipc_export")
+    return h.raw, off.value
+
+
+def ipc_open(handle: bytes, offset: int) -> int:
+    """Map another process's allocation on the current device; returns the pointer."""
+    out = ctypes.c_void_p()
+    check(lib.ttlg_ipc_open(handle, int(offset), ctypes.byref(out)), "ttlg_ipc_open")
+    return int(out.value)
+
+
+def ipc_close(ptr: int, offset: int):
+    check(lib.ttlg_ipc_close(ctypes.c_void_p(ptr), int(offset)), "ttlg_ipc_close")
 
 
 def execute(p: Plan, A_ptr: int, B_ptr: int, stream: int = 0):

@@ -86,10 +86,25 @@ constexpr double kFastPlanSeconds = 150e-6;
 
 static ttlg_status plan_into(ttlg_plan_s *p, ttlg_dtype dt, int rank, const int64_t *ext,
                              const int32_t *perm, const ttlg_plan_hints *hints,
-                             bool fast = false) {
+                             bool fast = false, const int64_t *in_strides = nullptr,
+                             const int64_t *out_strides = nullptr) {
   const int dev = current_device();
-  ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev), nullptr, fast);
+  ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev), nullptr, fast,
+                             in_strides, out_strides);
   if (st != TTLG_OK) return st;
+  p->strided = in_strides || out_strides;
+  {
+    int64_t acc = 1;
+    for (int k = 0; k < rank; k++) {
+      p->in_strides[k] = in_strides ? in_strides[k] : acc;
+      acc *= ext[k];
+    }
+    acc = 1;
+    for (int i = 0; i < rank; i++) {
+      p->out_strides[i] = out_strides ? out_strides[i] : acc;
+      acc *= ext[perm[i]];
+    }
+  }
   p->device = dev;
   p->dt = dt;
   p->rank = rank;
@@ -117,8 +132,7 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
   const int s = p->dt == TTLG_F64 ? 8 : 4;
   const uintptr_t a = (uintptr_t)A, b = (uintptr_t)B;
   if (a % s || b % s) return TTLG_ERR_INVALID_VALUE;
-  const uintptr_t nb = (uintptr_t)p->nbytes;
-  if (a < b + nb && b < a + nb) return TTLG_ERR_ALIASING;
+  if (a < b + (uintptr_t)p->spanB && b < a + (uintptr_t)p->spanA) return TTLG_ERR_ALIASING;
   if (p->device < 0) return TTLG_ERR_DEVICE;
   int dev = -1;
   if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) {
@@ -137,7 +151,9 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
     }
     h.elem_bytes_override = s;
     if (h.variant == 3) h.variant = 0;  // k_quad needs 16-byte alignment
-    ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h);
+    ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false,
+                               p->strided ? p->in_strides : nullptr,
+                               p->strided ? p->out_strides : nullptr);
     if (st != TTLG_OK) return st;
     return launch(&q, A, B, stream);
   }
@@ -313,6 +329,22 @@ ttlg_status ttlg_plan_ex(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_
   return TTLG_OK;
 }
 
+ttlg_status ttlg_plan_strided(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
+                              const int32_t *perm, const int64_t *in_strides,
+                              const int64_t *out_strides, const ttlg_plan_hints *hints) {
+  if (!out) return TTLG_ERR_INVALID_VALUE;
+  *out = nullptr;
+  ttlg_plan_s *p = new (std::nothrow) ttlg_plan_s;
+  if (!p) return TTLG_ERR_NO_MEMORY;
+  ttlg_status st = plan_into(p, dt, rank, extents, perm, hints, false, in_strides, out_strides);
+  if (st != TTLG_OK) {
+    delete p;
+    return st;
+  }
+  *out = p;
+  return TTLG_OK;
+}
+
 ttlg_status ttlg_plan(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *extents,
                       const int32_t *perm) {
   return ttlg_plan_ex(out, dt, rank, extents, perm, nullptr);
@@ -346,6 +378,7 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
 ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
                               void *B_dev, void *stream) {
   if (!plan || !A_host || !B_host || !A_dev || !B_dev) return TTLG_ERR_INVALID_VALUE;
+  if (plan->strided) return TTLG_ERR_UNSUPPORTED;  // dense tensors only
   return execute_host(plan, A_host, B_host, A_dev, B_dev, (cudaStream_t)stream);
 }
 
@@ -380,8 +413,11 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
   ttlg_plan_info list[kGbtTopK];
   CandidateSink sink{list, std::min<int>(max_candidates, kGbtTopK), 0, true};
   ttlg_plan_s scratch;
+  const int64_t *isx = p->strided ? p->in_strides : nullptr;
+  const int64_t *osx = p->strided ? p->out_strides : nullptr;
   ttlg_status st = make_plan(&scratch, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm,
-                             p->has_hints ? &p->hints : nullptr, device_profile(p->device), &sink);
+                             p->has_hints ? &p->hints : nullptr, device_profile(p->device), &sink,
+                             false, isx, osx);
   if (st != TTLG_OK) return st;
   cudaStream_t s = (cudaStream_t)stream;
   cudaEvent_t e0, e1;
@@ -402,7 +438,8 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
     h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : (ci.kernel == KK_QUAD ? 3 : 0));
     ttlg_plan_s *q = new (std::nothrow) ttlg_plan_s;
     if (!q) break;
-    if (plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h) != TTLG_OK) {
+    if (plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false, isx, osx) !=
+        TTLG_OK) {
       delete q;
       continue;
     }
@@ -435,6 +472,70 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
 ttlg_status ttlg_plan_describe(ttlg_plan_t plan, ttlg_plan_info *info) {
   if (!plan || !info) return TTLG_ERR_INVALID_VALUE;
   *info = plan->info;
+  return TTLG_OK;
+}
+
+// ---- peer memory (CUDA IPC) for the fused sharded exchange --------------------
+// The allocation base comes from the driver's cuMemGetAddressRange, reached
+// through the runtime's entry-point query (no link-time libcuda dependency, so
+// the library still loads on a host without a driver).
+typedef int (*MemGetAddressRangeFn)(unsigned long long *, size_t *, unsigned long long);
+
+static MemGetAddressRangeFn mem_range_fn() {
+  static MemGetAddressRangeFn fn = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuMemGetAddressRange", &f, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (MemGetAddressRangeFn)f;
+    else
+      cudaGetLastError();
+  }
+  return fn;
+}
+
+ttlg_status ttlg_ipc_export(const void *ptr, void *handle, int64_t *offset) {
+  if (!ptr || !handle || !offset) return TTLG_ERR_INVALID_VALUE;
+  static_assert(sizeof(cudaIpcMemHandle_t) <= TTLG_IPC_HANDLE_BYTES, "IPC handle size");
+  MemGetAddressRangeFn fn = mem_range_fn();
+  if (!fn) return TTLG_ERR_CUDA;
+  unsigned long long base = 0;
+  size_t size = 0;
+  if (fn(&base, &size, (unsigned long long)(uintptr_t)ptr) != 0) return TTLG_ERR_CUDA;
+  cudaIpcMemHandle_t h;
+  if (cudaIpcGetMemHandle(&h, (void *)(uintptr_t)base) != cudaSuccess) {
+    cudaGetLastError();
+    return TTLG_ERR_CUDA;
+  }
+  memset(handle, 0, TTLG_IPC_HANDLE_BYTES);
+  memcpy(handle, &h, sizeof(h));
+  *offset = (int64_t)((uintptr_t)ptr - (uintptr_t)base);
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_ipc_open(const void *handle, int64_t offset, void **ptr) {
+  if (!handle || !ptr || offset < 0) return TTLG_ERR_INVALID_VALUE;
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, sizeof(h));
+  void *base = nullptr;
+  if (cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    cudaGetLastError();
+    return TTLG_ERR_CUDA;
+  }
+  *ptr = (unsigned char *)base + offset;
+  return TTLG_OK;
+}
+
+ttlg_status ttlg_ipc_close(void *ptr, int64_t offset) {
+  if (!ptr || offset < 0) return TTLG_ERR_INVALID_VALUE;
+  if (cudaIpcCloseMemHandle((unsigned char *)ptr - offset) != cudaSuccess) {
+    cudaGetLastError();
+    return TTLG_ERR_CUDA;
+  }
   return TTLG_OK;
 }
 

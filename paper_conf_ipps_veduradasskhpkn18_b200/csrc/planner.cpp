@@ -42,15 +42,23 @@ ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t 
 
 // Squeeze extent-1 dims (reading R4), then fuse maximal runs of
 // input dims that stay consecutive and in the same order in the output
-// ([i0,i1,i2,i3] => [i3,i1,i2,i0] fuses i1,i2).
-static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool fuse,
-                         Problem &P) {
+// ([i0,i1,i2,i3] => [i3,i1,i2,i0] fuses i1,i2).  `sa` are
+// the input strides per input dim, `sbo` the output strides per OUTPUT dim
+// (elements); a sub-tensor (ttlg_plan_strided) fuses a pair only where both
+// tensors are dense across it.  Dense strides always fuse, so the dense
+// problem is exactly the paper's rule.
+static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, const int64_t *sa,
+                         const int64_t *sbo, bool fuse, Problem &P) {
   int map[TTLG_MAXD];
-  int64_t n[TTLG_MAXD];
+  int64_t n[TTLG_MAXD], ka[TTLG_MAXD], kb[TTLG_MAXD];
+  int64_t sbi[TTLG_MAXD];  // output stride per input dim
+  for (int i = 0; i < rank; i++) sbi[perm[i]] = sbo[i];
   int d = 0;
   for (int k = 0; k < rank; k++) {
     if (ext[k] > 1) {
       map[k] = d;
+      ka[d] = sa[k];
+      kb[d] = sbi[k];
       n[d++] = ext[k];
     } else {
       map[k] = -1;
@@ -64,6 +72,7 @@ static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool
     P.d = 1;
     P.n[0] = 1;
     P.p[0] = 0;
+    P.sA[0] = P.sB[0] = 1;
     return;
   }
   if (!fuse) {
@@ -71,13 +80,18 @@ static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool
     for (int k = 0; k < d; k++) {
       P.n[k] = n[k];
       P.p[k] = p[k];
+      P.sA[k] = ka[k];
+      P.sB[k] = kb[k];
     }
     return;
   }
   // groups in output order
   int gstart[TTLG_MAXD], glen[TTLG_MAXD], ng = 0;
   for (int i = 0; i < d; i++) {
-    if (i == 0 || p[i] != p[i - 1] + 1) {
+    const int k = p[i];
+    const bool joins = i > 0 && k == p[i - 1] + 1 && ka[k] == ka[k - 1] * n[k - 1] &&
+                       kb[k] == kb[k - 1] * n[k - 1];
+    if (!joins) {
       gstart[ng] = i;
       glen[ng] = 1;
       ng++;
@@ -96,6 +110,8 @@ static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool
     for (int q = 0; q < glen[g]; q++) e *= n[first[g] + q];
     P.n[r] = e;
     P.p[g] = r;
+    P.sA[r] = ka[first[g]];
+    P.sB[r] = kb[first[g]];
   }
   P.d = ng;
 }
@@ -103,26 +119,59 @@ static void canonicalize(int rank, const int64_t *ext, const int32_t *perm, bool
 // Matching FVI: the fused FVI row of n0*s bytes is moved as wider access
 // elements (16 B when the row allows).  A row of exactly one access element
 // squeezes away, turning e.g. FMS on [2,4096,4096] fp32 into a plain 2-D
-// transpose of 8-byte elements.
+// transpose of 8-byte elements.  Sub-tensors widen
+// only when every stride is a whole number of access elements, and keep the
+// row when squeezing it would leave a non-unit-stride FVI.
+static bool widen_ok(const Problem &P, int W) {
+  const int64_t R = P.n[0] * P.esize;
+  if (R % W) return false;
+  const int64_t f = W / P.esize;
+  for (int k = 1; k < P.d; k++)
+    if (P.sA[k] % f || P.sB[k] % f) return false;
+  if (R == W && P.d > 1) {  // dim 0 squeezes: the next dims become the FVIs
+    if (P.sA[1] != f || P.sB[P.p[1]] != f) return false;
+  }
+  return true;
+}
+
 static void widen(Problem &P, int forceW) {
   P.W = P.esize;
   if (P.p[0] != 0) return;
-  const int64_t R = P.n[0] * P.esize;
   int W = P.esize;
   if (forceW) {
     W = forceW;
-  } else if (R % 16 == 0) {
+  } else if (widen_ok(P, 16)) {
     W = 16;
-  } else if (R % 8 == 0) {
+  } else if (widen_ok(P, 8)) {
     W = 8;
   }
+  const int64_t f = W / P.esize;
   P.W = W;
-  P.n[0] = R / W;
+  P.n[0] = P.n[0] * P.esize / W;
+  for (int k = 1; k < P.d; k++) {
+    P.sA[k] /= f;
+    P.sB[k] /= f;
+  }
   if (P.n[0] == 1 && P.d > 1) {
-    for (int k = 0; k + 1 < P.d; k++) P.n[k] = P.n[k + 1];
+    for (int k = 0; k + 1 < P.d; k++) {
+      P.n[k] = P.n[k + 1];
+      P.sA[k] = P.sA[k + 1];
+      P.sB[k] = P.sB[k + 1];
+    }
     for (int i = 0; i + 1 < P.d; i++) P.p[i] = P.p[i + 1] - 1;
     P.d--;
   }
+}
+
+// Dense prefixes: the input run (dims 0..a) and the output run (dims
+// p[0..b]) of a tile must be contiguous in A and B.
+static void dense_prefixes(Problem &P) {
+  P.denseA = 0;
+  while (P.denseA + 1 < P.d && P.sA[P.denseA + 1] == P.sA[P.denseA] * P.n[P.denseA]) P.denseA++;
+  P.denseB = 0;
+  while (P.denseB + 1 < P.d &&
+         P.sB[P.p[P.denseB + 1]] == P.sB[P.p[P.denseB]] * P.n[P.p[P.denseB]])
+    P.denseB++;
 }
 
 namespace {
@@ -139,12 +188,9 @@ struct Strides {
 
 Strides strides_of(const Problem &P) {
   Strides S;
-  S.sA[0] = 1;
-  for (int k = 1; k < P.d; k++) S.sA[k] = S.sA[k - 1] * P.n[k - 1];
-  int64_t s = 1;
-  for (int i = 0; i < P.d; i++) {
-    S.sB[P.p[i]] = s;
-    s *= P.n[P.p[i]];
+  for (int k = 0; k < P.d; k++) {
+    S.sA[k] = P.sA[k];
+    S.sB[k] = P.sB[k];
   }
   return S;
 }
@@ -191,7 +237,10 @@ int quad_k(const Problem &P, const Tile &T) {
     if (P.p[i] <= T.a) return 0;  // groups overlap: not OD
   const int p0 = P.p[0];
   for (int K = 16 / P.W; K >= 2; K /= 2) {
-    if (P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 && T.t[p0] % K == 0) return K;
+    bool ok = P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 && T.t[p0] % K == 0;
+    for (int k = 0; k < P.d && ok; k++)  // sub-tensors: every row start chunk-aligned
+      ok = (k == 0 || P.sA[k] % K == 0) && (k == p0 || P.sB[k] % K == 0);
+    if (ok) return K;
     if (P.W == 8) break;  // fp64: 16-byte chunks only
   }
   return 0;
@@ -619,21 +668,69 @@ static void fill_info(ttlg_plan_info &I, ttlg_dtype dt, int rank, const Problem 
 
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints,
-                      const DeviceProfile &dev, CandidateSink *sink, bool fast) {
+                      const DeviceProfile &dev, CandidateSink *sink, bool fast,
+                      const int64_t *in_strides, const int64_t *out_strides) {
   ttlg_status st = validate(dt, rank, ext, perm);
   if (st != TTLG_OK) return st;
   const int s = (dt == TTLG_F64) ? 8 : 4;
+  // strides in elements: dense prefix products unless given (sub-tensor)
+  int64_t sa[TTLG_MAXD], sbo[TTLG_MAXD];
+  {
+    int64_t acc = 1;
+    for (int k = 0; k < rank; k++) {
+      sa[k] = in_strides ? in_strides[k] : acc;
+      acc *= ext[k];
+    }
+    acc = 1;
+    for (int i = 0; i < rank; i++) {
+      sbo[i] = out_strides ? out_strides[i] : acc;
+      acc *= ext[perm[i]];
+    }
+  }
+  int64_t spanA = 1, spanB = 1;
+  {
+    // strides of non-unit dims must be >= 1 and keep every offset in int64;
+    // B must be injective: sorted by stride, each dim must clear the box of
+    // the smaller ones (sufficient, and what any sub-tensor view satisfies)
+    int64_t ob[TTLG_MAXD], on[TTLG_MAXD];
+    int no = 0;
+    for (int k = 0; k < rank; k++) {
+      if (ext[k] == 1) continue;
+      if (sa[k] < 1 || sa[k] > (INT64_MAX / 8) / ext[k]) return TTLG_ERR_INVALID_VALUE;
+      spanA += (ext[k] - 1) * sa[k];
+      if (spanA > INT64_MAX / 16) return TTLG_ERR_INVALID_VALUE;
+    }
+    for (int i = 0; i < rank; i++) {
+      const int64_t e = ext[perm[i]];
+      if (e == 1) continue;
+      if (sbo[i] < 1 || sbo[i] > (INT64_MAX / 8) / e) return TTLG_ERR_INVALID_VALUE;
+      spanB += (e - 1) * sbo[i];
+      if (spanB > INT64_MAX / 16) return TTLG_ERR_INVALID_VALUE;
+      ob[no] = sbo[i];
+      on[no++] = e;
+    }
+    for (int x = 1; x < no; x++)  // insertion sort by stride
+      for (int y = x; y > 0 && ob[y] < ob[y - 1]; y--) {
+        std::swap(ob[y], ob[y - 1]);
+        std::swap(on[y], on[y - 1]);
+      }
+    for (int x = 0; x + 1 < no; x++)
+      if (ob[x + 1] < ob[x] * on[x]) return TTLG_ERR_INVALID_VALUE;
+  }
   Problem P;
   P.esize = s;
-  canonicalize(rank, ext, perm, !(hints && hints->no_fusion), P);
+  canonicalize(rank, ext, perm, sa, sbo, !(hints && hints->no_fusion), P);
+  // the kernels move contiguous runs along each tensor's FVI
+  if (P.sA[0] != 1 || P.sB[P.p[0]] != 1) return TTLG_ERR_UNSUPPORTED;
   int forceW = 0;
   if (hints && hints->elem_bytes_override) {
     forceW = hints->elem_bytes_override;
     if (forceW != 4 && forceW != 8 && forceW != 16) return TTLG_ERR_INVALID_VALUE;
     if (forceW < s) return TTLG_ERR_UNSUPPORTED;
-    if (forceW > s && (P.p[0] != 0 || (P.n[0] * s) % forceW != 0)) return TTLG_ERR_UNSUPPORTED;
+    if (forceW > s && (P.p[0] != 0 || !widen_ok(P, forceW))) return TTLG_ERR_UNSUPPORTED;
   }
   widen(P, forceW);
+  dense_prefixes(P);
 
   if (hints && hints->threads &&
       (hints->threads < 64 || hints->threads > 512 || hints->threads % 8))
@@ -901,7 +998,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (P.p[0] == 0) {
     // ---- direct (FML / COPY): input run = dims 0..a (contiguous), output run = dim 0
     int64_t pre = 1;
-    for (int a = 0; a < P.d; a++) {
+    for (int a = 0; a <= P.denseA; a++) {
       const int nb = cand_blocks(P.n[a], pre, P.W, blocksA, hints ? hints->in_block : 0,
                                  kTileTargets);
       for (int i = 0; i < nb; i++) {
@@ -917,11 +1014,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
-    for (int a = 0; a < P.d; a++) {
+    for (int a = 0; a <= P.denseA; a++) {
       const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0,
                                   kRunTargets);
       int64_t preB = 1;
-      for (int b = 0; b < P.d; b++) {
+      for (int b = 0; b <= P.denseB; b++) {
         const int pb = P.p[b];
         const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0,
                                     kRunTargets);
@@ -1063,6 +1160,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->threads = B.mi.threads;
   plan->grid = B.mi.grid;
   plan->nbytes = N * P.W;
+  plan->spanA = spanA * s;
+  plan->spanB = spanB * s;
   plan->kp = K;
   fill_info(plan->info, dt, rank, P, B.T, K, B.mi, B.schema, B.kind, win_t, ncand);
   {

@@ -116,6 +116,13 @@ struct Problem {
   int d;           // fused rank
   int64_t n[TTLG_MAXD];
   int32_t p[TTLG_MAXD];
+  // strides per fused INPUT dim, in access elements: offset in A of digit k
+  // is i_k * sA[k], offset in B is i_k * sB[k] (dense tensors: prefix
+  // products; sub-tensors: ttlg_plan_strided).  sA[0] = sB[p[0]] = 1.
+  int64_t sA[TTLG_MAXD], sB[TTLG_MAXD];
+  // largest input-run dim a / output-run position b whose prefix is dense
+  // (a tile's input and output runs must stay contiguous)
+  int denseA, denseB;
 };
 
 struct DeviceProfile {
@@ -139,6 +146,7 @@ struct ttlg_plan_s {
   int grid;
   int variant;  // reserved (hints->variant)
   int64_t nbytes;  // N * s
+  int64_t spanA, spanB;  // bytes from the base pointer to one past the last element
   ttlg::TileParams kp;
   ttlg_plan_info info;
   // original request (for the misaligned-pointer fallback)
@@ -147,6 +155,9 @@ struct ttlg_plan_s {
   int32_t perm[TTLG_MAXD];
   ttlg_plan_hints hints;
   bool has_hints;
+  // sub-tensor (ttlg_plan_strided) request: strides in elements as given
+  bool strided;
+  int64_t in_strides[TTLG_MAXD], out_strides[TTLG_MAXD];
 };
 
 namespace ttlg {
@@ -163,9 +174,12 @@ ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t 
 // fast = the single-use effort level: refine the linear screen's best
 // kFastRefine candidates and rank kFastTopK of them with the trees
 constexpr int kFastRefine = 12, kFastTopK = 8;
+// in_strides / out_strides (elements; NULL = dense): the sub-tensor form of
+// ttlg_plan_strided -- in_strides[k] per input dim, out_strides[i] per output dim
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev,
-                      CandidateSink *sink = nullptr, bool fast = false);
+                      CandidateSink *sink = nullptr, bool fast = false,
+                      const int64_t *in_strides = nullptr, const int64_t *out_strides = nullptr);
 // api.cpp
 const DeviceProfile &device_profile(int device);
 // kernels.cu

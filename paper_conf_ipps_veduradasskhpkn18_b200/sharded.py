@@ -23,6 +23,16 @@ dim o_{d-1} = input dim q = perm[d-1] (also a contiguous slab of B).
 `local_fn(extents, perm, src, dst)` performs one dense transposition; the
 default is the CUDA library (ttlg_transpose on the current stream).  CPU unit
 tests inject the oracle there to check the decomposition over gloo.
+
+Fused exchange (`P2PExchange`): instead of local transpose ->
+all-to-all -> fold (three HBM passes plus NCCL staging), rank p runs P
+sub-tensor transpositions (ttlg_plan_strided), one per destination q: the
+input is the sub-box i_q in [q*cq, (q+1)*cq) of its A slab, the output is the
+box o_k in [p*c, (p+1)*c) of rank q's B slab, written straight into q's
+memory through a CUDA IPC mapping (NVLink/NVSwitch stores).  One HBM read of A
+and one (remote) write of B per element; no send/receive buffers, no fold.
+`p2p_subproblems` is the pure index arithmetic (tested on the CPU and, with
+every "peer" slab on one device, against the oracle on the GPU).
 """
 from __future__ import annotations
 
@@ -125,3 +135,119 @@ def sharded_transpose(A_local, extents: Sequence[int], perm: Sequence[int], grou
     if phase_events is not None and e0 is not None:
         phase_events += [("local", e0, e1), ("alltoall", e1, e2), ("fold", e2, ev())]
     return out
+
+
+# ---- fused transpose + exchange over peer memory ------------------
+@dataclass
+class SubProblem:
+    dest: int                 # destination rank q
+    extents: List[int]        # sub-box of the local A slab (input order)
+    in_strides: List[int]     # strides of the local A slab (elements)
+    out_strides: List[int]    # strides of rank q's B slab, output order (elements)
+    a_offset: int             # element offset of the sub-box in the local A slab
+    b_offset: int             # element offset of this rank's box in q's B slab
+
+
+def _dense_strides(ext):
+    s, acc = [], 1
+    for e in ext:
+        s.append(acc)
+        acc *= e
+    return s
+
+
+def p2p_subproblems(sp: ShardPlan, rank: int) -> List[SubProblem]:
+    """The P sub-tensor transpositions rank `rank` runs in the fused exchange.
+    No-move plans: one dense local transposition into its own slab."""
+    d = len(sp.extents)
+    sA = _dense_strides(sp.local_extents)
+    if not sp.moved:
+        out_s = _dense_strides(sp.out_local_extents)
+        return [SubProblem(rank, list(sp.local_extents), sA, out_s, 0, 0)]
+    j = sp.perm[d - 1]                      # A dim that becomes B's sharded outermost dim
+    cq = sp.extents[j] // sp.world
+    k = sp.perm.index(d - 1)                # output position of A's sharded dim
+    c = sp.local_extents[d - 1]
+    sB = _dense_strides(sp.out_local_extents)   # every B slab has the same layout
+    subs = []
+    for q in range(sp.world):
+        ext = list(sp.local_extents)
+        ext[j] = cq
+        subs.append(SubProblem(q, ext, sA, sB, q * cq * sA[j], rank * c * sB[k]))
+    return subs
+
+
+def map_peer_slabs(out, group=None):
+    """Exchange CUDA IPC handles of every rank's `out` over the process group
+    and map the peers' buffers on this device.  Returns (pointers by rank,
+    [(pointer, offset)] to pass to unmap_peer_slabs)."""
+    import torch.distributed as dist
+    from . import api
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    h, off = api.ipc_export(out.data_ptr())
+    allh = [None] * world
+    dist.all_gather_object(allh, (h, off), group=group)
+    ptrs, opened = [], []
+    for q, (hq, oq) in enumerate(allh):
+        if q == rank:
+            ptrs.append(out.data_ptr())
+        else:
+            ptr = api.ipc_open(hq, oq)
+            opened.append((ptr, oq))
+            ptrs.append(ptr)
+    return ptrs, opened
+
+
+def unmap_peer_slabs(opened):
+    from . import api
+    for ptr, off in opened:
+        api.ipc_close(ptr, off)
+
+
+class P2PExchange:
+    """Rank-local driver of the fused exchange: maps every peer's B slab
+    (CUDA IPC through the process group), plans the sub-transpositions once
+    (repeated use), and launches them on one stream.
+
+    `out` is this rank's B slab (a CUDA tensor of n_local elements); it must
+    stay allocated while the exchange object lives.  `run()` must be bracketed
+    by a barrier (peers may still read their previous B) and followed by a
+    stream synchronise + barrier before B is read (incoming remote stores)."""
+
+    def __init__(self, extents: Sequence[int], perm: Sequence[int], out, group=None,
+                 dtype=None, peer_ptrs: Optional[List[int]] = None, rank: Optional[int] = None,
+                 world: Optional[int] = None):
+        from . import api
+        self.group = group
+        if world is None or rank is None:
+            import torch.distributed as dist
+            world = dist.get_world_size(group)
+            rank = dist.get_rank(group)
+        self.rank, self.world = rank, world
+        self.sp = plan_shards(extents, perm, world)
+        self.esize = out.element_size()
+        dt = dtype if dtype is not None else api._dt_of_tensor(out)
+        self._opened = []
+        if peer_ptrs is None:
+            peer_ptrs = self._map_peers(out)
+        self.peers = peer_ptrs
+        self.subs = p2p_subproblems(self.sp, rank)
+        self.plans = [api.plan_strided(dt, s.extents, self.sp.perm, s.in_strides, s.out_strides)
+                      for s in self.subs]
+
+    def _map_peers(self, out):
+        ptrs, self._opened = map_peer_slabs(out, self.group)
+        return ptrs
+
+    def predicted_seconds(self) -> float:
+        return sum(p.describe()["predicted_seconds"] for p in self.plans)
+
+    def run(self, A_local, stream: int):
+        a0 = A_local.data_ptr()
+        for s, p in zip(self.subs, self.plans):
+            p.execute(a0 + s.a_offset * self.esize,
+                      self.peers[s.dest] + s.b_offset * self.esize, stream)
+
+    def close(self):
+        unmap_peer_slabs(self._opened)
+        self._opened = []

@@ -96,3 +96,74 @@ def test_plan_shards_rules():
     assert sp.moved and sp.fold_extents == [16, 64 * 64 * 64 * 8, 8]
     with pytest.raises(ValueError):
         plan_shards([4, 4, 4, 2, 8], [2, 0, 1, 4, 3], 4)  # P=4 does not divide n_q = n_3 = 2
+
+
+# ---- the same over the CUDA kernels: two processes sharing cuda:0 (gloo) -----------------
+GPU_CASES = [
+    ([8, 6, 4, 8], [3, 2, 1, 0]),
+    ([8, 6, 4, 8], [0, 3, 2, 1]),
+    ([16, 8, 8, 16, 32], [4, 3, 2, 1, 0]),
+    ([16, 8, 8, 16, 32], [0, 4, 2, 1, 3]),
+    ([16, 8, 8, 16, 32], [2, 0, 1, 4, 3]),
+    ([16, 8, 8, 16, 32], [3, 2, 1, 0, 4]),
+    ([16, 8, 8, 16, 32], [1, 0, 3, 2, 4]),
+]
+
+
+def _gpu_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ipps_veduradasskhpkn18_b200.sharded import P2PExchange
+    try:
+        results = []
+        for ci, (ext, perm) in enumerate(GPU_CASES):
+            sp = plan_shards(ext, perm, world)
+            n = int(np.prod(ext))
+            full = gen_tensor_np(300 + ci, n, 8)
+            slab = full[rank * sp.n_local:(rank + 1) * sp.n_local]
+            A_local = torch.from_numpy(slab.view(np.float64).copy()).cuda()
+            expect = oracle.transpose(full, ext, perm) if rank == 0 else None
+            # (1) local transpose -> all_to_all_single (gloo, CUDA tensors) -> fold
+            B1 = sharded_transpose(A_local, ext, perm)
+            torch.cuda.synchronize()
+            # (2) fused exchange: sub-transpositions store into the peer's slab via CUDA IPC
+            B2 = torch.empty_like(A_local)
+            ex = P2PExchange(ext, perm, B2)
+            torch.cuda.synchronize()
+            dist.barrier()
+            ex.run(A_local, torch.cuda.current_stream().cuda_stream)
+            torch.cuda.synchronize()
+            dist.barrier()
+            for B in (B1, B2):
+                gathered = [torch.empty(sp.n_local, dtype=torch.float64) for _ in range(world)]
+                dist.all_gather(gathered, B.cpu())
+                if rank == 0:
+                    got = torch.cat(gathered).numpy().view(np.uint64)
+                    results.append(bool(np.array_equal(got, expect)))
+            dist.barrier()
+            ex.close()
+        if rank == 0:
+            q.put(results)
+    except Exception as e:  # surface the error in the parent
+        if rank == 0:
+            q.put(repr(e))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+def test_sharded_gpu_two_processes_one_device():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gpu_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=600)
+    for p in procs:
+        p.join(timeout=120)
+    assert isinstance(res, list), res
+    assert len(res) == 2 * len(GPU_CASES) and all(res), res
