@@ -180,7 +180,7 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
-def run_sharded(args, rank, world, local_rank, dev):
+def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
     """--workload sharded: BASELINE config 5, the 8 GiB rank-5 fp32 tensor
     [64,64,64,64,128] sharded on A's outermost dim across the ranks (one
     process per GPU).  No-move perms: one local transposition per rank, no
@@ -191,8 +191,10 @@ def run_sharded(args, rank, world, local_rank, dev):
     the HBM-side cost of its sub-box launches."""
     import torch
     import torch.distributed as dist
+    import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
     from paper_conf_ipps_veduradasskhpkn18_b200.sharded import (
-        plan_shards, P2PExchange, map_peer_slabs, unmap_peer_slabs, sharded_transpose)
+        plan_shards, P2PExchange, map_peer_slabs, unmap_peer_slabs, sharded_transpose,
+        choose_exchange)
     from synth import configs, gen_tensor_torch, case_seed
 
     cases = configs.config5()
@@ -210,7 +212,12 @@ def run_sharded(args, rank, world, local_rank, dev):
     else:
         peers, opened = [B.data_ptr()], []
     work = (torch.empty_like(A), torch.empty_like(A)) if world > 1 else None
-    exs = [P2PExchange(ext, c.perm, B, peer_ptrs=peers, rank=rank, world=world) for c in cases]
+    def make_ex(perm, out, ptrs, r, P):
+        try:
+            return P2PExchange(ext, perm, out, peer_ptrs=ptrs, rank=r, world=P)
+        except ttlg.TtlgError:  # no p2p plan (sub-box FVI collapses): all-to-all only
+            return None
+    exs = [make_ex(c.perm, B, peers, rank, world) for c in cases]
     torch.cuda.synchronize()
 
     def timed(fn, steps):
@@ -231,25 +238,32 @@ def run_sharded(args, rank, world, local_rank, dev):
             dist.barrier()
         return ms
 
-    per, a2a = [], {}
+    per, other, modes = [], {}, {}
     clocks = ClockSampler(local_rank)
     clocks.start()
     time.sleep(0.3)
     for c, ex in zip(cases, exs):
+        key = "".join(map(str, c.perm))
+
         def f_p2p(ex=ex):
             ex.run(A, sptr)
+
+        def f_a2a(c=c):
+            with torch.cuda.stream(stream):
+                sharded_transpose(A, ext, c.perm, work=work)
+        # model-driven choice between the fused exchange and the all-to-all
+        mode = choose_exchange(ext, c.perm, world, "f32")["mode"] if world > 1 else "local"
+        modes[key] = mode
+        fns = {"p2p": f_p2p, "local": f_p2p, "alltoall": f_a2a}
         for _ in range(args.warmup):
-            f_p2p()
-        ms = timed(f_p2p, args.steps)
-        per.append(ms)
-        if world > 1 and ex.sp.moved:
-            def f_a2a(c=c):
-                with torch.cuda.stream(stream):
-                    sharded_transpose(A, ext, c.perm, work=work)
+            fns[mode]()
+        per.append(timed(fns[mode], args.steps))
+        if world > 1 and ex is not None and ex.sp.moved:  # the path not chosen, for comparison
+            alt = "alltoall" if mode == "p2p" else "p2p"
             for _ in range(args.warmup):
-                f_a2a()
-            a2a["".join(map(str, c.perm))] = 2 * n * 4 * args.steps / (
-                timed(f_a2a, args.steps) / 1e3) / 1e9
+                fns[alt]()
+            other[f"{alt}:{key}"] = 2 * n * 4 * args.steps / (
+                timed(fns[alt], args.steps) / 1e3) / 1e9
     clk = clocks.stop()
     total_ms = sum(per)
     value = 2 * n * 4 * len(cases) * args.steps / (total_ms / 1e3) / 1e9
@@ -265,8 +279,9 @@ def run_sharded(args, rank, world, local_rank, dev):
                 sp = plan_shards(ext, c.perm, P)
                 if not sp.moved:
                     continue
-                rexs = [P2PExchange(ext, c.perm, slabs[p], peer_ptrs=ptrs, rank=p, world=P)
-                        for p in range(P)]
+                rexs = [make_ex(c.perm, slabs[p], ptrs, p, P) for p in range(P)]
+                if rexs[0] is None:
+                    continue
 
                 def f_all(rexs=rexs, P=P):
                     for p, ex in enumerate(rexs):
@@ -277,7 +292,8 @@ def run_sharded(args, rank, world, local_rank, dev):
                 emulated[f"P{P}:{''.join(map(str, c.perm))}"] = \
                     2 * n * 4 * max(2, args.steps // 2) / (ms / 1e3) / 1e9
     for ex in exs:
-        ex.close()
+        if ex is not None:
+            ex.close()
     unmap_peer_slabs(opened)
     if rank == 0:
         peak, peak_src, _ = _peaks()
@@ -289,12 +305,17 @@ def run_sharded(args, rank, world, local_rank, dev):
             "data": "synthetic (SplitMix64 bit patterns, generated on device)",
             "config": {"workload": "c5-8GiB-rank5-fp32 sharded on A's outermost dim (BASELINE config 5)",
                        "extents": ext, "perms": [list(c.perm) for c in cases],
-                       "parallelism": f"shard x{world}", "exchange": "fused p2p (CUDA IPC stores)",
+                       "parallelism": f"shard x{world}",
+                       "exchange": "per perm, model-chosen: local (no move) | p2p (fused "
+                                   "sub-transpositions storing over CUDA IPC) | alltoall "
+                                   "(local + NCCL all_to_all_single + fold)",
                        "l2": "no flush: 8 GiB tensors (inputs larger than L2)"},
-            "gpu_launches": sum(len(ex.subs) for ex in exs) * args.steps,
+            "gpu_launches": sum(len(ex.subs) if ex is not None and modes[k] != "alltoall" else 2
+                                for ex, k in zip(exs, modes)) * args.steps,
             "per_perm_gbs": {"".join(map(str, c.perm)): 2 * n * 4 * args.steps / (m / 1e3) / 1e9
                              for c, m in zip(cases, per)},
-            "alltoall_path_gbs": a2a or None,
+            "modes": modes,
+            "other_path_gbs": other or None,
             "p2p_emulated_one_gpu_gbs": emulated or None,
             "frac_of_peak": value / world / peak,
             "clocks": clk,

@@ -31,6 +31,7 @@
 // index with fast-divmod (the paper's decode/compute_base, L725-737).
 #include <cuda_runtime.h>
 
+#include <atomic>
 #include <mutex>
 #include <type_traits>
 
@@ -776,10 +777,16 @@ static const void *quad_ptr(int W, int cb, int nj) {
 }
 
 int kernel_regs(int kind, int W) {
-  static int regs[KK_NUM][3] = {{-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}, {-1, -1, -1}};
+  // read once per (kind, width) under the lock, then lock-free: the planner
+  // asks for every scored candidate
+  static std::atomic<int> regs[KK_NUM][3] = {{{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
+  std::atomic<int> &slot = regs[kind][widx(W)];
+  int r = slot.load(std::memory_order_acquire);
+  if (r >= 0) return r;
   static std::mutex mu;
   std::lock_guard<std::mutex> g(mu);
-  int &r = regs[kind][widx(W)];
+  r = slot.load(std::memory_order_relaxed);
   if (r < 0) {
     cudaFuncAttributes attr;
     const void *fn = kind == KK_QUAD ? quad_ptr(W, 16, 1) : kernel_ptr(kind, W, false, false);
@@ -789,6 +796,7 @@ int kernel_regs(int kind, int W) {
       cudaGetLastError();
       r = 0;
     }
+    slot.store(r, std::memory_order_release);
   }
   return r;
 }

@@ -162,12 +162,15 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
     for (int t = 0; t < kGbtTrees; t++) {
       const int8_t *F = kGbtF[t];
       const float *T = kGbtT[t];
-      for (int c = 0; c < m; c++) {
-        int i = 0;
-#pragma GCC unroll 8
-        for (int l = 0; l < kGbtDepth; l++) i = 2 * i + 1 + (d[c][F[i]] > T[i]);
-        s[c] += kGbtV[t][i - NI];
-      }
+      // level-major: the m walks of one level are independent load chains
+      int idx[kB];
+      for (int c = 0; c < m; c++) idx[c] = 0;
+      for (int l = 0; l < kGbtDepth; l++)
+        for (int c = 0; c < m; c++) {
+          const int i = idx[c];
+          idx[c] = 2 * i + 1 + (d[c][F[i]] > T[i]);
+        }
+      for (int c = 0; c < m; c++) s[c] += kGbtV[t][idx[c] - NI];
     }
     for (int c = 0; c < m; c++) {
       const ModelInput &mi = mis[b0 + c];

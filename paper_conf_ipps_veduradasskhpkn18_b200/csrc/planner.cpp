@@ -166,6 +166,11 @@ static void widen(Problem &P, int forceW) {
 // Dense prefixes: the input run (dims 0..a) and the output run (dims
 // p[0..b]) of a tile must be contiguous in A and B.
 static void dense_prefixes(Problem &P) {
+  P.kalign = 4;
+  for (int k = 0; k < P.d; k++) {
+    if (k > 0) P.kalign = (P.sA[k] % 4 == 0) ? P.kalign : ((P.sA[k] % 2 == 0) ? std::min(P.kalign, 2) : 1);
+    if (k != P.p[0]) P.kalign = (P.sB[k] % 4 == 0) ? P.kalign : ((P.sB[k] % 2 == 0) ? std::min(P.kalign, 2) : 1);
+  }
   P.denseA = 0;
   while (P.denseA + 1 < P.d && P.sA[P.denseA + 1] == P.sA[P.denseA] * P.n[P.denseA]) P.denseA++;
   P.denseB = 0;
@@ -237,10 +242,10 @@ int quad_k(const Problem &P, const Tile &T) {
     if (P.p[i] <= T.a) return 0;  // groups overlap: not OD
   const int p0 = P.p[0];
   for (int K = 16 / P.W; K >= 2; K /= 2) {
-    bool ok = P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 && T.t[p0] % K == 0;
-    for (int k = 0; k < P.d && ok; k++)  // sub-tensors: every row start chunk-aligned
-      ok = (k == 0 || P.sA[k] % K == 0) && (k == p0 || P.sB[k] % K == 0);
-    if (ok) return K;
+    // P.kalign: sub-tensors need every row start chunk-aligned
+    if (P.kalign % K == 0 && P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 &&
+        T.t[p0] % K == 0)
+      return K;
     if (P.W == 8) break;  // fp64: 16-byte chunks only
   }
   return 0;

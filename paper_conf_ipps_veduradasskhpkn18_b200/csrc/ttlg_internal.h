@@ -123,6 +123,9 @@ struct Problem {
   // largest input-run dim a / output-run position b whose prefix is dense
   // (a tile's input and output runs must stay contiguous)
   int denseA, denseB;
+  // largest K in {2, 4} (k_quad chunk elements) dividing every row stride
+  // that a chunk must stay aligned to (A: dims >= 1; B: dims != p[0])
+  int kalign;
 };
 
 struct DeviceProfile {

@@ -251,3 +251,40 @@ class P2PExchange:
     def close(self):
         unmap_peer_slabs(self._opened)
         self._opened = []
+
+
+# ---- choosing the exchange (model-driven, like the paper's schema choice) -----------
+NVLINK_GBS = 770.0  # measured peer copy per direction per GPU (B200_PROFILING.md)
+
+
+def _dtype_bytes(dtype) -> int:
+    return 8 if str(dtype) in ("f64", "float64", "torch.float64", "fp64", "1") else 4
+
+
+def choose_exchange(extents: Sequence[int], perm: Sequence[int], world: int, dtype="f32",
+                    nvlink_gbs: float = NVLINK_GBS) -> dict:
+    """Predicted per-rank seconds of the two exchange paths and the choice.
+
+    p2p     : max(sum of the sub-transpositions' model predictions,
+                  remote bytes / NVLink)  (the stores overlap the kernels);
+    alltoall: local transposition + (P-1)/P of the slab over NVLink + fold.
+    Either prediction is None when the path does not apply (a sub-box whose
+    FVI collapses to a non-unit stride, cq = 1 on A's FVI, has no p2p plan)."""
+    from . import api
+    sp = plan_shards(extents, perm, world)
+    s = _dtype_bytes(dtype)
+    slab = sp.n_local * s
+    if not sp.moved:
+        t = api.predict_time(dtype, sp.local_extents, sp.perm)
+        return {"mode": "local", "p2p": t, "alltoall": t}
+    remote = slab * (world - 1) / world / (nvlink_gbs * 1e9)
+    try:
+        t_sub = sum(api.plan_strided(dtype, q.extents, sp.perm, q.in_strides, q.out_strides)
+                    .describe()["predicted_seconds"] for q in p2p_subproblems(sp, 0))
+        t_p2p = max(t_sub, remote)
+    except api.TtlgError:
+        t_p2p = None
+    t_a2a = (api.predict_time(dtype, sp.local_extents, sp.perm) + remote +
+             api.predict_time(dtype, sp.fold_extents, [0, 2, 1]))
+    mode = "p2p" if t_p2p is not None and t_p2p <= t_a2a else "alltoall"
+    return {"mode": mode, "p2p": t_p2p, "alltoall": t_a2a}

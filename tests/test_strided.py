@@ -114,6 +114,19 @@ def test_fusion_stops_at_gaps():
     assert gap["fused_rank"] == 4
 
 
+def test_choose_exchange_rules():
+    from paper_conf_ipps_veduradasskhpkn18_b200.sharded import choose_exchange
+    ext = [64, 64, 64, 64, 128]
+    assert choose_exchange(ext, [3, 2, 1, 0, 4], 8)["mode"] == "local"
+    r = choose_exchange(ext, [0, 4, 2, 1, 3], 8)
+    assert r["mode"] == "p2p" and r["p2p"] < r["alltoall"]
+    # 32-byte sub-box runs on A's FVI at P = 8: the model prefers the all-to-all
+    assert choose_exchange(ext, [4, 3, 2, 1, 0], 8)["mode"] == "alltoall"
+    # cq = 1 on A's FVI: no p2p plan at all
+    r = choose_exchange([4, 6, 4, 8], [3, 2, 1, 0], 4)
+    assert r["p2p"] is None and r["mode"] == "alltoall"
+
+
 def test_strided_rejections():
     with pytest.raises(ttlg.TtlgError) as e:   # A's FVI not unit-stride
         ttlg.plan_strided("f32", [8, 8], [1, 0], [2, 16], None)
@@ -228,6 +241,11 @@ def test_gpu_p2p_exchange_virtual_peers(case, world):
         sp = plan_shards(ext, perm, world)
     except ValueError:
         pytest.skip("P does not divide the sharded extents")
+    from paper_conf_ipps_veduradasskhpkn18_b200.sharded import choose_exchange
+    if choose_exchange(ext, perm, world)["p2p"] is None:
+        # cq = 1 on A's FVI: no unit-stride run left; the all-to-all path serves it
+        assert choose_exchange(ext, perm, world)["mode"] == "alltoall"
+        pytest.skip("no p2p plan (sub-box FVI collapses)")
     n = int(np.prod(ext))
     for eb in (4, 8):
         A = gen_tensor_torch(41, n, eb, device="cuda:0")
