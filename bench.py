@@ -432,9 +432,22 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         elapsed_ms = float(t.item())
     launches = len(plans) * args.steps
-    # per-launch durations: the same K steps again with an event pair around
-    # every launch (event records between kernels add bubbles, so the headline
-    # step above is timed uninstrumented)
+    # per-kernel durations: the same K steps again, the launches of each kernel
+    # grouped between ONE event pair per kernel and step (an event record
+    # between two launches adds a bubble, so per-launch pairs would inflate
+    # every duration; the headline step above is timed uninstrumented)
+    kinds = sorted({kname(inf) for inf in infos})
+    kev = {k: [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)] for k in kinds}
+    with torch.cuda.stream(stream):
+        for s in range(args.steps):
+            for k in kinds:
+                kev[k][s][0].record(stream)
+                for i, p in enumerate(plans):
+                    if kname(infos[i]) == k:
+                        p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
+                kev[k][s][1].record(stream)
+    # per-case durations (model error, per-case table): an event pair per launch
     for s in range(args.steps):
         one_step(evs[s])
     torch.cuda.synchronize()
@@ -447,9 +460,10 @@ def main():
     for i, info in enumerate(infos):
         k = kname(info)
         g = groups.setdefault(k, {"ms": 0.0, "bytes": 0, "launches": 0})
-        g["ms"] += sum(per_case_ms[i])
         g["bytes"] += cases[i].alg_bytes * args.steps
         g["launches"] += args.steps
+    for k, g in groups.items():
+        g["ms"] = sum(a.elapsed_time(b) for a, b in kev[k])
     dom = max(groups, key=lambda k: groups[k]["ms"])
     dg = groups[dom]
     achieved = dg["bytes"] / (dg["ms"] / 1e3) / 1e9
@@ -563,8 +577,9 @@ def main():
                        "bytes_per_step": step_bytes, "parallelism": f"replica x{world}",
                        "mode": "repeated-use (pre-built plans)",
                        "timing": "value: K steps between two events (no per-launch events); "
-                                 "roofline/kernels/cases: a second pass of K steps with an "
-                                 "event pair around every launch",
+                                 "roofline/kernels: a second pass of K steps, each kernel's "
+                                 "launches grouped between one event pair per step; cases / "
+                                 "model error: a third pass with an event pair per launch",
                        "l2": "no flush: every case moves >= 2x126 MB L2 (inputs larger than L2)"},
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
