@@ -345,21 +345,11 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
   };
   if (decoder && first < P.num_tiles) put_ctx(0, first);
 
+  // A-side tables first (A-row table, icol): the first tile's loads are
+  // issued before the B-side tables are built, so that build runs under the
+  // load latency
   build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
              reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB), W);
-  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
-             reinterpret_cast<int2 *>(smem + P.off_tabB),
-             reinterpret_cast<int *>(smem + P.off_digA), W);
-#pragma unroll 1
-  for (int j = tid; j < P.LB; j += NT) {
-    int rem = j, s = 0;
-    for (int k = 0; k < P.nj; k++) {
-      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
-      s += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
-      rem = cq;
-    }
-    reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
-  }
   if constexpr (XT) {
 #pragma unroll 1
     for (int x = tid; x < P.LA; x += NT) {
@@ -372,27 +362,43 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
       reinterpret_cast<int *>(smem + P.off_icol)[x] = s * W;  // byte offset
     }
   }
-  __syncthreads();
+  __syncthreads();  // tabA, digB, icol, ctx[0] visible
 
   const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB, V = P.V;
   // load walk: element e = tid + k*NT
   const int rA0 = (int)fdiv1(tid, P.fd_LA), xA0 = tid - rA0 * LA;
   const int nA = tid < V ? (int)fdiv1(V - 1 - tid, P.fd_NT) + 1 : 0;
   const int drA = P.drA, dxA = P.dxA;
-  // store walk
-  int jB0, rB0, nB;
+  // store walk (set up once the B-side tables exist)
+  int jB0 = 0, rB0 = 0, nB = 0;
   uint32_t jc0 = 0;
-  if constexpr (!SM2) {
-    rB0 = (int)fdiv1(tid, P.fd_LB);
-    jB0 = tid - rB0 * LB;
-    // threads past rsB*LB idle
-    nB = (rB0 < P.rsB && rB0 < RB) ? (int)fdiv1(RB - 1 - rB0, P.fd_rsB) + 1 : 0;
-    jc0 = lds_int(s_jcol + 4 * jB0);
-  } else {
-    jB0 = tid;
-    rB0 = 0;
-    nB = RB;
-  }
+  auto build_b_side = [&]() {
+    build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
+               reinterpret_cast<int2 *>(smem + P.off_tabB),
+               reinterpret_cast<int *>(smem + P.off_digA), W);
+#pragma unroll 1
+    for (int j = tid; j < P.LB; j += NT) {
+      int rem = j, s = 0;
+      for (int k = 0; k < P.nj; k++) {
+        const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+        s += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
+        rem = cq;
+      }
+      reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * W;  // byte offset
+    }
+    __syncthreads();  // tabB, digA, jcol visible
+    if constexpr (!SM2) {
+      rB0 = (int)fdiv1(tid, P.fd_LB);
+      jB0 = tid - rB0 * LB;
+      // threads past rsB*LB idle
+      nB = (rB0 < P.rsB && rB0 < RB) ? (int)fdiv1(RB - 1 - rB0, P.fd_rsB) + 1 : 0;
+      jc0 = lds_int(s_jcol + 4 * jB0);
+    } else {
+      jB0 = tid;
+      rB0 = 0;
+      nB = RB;
+    }
+  };
 
   // load phase of one tile: A-rows -> smem with predicated cp.async.  Row
   // table entries hold (global element offset, shared byte offset).  FULL
@@ -491,13 +497,19 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
     // k_tile: one tile (or tpc consecutive tiles) per CTA, single buffer, many
     // CTAs per SM -- the cp.async skeleton that reaches the D2D copy rate
     // (tools/copybench.cu)
+    TileCtx c = get_ctx(0);
+    if (first < P.num_tiles) issue(c, s_buf0);
+    cp_async_commit();
+    build_b_side();
     for (int it = 0; it < P.tpc; it++) {
       const uint32_t tile = first + it;
       if (tile >= P.num_tiles) break;
-      if (it > 0) __syncthreads();  // buffer drained, ctx[it & 1] visible
-      const TileCtx c = get_ctx(it & 1);
-      issue(c, s_buf0);
-      cp_async_commit();
+      if (it > 0) {
+        __syncthreads();  // buffer drained, ctx[it & 1] visible
+        c = get_ctx(it & 1);
+        issue(c, s_buf0);
+        cp_async_commit();
+      }
       if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
       cp_async_wait<0>();
       __syncthreads();
@@ -505,11 +517,12 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
     }
   } else {
     uint32_t tile = first;
-    if (tile >= P.num_tiles) return;
     TileCtx cur = get_ctx(0);
-    issue(cur, s_buf0);
+    if (tile < P.num_tiles) issue(cur, s_buf0);
     cp_async_commit();
-    if (decoder && tile + tstep < P.num_tiles) put_ctx(1, tile + tstep);
+    if (decoder && tile < P.num_tiles && tile + tstep < P.num_tiles) put_ctx(1, tile + tstep);
+    build_b_side();
+    if (tile >= P.num_tiles) return;
     for (int k = 0; tile < P.num_tiles; k++) {
       __syncthreads();  // ctx[(k+1)&1] visible; buffer (k+1)&1 drained (iteration k-1)
       const uint32_t next = tile + tstep;
@@ -628,9 +641,53 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
     ctx[slot].limB = c.limB;
   };
   if (decoder && first < P.num_tiles) put_ctx(0, first);
-  // row tables: (global element offset, shared byte offset)
+  // A-row table (global element offset, shared byte offset) first: the first
+  // tile's loads are issued before the B-side tables are built, so that
+  // build runs under the load latency
   build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
              reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB), S);
+  __syncthreads();  // tabA, digB, ctx[0] visible
+
+  const int LB = P.LB, LAc = P.LA / K;  // chunks per A-row
+  const int nChunks = P.V / K;
+  // load walk over chunks: chunk e = tid + k*NT -> A-row e / LAc, chunk e mod LAc
+  const int rA0 = (int)fdiv1(tid, P.fd_LA), cA0 = tid - rA0 * LAc;
+  const int nA = tid < nChunks ? (int)fdiv1(nChunks - 1 - tid, P.fd_NT) + 1 : 0;
+  const int drA = P.drA, dxA = P.dxA;
+  auto get_ctx = [&](int slot) {
+    TileCtx c;
+    c.bA = ctx[slot].bA;
+    c.bB = ctx[slot].bB;
+    c.limA = ctx[slot].limA;
+    c.limB = ctx[slot].limB;
+    return c;
+  };
+  auto load = [&](const TileCtx &c, bool full) {
+    const C *Ab = reinterpret_cast<const C *>(A + c.bA * S);  // chunk-aligned
+    const int limc = full ? LAc : (P.LAunit * c.limA) / K;
+    int r = rA0, cx = cA0;
+#pragma unroll 4
+    for (int k = 0; k < nA; k++) {
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const uint32_t soff = t.y + cx * CB;
+      const C *g = wadd(Ab, ((uint32_t)t.x >> LGK) + cx);
+      if (full)
+        cp_async<CB>(s_buf + soff, g);
+      else
+        cp_async_p<CB>(s_buf + soff, g, cx < limc && lds_int(s_digB + 4 * r) < c.limB);
+      cx += dxA;
+      r += drA;
+      if (cx >= LAc) {
+        cx -= LAc;
+        r++;
+      }
+    }
+  };
+  TileCtx c = get_ctx(0);
+  bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+  if (first < P.num_tiles) load(c, full);
+  cp_async_commit();
+
   build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
              reinterpret_cast<int2 *>(smem + P.off_tabB),
              reinterpret_cast<int *>(smem + P.off_digA), S);
@@ -644,14 +701,8 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
     }
     reinterpret_cast<int *>(smem + P.off_jcol)[j] = s * S;
   }
-  __syncthreads();
+  __syncthreads();  // tabB, digA, jcol visible (the first tile's loads still in flight)
 
-  const int LB = P.LB, LAc = P.LA / K;  // chunks per A-row
-  const int nChunks = P.V / K;
-  // load walk over chunks: chunk e = tid + k*NT -> A-row e / LAc, chunk e mod LAc
-  const int rA0 = (int)fdiv1(tid, P.fd_LA), cA0 = tid - rA0 * LAc;
-  const int nA = tid < nChunks ? (int)fdiv1(nChunks - 1 - tid, P.fd_NT) + 1 : 0;
-  const int drA = P.drA, dxA = P.dxA;
   // store walk: output positions j0 + c*NT (c < NJ; NJ = 1 when LB <= NT),
   // row quads m0, m0 + rsB, ...
   int m0, j0, rs;
@@ -674,44 +725,22 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
   uint32_t jc[NJ];
   bool jv[NJ];
 #pragma unroll
-  for (int c = 0; c < NJ; c++) {
-    const int jj = j0 + c * NT;
-    jv[c] = jj < LB;
-    jc[c] = lds_int(s_jcol + 4 * (jv[c] ? jj : j0));
+  for (int cc = 0; cc < NJ; cc++) {
+    const int jj = j0 + cc * NT;
+    jv[cc] = jj < LB;
+    jc[cc] = lds_int(s_jcol + 4 * (jv[cc] ? jj : j0));
   }
 
   for (int it = 0; it < P.tpc; it++) {
     const uint32_t tile = first + it;
     if (tile >= P.num_tiles) break;
-    if (it > 0) __syncthreads();
-    TileCtx c;
-    c.bA = ctx[it & 1].bA;
-    c.bB = ctx[it & 1].bB;
-    c.limA = ctx[it & 1].limA;
-    c.limB = ctx[it & 1].limB;
-    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
-    {  // load
-      const C *Ab = reinterpret_cast<const C *>(A + c.bA * S);  // chunk-aligned
-      const int limc = full ? LAc : (P.LAunit * c.limA) / K;
-      int r = rA0, cx = cA0;
-#pragma unroll 4
-      for (int k = 0; k < nA; k++) {
-        const int2 t = lds_int2(s_tabA + 8 * r);
-        const uint32_t soff = t.y + cx * CB;
-        const C *g = wadd(Ab, ((uint32_t)t.x >> LGK) + cx);
-        if (full)
-          cp_async<CB>(s_buf + soff, g);
-        else
-          cp_async_p<CB>(s_buf + soff, g, cx < limc && lds_int(s_digB + 4 * r) < c.limB);
-        cx += dxA;
-        r += drA;
-        if (cx >= LAc) {
-          cx -= LAc;
-          r++;
-        }
-      }
+    if (it > 0) {
+      __syncthreads();  // buffer drained, ctx[it & 1] visible
+      c = get_ctx(it & 1);
+      full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+      load(c, full);
+      cp_async_commit();
     }
-    cp_async_commit();
     if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
     cp_async_wait<0>();
     __syncthreads();
