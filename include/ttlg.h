@@ -91,7 +91,10 @@ typedef struct {
   int32_t variant;                       /* staged kernel: 0 = model choice, 1 = k_tile
                                             (one tile per CTA), 2 = k_pipe (persistent,
                                             double-buffered), 3 = k_quad (OD in 16-byte
-                                            chunks, K x K register transpose)            */
+                                            chunks, K x K register transpose), 4 = k_deint
+                                            ([n0,M(,nb)] perm (1 0 (2)), 2 <= n0 <= 8,
+                                            M a multiple of 16/s: 16-byte accesses both
+                                            ways, no shared memory)                       */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -114,7 +117,7 @@ typedef struct {
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
   int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe,
-                                             3 k_quad                                    */
+                                             3 k_quad, 4 k_deint                         */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[12];

@@ -199,12 +199,14 @@ def plan_candidates(dtype, extents, perm, max_out: int = 4096, **hints) -> list:
 
 def candidate_hints(d: dict) -> dict:
     """Hints that reproduce a candidate returned by plan_candidates()."""
+    if d["kernel"] == "deint":
+        return {"variant": 4}
     a, b = d["in_dim"], d["out_dim"]
     h = {"schema": d["schema"] if d["schema"] != "COPY" else "FML", "in_dim": a,
          "in_block": d["tile_extents"][a], "out_dim": b,
          "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
     if d["kernel"] != "direct":
-        h["variant"] = {"tile": 1, "pipe": 2, "quad": 3}[d["kernel"]]
+        h["variant"] = {"tile": 1, "pipe": 2, "quad": 3, "deint": 4}[d["kernel"]]
     return h
 
 

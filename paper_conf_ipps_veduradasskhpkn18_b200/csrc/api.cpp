@@ -150,7 +150,7 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
       ttlg_plan_hints_init(&h);
     }
     h.elem_bytes_override = s;
-    if (h.variant == 3) h.variant = 0;  // k_quad needs 16-byte alignment
+    if (h.variant == 3 || h.variant == 4) h.variant = 0;  // k_quad / k_deint need 16-byte alignment
     ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false,
                                p->strided ? p->in_strides : nullptr,
                                p->strided ? p->out_strides : nullptr);
@@ -436,6 +436,10 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
     h.out_block = ci.tile_extents[ci.fused_perm[ci.out_dim]];
     h.threads = ci.threads;
     h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : (ci.kernel == KK_QUAD ? 3 : 0));
+    if (ci.kernel == KK_DEINT) {  // no slice parameters: the structure size fixes the slice
+      ttlg_plan_hints_init(&h);
+      h.variant = 4;
+    }
     ttlg_plan_s *q = new (std::nothrow) ttlg_plan_s;
     if (!q) break;
     if (plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false, isx, osx) !=

@@ -768,6 +768,77 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
   }
 }
 
+// k_deint (Orthogonal-Arbitrary with a tiny input FVI: array-of-structures ->
+// structure-of-arrays): the fused problem [n0, M] perm (1 0), or the batch
+// [n0, M, nb] perm (1 0 2), with N0 = n0 <= 8 and M a multiple of K = 16/S.
+// The slice of one thread is N0 x K elements: chunk c (grid-stride) = batch b
+// = c / (M/K), column block q = c mod (M/K).  Its input is ONE contiguous run
+// of N0*K elements, A[N0*(K*q + M*b) ...], loaded as N0 16-byte vectors; its
+// output is N0 runs of K elements, B[M*(r + N0*b) + K*q ...] for r < N0, each
+// written as ONE 16-byte vector after an in-register regrouping (element
+// u*N0 + r of the input run is position u of output row r).  No shared
+// memory, no shuffles: the warp's N0 load instructions together cover 512*N0
+// contiguous bytes (the later ones hit the lines the first ones brought into
+// L1), and every store instruction writes 512 contiguous bytes.
+// Parameters ride in TileParams: deint_n0 = N0, gdiv[0] = fastdiv(M/K),
+// num_tiles = chunks.
+template <int S, int N0>
+__global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParams P,
+                                               const void *__restrict__ Av,
+                                               void *__restrict__ Bv) {
+  constexpr int K = 16 / S;          // elements per 16-byte vector
+  constexpr int E = N0 * K;          // elements per thread slice
+  constexpr int WPE = S / 4;         // 32-bit words per element
+  const uint4 *A = reinterpret_cast<const uint4 *>(Av);
+  uint4 *B = reinterpret_cast<uint4 *>(Bv);
+  const uint32_t nq = P.gdiv[0].div;  // M / K
+  const uint32_t total = P.num_tiles;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < total;
+       c += gridDim.x * blockDim.x) {
+    const uint32_t b = fdiv1(c, P.gdiv[0]);
+    const uint32_t q = c - b * nq;
+    // input run: N0 vectors starting at vector N0 * c (the batch is contiguous)
+    uint32_t w[E * WPE];
+    const uint4 *src = wadd(A, 0u) + (size_t)c * N0;
+#pragma unroll
+    for (int i = 0; i < N0; i++) {
+      const uint4 v = __ldcs(src + i);
+      w[4 * i + 0] = v.x;
+      w[4 * i + 1] = v.y;
+      w[4 * i + 2] = v.z;
+      w[4 * i + 3] = v.w;
+    }
+    // output row r of batch b: vector index (r + N0*b) * (M/K) + q
+    uint4 *dst = B + ((size_t)b * N0) * nq + q;
+#pragma unroll
+    for (int r = 0; r < N0; r++) {
+      uint32_t o[4];
+#pragma unroll
+      for (int u = 0; u < K; u++)
+#pragma unroll
+        for (int h = 0; h < WPE; h++) o[u * WPE + h] = w[(u * N0 + r) * WPE + h];
+      __stcs(dst + (size_t)r * nq, make_uint4(o[0], o[1], o[2], o[3]));
+    }
+  }
+}
+
+template <int S>
+static const void *deint_ptr_s(int n0) {
+  switch (n0) {
+    case 2: return (const void *)k_deint<S, 2>;
+    case 3: return (const void *)k_deint<S, 3>;
+    case 4: return (const void *)k_deint<S, 4>;
+    case 5: return (const void *)k_deint<S, 5>;
+    case 6: return (const void *)k_deint<S, 6>;
+    case 7: return (const void *)k_deint<S, 7>;
+    case 8: return (const void *)k_deint<S, 8>;
+  }
+  return nullptr;
+}
+static const void *deint_ptr(int W, int n0) {
+  return W == 8 ? deint_ptr_s<8>(n0) : (W == 4 ? deint_ptr_s<4>(n0) : nullptr);
+}
+
 // ---------------------------------------------------------------------------
 // launch plumbing
 template <int W, bool XT>
@@ -809,7 +880,8 @@ int kernel_regs(int kind, int W) {
   // read once per (kind, width) under the lock, then lock-free: the planner
   // asks for every scored candidate
   static std::atomic<int> regs[KK_NUM][3] = {{{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
-                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
+                                             {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
   if (r >= 0) return r;
@@ -818,7 +890,9 @@ int kernel_regs(int kind, int W) {
   r = slot.load(std::memory_order_relaxed);
   if (r < 0) {
     cudaFuncAttributes attr;
-    const void *fn = kind == KK_QUAD ? quad_ptr(W, 16, 1) : kernel_ptr(kind, W, false, false);
+    const void *fn = kind == KK_QUAD    ? quad_ptr(W, 16, 1)
+                     : kind == KK_DEINT ? deint_ptr(W == 8 ? 8 : 4, 4)
+                                        : kernel_ptr(kind, W, false, false);
     if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
       r = attr.numRegs;
     } else {
@@ -833,7 +907,10 @@ int kernel_regs(int kind, int W) {
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
   const void *fn = plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
-                       : kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0, plan->kp.xtab != 0);
+                       : plan->kind == KK_DEINT
+                             ? deint_ptr(plan->W, plan->kp.deint_n0)
+                             : kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0,
+                                          plan->kp.xtab != 0);
   if (!fn) return TTLG_ERR_INTERNAL;
   const int smem = plan->kp.smem_bytes;
   if (smem > 48 * 1024) {

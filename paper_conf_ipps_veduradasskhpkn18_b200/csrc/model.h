@@ -40,4 +40,9 @@ void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d)
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
 void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
 
+// k_deint (one streaming pass, 16-byte accesses both ways): time = this
+// factor x the one-pass ideal 2*N*s / HBM bandwidth -- measured on B200 at
+// the config-4 sizes, n0 = 2..5: 5.41-5.63 TB/s back to back (exp49)
+constexpr double kDeintFactor = 1.18;
+
 }  // namespace ttlg

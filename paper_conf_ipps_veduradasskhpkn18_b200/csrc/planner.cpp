@@ -913,6 +913,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB) x every kernel
   // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
+    if (hv == 4) return;  // k_deint forced: no staged / direct candidates
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -1047,6 +1048,74 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) break;
     }
   }
+  // ---- k_deint: [n0, M(, nb)] perm (1 0 (2)) with 2 <= n0 <= 8 (array of
+  // structures -> structure of arrays, the Orthogonal-Arbitrary case whose
+  // input FVI is shorter than one 16-byte vector).  One streaming pass with
+  // 16-byte accesses both ways; its time is the one-pass ideal times the
+  // factor measured for it on B200 (kDeintFactor, model.h) -- it competes
+  // with the ranked candidates below.
+  const int Kd = 16 / P.W;
+  const bool deint_ok =
+      P.W == P.esize && (P.d == 2 || (P.d == 3 && P.p[2] == 2)) && P.p[0] == 1 && P.p[1] == 0 &&
+      P.n[0] >= 2 && P.n[0] <= 8 && P.n[1] % Kd == 0 && P.denseA == P.d - 1 &&
+      P.denseB == P.d - 1 && !forceW && (hv == 0 || hv == 4) &&
+      (force_schema == TTLG_SCHEMA_AUTO || force_schema == TTLG_SCHEMA_OA) &&
+      !(hints && (hints->in_dim >= 0 || hints->in_block > 0 || hints->out_dim >= 0 ||
+                  hints->out_block > 0 || (hints->threads && hints->threads != 256))) &&
+      N / ((int64_t)P.n[0] * Kd) < (1ll << 31);
+  const double deint_t =
+      deint_ok ? kDeintFactor * 2.0 * (double)N * P.W / (dev.hbm_gbs * 1e9) : 1e300;
+  auto make_deint = [&](ttlg_plan_s *pl, ttlg_plan_info *info, double t) {
+    TileParams K;
+    memset(&K, 0, sizeof(K));
+    const int64_t nq = P.n[1] / Kd, chunks = N / ((int64_t)P.n[0] * Kd);
+    K.deint_n0 = (int32_t)P.n[0];
+    K.gdiv[0] = make_fastdiv((uint32_t)nq);
+    K.num_tiles = (uint32_t)chunks;
+    K.V = (int32_t)(P.n[0] * Kd);
+    K.LA = K.V;
+    K.LB = Kd;
+    K.RA = 1;
+    K.RB = (int32_t)P.n[0];
+    K.tpc = 1;
+    Tile T;
+    T.a = 1;
+    T.b = 0;
+    T.ok = true;
+    for (int k = 0; k < P.d; k++) T.t[k] = 1;
+    T.t[0] = P.n[0];
+    T.t[1] = Kd;
+    ModelInput mi;
+    memset(&mi, 0, sizeof(mi));
+    mi.kind = KK_DEINT;
+    mi.schema = TTLG_SCHEMA_OA;
+    mi.W = P.W;
+    mi.N = N;
+    mi.threads = 256;
+    mi.occ = 8;
+    mi.grid = (int)std::min<int64_t>(ceil_div(chunks, 256), (int64_t)dev.sms * 8);
+    if (pl) {
+      pl->kind = KK_DEINT;
+      pl->variant = 4;
+      pl->W = P.W;
+      pl->align = 16;
+      pl->threads = 256;
+      pl->grid = mi.grid;
+      pl->nbytes = N * P.W;
+      pl->spanA = spanA * s;
+      pl->spanB = spanB * s;
+      pl->kp = K;
+    }
+    fill_info(*info, dt, rank, P, T, K, mi, TTLG_SCHEMA_OA, KK_DEINT, t, ncand + 1);
+    info->num_features = 0;
+  };
+  if (deint_ok && listing && sink->n < sink->max) make_deint(nullptr, &sink->out[sink->n++], deint_t);
+  if (deint_ok && hv == 4) {
+    if (sink && sink->shortlist && sink->n < sink->max)
+      make_deint(nullptr, &sink->out[sink->n++], deint_t);
+    make_deint(plan, &plan->info, deint_t);
+    return TTLG_OK;
+  }
   if (ntop == 0) {
     const bool forced = hints && (hints->schema != TTLG_SCHEMA_AUTO || hints->in_dim >= 0 ||
                                   hints->in_block > 0 || hints->out_dim >= 0 ||
@@ -1141,6 +1210,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       fill_info(sink->out[sink->n++], dt, rank, P, e.T, K, e.mi, e.schema, e.kind,
                 predict_ranked_seconds(e.mi, dev), ncand);
     }
+  }
+  if (deint_ok && sink && sink->shortlist && sink->n < sink->max)
+    make_deint(nullptr, &sink->out[sink->n++], deint_t);
+  // auto choice up to n0 = 6: at n0 = 8 k_quad's 4 x 4 register transposes win
+  // (exp49: 5.45 vs 5.13 TB/s), n0 = 7 is unmeasured
+  if (deint_ok && P.n[0] <= 6 && deint_t < win_t) {
+    make_deint(plan, &plan->info, deint_t);
+    return TTLG_OK;
   }
   const Entry &B = pool[win];
   if (B.lin >= 1e299) return TTLG_ERR_INTERNAL;

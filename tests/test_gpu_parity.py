@@ -392,3 +392,38 @@ def test_all_720_rank6_perms(eb):
     for k, perm in enumerate(itertools.permutations(range(6))):
         got, exp, info = _run(ext, list(perm), eb, 3000 + k)
         _assert_equal(got, exp, f"{perm} {info['schema']} {info['kernel']}")
+
+
+# ---- k_deint: [n0, M(, nb)] perm (1 0 (2)), 2 <= n0 <= 8 (AoS -> SoA) ------------------------
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.parametrize("n0", [2, 3, 4, 5, 6, 7, 8])
+def test_deint_forced(n0, eb):
+    K = 16 // eb
+    for ext, perm in (([n0, 11 * K, 7], [1, 0, 2]), ([n0, 250 * K], [1, 0]), ([n0, K, 3], [1, 0, 2])):
+        got, exp, info = _run(ext, perm, eb, 500 + n0, plan_kwargs={"variant": 4}, canary=64)
+        assert info["kernel"] == "deint" and info["schema"] == "OA", info
+        _assert_equal(got, exp, f"deint {ext} {perm}")
+
+
+def test_deint_auto_and_rules():
+    # the config-4 AoS -> SoA cases plan onto k_deint; it does not apply when M is
+    # not a multiple of 16/s or n0 > 8 (forcing it is then TTLG_ERR_UNSUPPORTED)
+    for n0, perm in ((2, [1, 0, 2]), (3, [1, 2, 0]), (5, [1, 0, 2])):
+        got, exp, info = _run([n0, 256, 24], perm, 4, 600 + n0)
+        _assert_equal(got, exp, f"auto {n0} {perm} {info['kernel']}")
+    for ext in ([3, 42, 5], [9, 40, 5]):
+        with pytest.raises(ttlg.TtlgError) as e:
+            ttlg.plan("f32", ext, [1, 0, 2], variant=4)
+        assert e.value.code == 7
+
+
+def test_deint_misaligned_pointers_fall_back():
+    ext, perm = [3, 400, 5], [1, 0, 2]
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(6, n + 1, 4, device=DEV)
+    B = torch.empty(n + 1, dtype=torch.float32, device=DEV)
+    p = ttlg.plan("f32", ext, perm, variant=4)
+    assert p.describe()["kernel"] == "deint"
+    p.execute(A[1:].data_ptr(), B[1:].data_ptr(), torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    _assert_equal(_bits(B[1:]), oracle.transpose(_bits(A[1:]), ext, perm), "deint misaligned")

@@ -212,4 +212,4 @@ def test_plan_candidates_every_config_case():
             cands = ttlg.plan_candidates(dt, c.extents, c.perm)
             assert cands, c.label()
             kinds = {d["kernel"] for d in cands}
-            assert kinds <= {"direct", "tile", "pipe", "quad"}
+            assert kinds <= {"direct", "tile", "pipe", "quad", "deint"}
