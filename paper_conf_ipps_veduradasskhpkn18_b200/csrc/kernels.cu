@@ -364,7 +364,7 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
   }
   __syncthreads();  // tabA, digB, icol, ctx[0] visible
 
-  const int RA = P.RA, RB = P.RB, LA = P.LA, LB = P.LB, V = P.V;
+  const int RB = P.RB, LA = P.LA, LB = P.LB, V = P.V;
   // load walk: element e = tid + k*NT
   const int rA0 = (int)fdiv1(tid, P.fd_LA), xA0 = tid - rA0 * LA;
   const int nA = tid < V ? (int)fdiv1(V - 1 - tid, P.fd_NT) + 1 : 0;

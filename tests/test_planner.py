@@ -213,3 +213,27 @@ def test_plan_candidates_every_config_case():
             assert cands, c.label()
             kinds = {d["kernel"] for d in cands}
             assert kinds <= {"direct", "tile", "pipe", "quad", "deint"}
+
+
+def test_bench_reference_arm_contract():
+    """bench.py --impl reference (the oracle on the host cores) prints ONE JSON
+    line with the driver's keys; runs on a CPU-only host."""
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--impl", "reference",
+                          "--workload", "c1", "--steps", "2", "--warmup", "3",
+                          "--ref-cases-per-step", "4"], capture_output=True, text=True,
+                         timeout=300, cwd=root)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
+              "higher_is_better", "scaling", "vs_baseline", "dtype", "data", "config",
+              "cpu_baseline", "e2e", "impl"):
+        assert k in d, k
+    assert d["impl"] == "reference" and d["value"] > 0 and d["steps"] == 2
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0
