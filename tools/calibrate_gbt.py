@@ -72,6 +72,8 @@ def main():
     ap.add_argument("--lr", type=float, default=0.2)
     args = ap.parse_args()
     rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
+    # k_deint is not ranked by the trees (its time is a measured factor, model.h)
+    rows = [r for r in rows if r["kernel"] in KID]
     co = linear_coefs()
     by = collections.defaultdict(list)
     for r in rows:
