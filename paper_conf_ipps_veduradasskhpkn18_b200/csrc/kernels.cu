@@ -130,6 +130,18 @@ __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
 }
 
+// Programmatic dependent launch (launch(): cudaLaunchAttributeProgrammaticStream-
+// Serialization).  Every kernel lets the next grid in the stream launch as soon
+// as all of its CTAs have started (pdl_trigger at entry), and waits for the
+// previous grid to complete and flush (pdl_wait) before its first global
+// access -- so the next transposition's CTAs fill the SMs freed in this one's
+// last wave and build their tables there, and back-to-back launches lose no
+// launch latency; data dependencies between stream-ordered calls are kept.
+__device__ __forceinline__ void pdl_trigger() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // p + i (i unsigned 32-bit, scaled by sizeof(T)) as ONE wide multiply-add
 // (IMAD.WIDE.U32) instead of a 64-bit add + shift chain
 template <typename T>
@@ -216,8 +228,10 @@ __global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TilePara
   const T *A = reinterpret_cast<const T *>(Av);
   T *B = reinterpret_cast<T *>(Bv);
 
+  pdl_trigger();
   build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
   __syncthreads();
+  pdl_wait();
 
   const int NT = blockDim.x, tid = threadIdx.x;
   const int r0 = (int)fdiv1(tid, P.fd_LB), j0 = tid - r0 * P.LB;
@@ -343,6 +357,7 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
     c.limB = ctx[slot].limB;
     return c;
   };
+  pdl_trigger();
   if (decoder && first < P.num_tiles) put_ctx(0, first);
 
   // A-side tables first (A-row table, icol): the first tile's loads are
@@ -363,6 +378,7 @@ __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const 
     }
   }
   __syncthreads();  // tabA, digB, icol, ctx[0] visible
+  pdl_wait();       // the previous grid in the stream has completed
 
   const int RB = P.RB, LA = P.LA, LB = P.LB, V = P.V;
   // load walk: element e = tid + k*NT
@@ -640,6 +656,7 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
     ctx[slot].limA = c.limA;
     ctx[slot].limB = c.limB;
   };
+  pdl_trigger();
   if (decoder && first < P.num_tiles) put_ctx(0, first);
   // A-row table (global element offset, shared byte offset) first: the first
   // tile's loads are issued before the B-side tables are built, so that
@@ -647,6 +664,7 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
   build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk,
              reinterpret_cast<int2 *>(smem), reinterpret_cast<int *>(smem + P.off_digB), S);
   __syncthreads();  // tabA, digB, ctx[0] visible
+  pdl_wait();       // the previous grid in the stream has completed
 
   const int LB = P.LB, LAc = P.LA / K;  // chunks per A-row
   const int nChunks = P.V / K;
@@ -793,6 +811,8 @@ __global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParam
   uint4 *B = reinterpret_cast<uint4 *>(Bv);
   const uint32_t nq = P.gdiv[0].div;  // M / K
   const uint32_t total = P.num_tiles;
+  pdl_trigger();
+  pdl_wait();
   for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < total;
        c += gridDim.x * blockDim.x) {
     const uint32_t b = fdiv1(c, P.gdiv[0]);
@@ -904,6 +924,20 @@ int kernel_regs(int kind, int W) {
   return r;
 }
 
+// Programmatic dependent launch is opt-in (TTLG_PDL=1): measured on B200
+// (exp55) it speeds up runs of the SAME kernel (per-kernel grouped launches
+// +1.5-4 %, the launch-bound 16^4 suite +3 %) but slows a mixed suite of
+// different kernels by 8 % (TTC-57, small-FVI), so plain stream
+// serialisation is the default.
+static bool pdl_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_PDL");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
 ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
   const void *fn = plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
@@ -933,8 +967,17 @@ ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream
   }
   TileParams kp = plan->kp;
   void *args[] = {(void *)&kp, (void *)&A, (void *)&B};
-  cudaError_t e = cudaLaunchKernel(fn, dim3(plan->grid), dim3(plan->threads), args, smem,
-                                   (cudaStream_t)stream);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(plan->grid);
+  cfg.blockDim = dim3(plan->threads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = (cudaStream_t)stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  cudaError_t e = cudaLaunchKernelExC(&cfg, fn, args);
   if (e != cudaSuccess) return TTLG_ERR_CUDA;
   return TTLG_OK;
 }
