@@ -232,24 +232,35 @@ def _dt_of_tensor(x) -> int:
 
 
 def transpose_tensor(x, perm_t: Sequence[int], out=None, plan_: Optional[Plan] = None):
-    """out = x.permute(perm_t).contiguous(), computed by the library on x's device
-    and current stream."""
+    """out = x.permute(perm_t) materialised, computed by the library on x's device
+    and current stream.  x and out may be strided views (e.g. slices of larger
+    tensors): their strides go to ttlg_plan_strided (the innermost non-unit dim
+    of each must be unit-stride; otherwise TtlgError UNSUPPORTED -- there is no
+    copy fallback).  `out` defaults to a new contiguous tensor."""
     import torch
 
     if not x.is_cuda:
         raise ValueError("transpose_tensor needs a CUDA tensor (no CPU path)")
-    if not x.is_contiguous():
-        raise ValueError("input must be contiguous")
     shape_out = [x.shape[p] for p in perm_t]
     if out is None:
         out = torch.empty(shape_out, dtype=x.dtype, device=x.device)
+    elif list(out.shape) != shape_out or out.dtype != x.dtype or out.device != x.device:
+        raise ValueError("out must have x.permute(perm_t)'s shape, x's dtype and device")
     if x.numel() == 0:
         return out
     ext, perm = torch_to_c(list(x.shape), perm_t)
+    d = len(ext)
     stream = torch.cuda.current_stream(x.device).cuda_stream
     with torch.cuda.device(x.device):
         if plan_ is not None:
             plan_.execute(x.data_ptr(), out.data_ptr(), stream)
-        else:
+        elif x.is_contiguous() and out.is_contiguous():
             transpose(_dt_of_tensor(x), ext, perm, x.data_ptr(), out.data_ptr(), stream)
+        else:
+            # FVI-first strides: input dim k is torch dim d-1-k, output dim i is
+            # out's torch dim d-1-i
+            in_strides = [x.stride(d - 1 - k) for k in range(d)]
+            out_strides = [out.stride(d - 1 - i) for i in range(d)]
+            plan_strided(_dt_of_tensor(x), ext, perm, in_strides, out_strides).execute(
+                x.data_ptr(), out.data_ptr(), stream)
     return out

@@ -258,3 +258,25 @@ def test_gpu_p2p_exchange_virtual_peers(case, world):
             ex.run(A[p * sp.n_local:(p + 1) * sp.n_local], stream)
         torch.cuda.synchronize()
         assert np.array_equal(_torch_bits(B), oracle.transpose(_torch_bits(A), ext, perm))
+
+
+@pytest.mark.gpu
+def test_gpu_transpose_tensor_strided_views():
+    """transpose_tensor on strided views (slices of larger tensors) in and out,
+    through ttlg_plan_strided: equals torch's permute, bit for bit."""
+    import torch
+    from synth import gen_tensor_torch
+    base = gen_tensor_torch(51, 40 * 30 * 24, 8, device="cuda:0").view(40, 30, 24)
+    x = base[3:35, 2:27, 4:20]                       # non-contiguous, innermost unit-stride
+    for perm in ([2, 1, 0], [1, 0, 2], [0, 2, 1], [2, 0, 1]):
+        y = ttlg.transpose_tensor(x, perm)
+        ref = x.permute(*perm).contiguous()
+        assert torch.equal(y.view(torch.int64), ref.view(torch.int64)), perm
+        big = torch.zeros([s + 3 for s in ref.shape], dtype=x.dtype, device="cuda:0")
+        view = big[1:1 + ref.shape[0], 2:2 + ref.shape[1], :ref.shape[2]]
+        ttlg.transpose_tensor(x, perm, out=view)
+        assert torch.equal(view.contiguous().view(torch.int64), ref.view(torch.int64)), perm
+        assert int(torch.count_nonzero(big.view(torch.int64))) == \
+            int(torch.count_nonzero(ref.view(torch.int64)))   # nothing written outside the view
+    with pytest.raises(ttlg.TtlgError):
+        ttlg.transpose_tensor(base[:, :, ::2], [2, 1, 0])   # innermost dim not unit-stride
