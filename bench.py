@@ -565,8 +565,10 @@ def main():
     small = [c for c in cases if c.alg_bytes < 2 * l2_bytes]
     l2_label = ("no flush: every case moves > 2x L2 (%d MB) -- inputs larger than L2"
                 % (l2_bytes // 2 ** 20)) if not small else (
-        "no flush; %d of %d cases move < 2x L2 (%d MB): partly L2-resident, consecutive "
-        "cases use different buffers" % (len(small), len(cases), l2_bytes // 2 ** 20))
+        "no flush; %d of %d cases move < 2x L2 (%d MB): partly L2-resident; %s"
+        % (len(small), len(cases), l2_bytes // 2 ** 20,
+           "cases of one size share one A/B pair" if share else
+           "every case has its own A/B pair"))
     if rank == 0:
         cpu = None
         if not args.no_cpu_baseline and world == 1:
