@@ -43,6 +43,7 @@ def main():
         dt = "f64" if c.elem_bytes == 8 else "f32"
         A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device="cuda")
         B = torch.empty_like(A)
+        torch.cuda.synchronize()  # A is generated on the default stream
         pm = ttlg.plan(dt, c.extents, c.perm)
         pt = ttlg.plan(dt, c.extents, c.perm)
         pt.tune(A.data_ptr(), B.data_ptr(), sp, args.cands)
