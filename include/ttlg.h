@@ -169,14 +169,16 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
                            const void *A, void *B, void *stream);
 
 /* Host-buffer end-to-end path: A_host -> A_dev, transpose, B_dev -> B_host.
- * B is split along its outermost output dimension into up to 32 chunks
- * (>= 16 MiB each); chunk k's input slab is a strided 2-D region of A copied
- * densely (cudaMemcpy2DAsync), transposed with a sub-plan, and its contiguous
- * output range copied back -- H2D, kernels and D2H of successive chunks run on
- * internal streams so both PCIe directions overlap.  Ordered after prior work
- * on `stream`; `stream` waits for completion (no host sync).  A_host/B_host
- * should be pinned; A_dev/B_dev are device scratch of N*s bytes each (A_dev's
- * contents are chunk slabs afterwards, not A).  Small tensors: one stream. */
+ * A is split along one input dim into up to 32 chunks (>= 16 MiB each); the
+ * dim is chosen so that the narrower of the chunk's host-side row widths (its
+ * slab of A, a strided 2-D region; its slab of B, likewise) is as wide as
+ * possible.  Each chunk is copied densely (cudaMemcpy2DAsync), transposed
+ * with a sub-plan, and copied back -- H2D, kernels and D2H of successive
+ * chunks run on internal streams so both PCIe directions overlap.  Ordered
+ * after prior work on `stream`; `stream` waits for completion (no host sync).
+ * A_host/B_host should be pinned; A_dev/B_dev are device scratch of N*s bytes
+ * each (their contents are chunk slabs afterwards, not A / B).  Small or
+ * unsplittable tensors: one stream, in order.  Dense plans only. */
 ttlg_status ttlg_execute_host(ttlg_plan_t plan, const void *A_host, void *B_host, void *A_dev,
                               void *B_dev, void *stream);
 

@@ -166,12 +166,16 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
 
 
 // ---- host-buffer pipeline (ttlg_execute_host) --------------------------------
-// B is split along its outermost output dim o_{d-1} = input dim q into C chunks.
-// Chunk k needs the A slab i_q in [q0, q0+cq): a 2-D strided region of A
-// (outer x (inner*cq) elements, pitch inner*n_q), copied densely with
-// cudaMemcpy2DAsync; its transposition is the same permutation on extents with
-// n_q -> cq, and its output is a contiguous range of B.  H2D, kernel and D2H of
-// successive chunks run on three internal streams joined by events, so the
+// A is split along one input dim cd into C chunks.  Chunk k's input slab is
+// i_cd in [c0, c0+cc): rows of (prod_{j<cd} n_j) * cc elements at pitch
+// prod_{j<=cd} n_j (one contiguous block when cd = d-1), copied densely with
+// cudaMemcpy2DAsync; its transposition is the same permutation on extents
+// with n_cd -> cc, and its output is B restricted to o_pos in [c0, c0+cc)
+// (pos = position of cd in perm): rows of (prod_{i<pos} m_i) * cc elements at
+// pitch prod_{i<=pos} m_i (contiguous when pos = d-1).  cd maximises the
+// narrower of the two row widths (PCIe DMA of narrow rows is slow), so e.g. a
+// full reversal splits a middle dim.  H2D, kernel and D2H of successive
+// chunks run on three internal streams joined by events, so the
 // host->device and device->host PCIe directions overlap.
 namespace {
 constexpr int kMaxChunks = 32;
@@ -211,26 +215,31 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
   for (int i = 0; i < d; i++) m[i] = p->ext[p->perm[i]];
   const int64_t nbytes = N * esize;
   if (p->device < 0) return TTLG_ERR_DEVICE;
-  // Two ways to split into chunks; each keeps one side contiguous and makes
-  // the other a 2-D strided copy.  Mode B splits B's outermost dim (input dim
-  // q = perm[d-1]): H2D rows of inner_q*c elements.  Mode A splits A's
-  // outermost dim (d-1, output position k): D2H rows of inner_B*c elements.
-  // Pick the mode with the wider rows (PCIe DMA of narrow rows is slow).
-  const int q = p->perm[d - 1];
-  int kpos = 0;
-  while (p->perm[kpos] != d - 1) kpos++;
-  int64_t inner_q = 1, inner_b = 1;
-  for (int k = 0; k < q; k++) inner_q *= p->ext[k];
-  for (int i = 0; i < kpos; i++) inner_b *= m[i];
-  const int64_t nq = p->ext[q], na = p->ext[d - 1];
   const int64_t want = std::min<int64_t>((int64_t)kMaxChunks, nbytes / (16ll << 20));
-  const int64_t CB = std::min<int64_t>(nq, want), CA = std::min<int64_t>(na, want);
-  const double wB = CB >= 2 ? (double)inner_q * (nq / CB) * esize : 0.0;
-  const double wA = CA >= 2 ? (double)inner_b * (na / CA) * esize : 0.0;
-  const bool modeA = wA > wB;
-  const int64_t C = modeA ? CA : CB;
-  const double width_min = modeA ? wA : wB;
-  HostPipe *hp = (C >= 2 && width_min >= 2048.0) ? host_pipe(p->device) : nullptr;
+  // the split dim: widest narrower row (contiguous side = unbounded)
+  int cd = -1, pos = -1;
+  int64_t C = 0;
+  double best = 0.0;
+  for (int k = 0; k < d; k++) {
+    const int64_t Ck = std::min<int64_t>(p->ext[k], want);
+    if (Ck < 2) continue;
+    int pk = 0;
+    while (p->perm[pk] != k) pk++;
+    int64_t inA = 1, inB = 1;
+    for (int j = 0; j < k; j++) inA *= p->ext[j];
+    for (int i = 0; i < pk; i++) inB *= m[i];
+    const int64_t cc = p->ext[k] / Ck;
+    const double wA = (k == d - 1) ? 1e300 : (double)inA * cc * esize;
+    const double wB = (pk == d - 1) ? 1e300 : (double)inB * cc * esize;
+    const double w = std::min(wA, wB);
+    if (w > best) {
+      best = w;
+      cd = k;
+      pos = pk;
+      C = Ck;
+    }
+  }
+  HostPipe *hp = (cd >= 0 && best >= 2048.0) ? host_pipe(p->device) : nullptr;
   if (!hp) {  // small, unsplittable or too narrow: one stream, in order
     if (cudaMemcpyAsync(A_dev, A_host, (size_t)nbytes, cudaMemcpyHostToDevice, s) != cudaSuccess)
       return TTLG_ERR_CUDA;
@@ -241,8 +250,11 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
     return TTLG_OK;
   }
   std::lock_guard<std::mutex> g(hp->mu);
-  const int cd = modeA ? d - 1 : q;  // the split input dim
   const int64_t nc = p->ext[cd];
+  int64_t inA = 1, inB = 1;
+  for (int j = 0; j < cd; j++) inA *= p->ext[j];
+  for (int i = 0; i < pos; i++) inB *= m[i];
+  const int64_t rowsA = N / (inA * nc), rowsB = N / (inB * nc);
   // at most two distinct chunk extents -> two sub-plans
   const int64_t base = nc / C, rem = nc % C;
   ttlg_plan_s sub[2];
@@ -261,22 +273,18 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
   cudaStreamWaitEvent(hp->comp, hp->start, 0);
   cudaStreamWaitEvent(hp->d2h, hp->start, 0);
   const int64_t per = N / nc;  // elements per index of the split dim
-  unsigned char *Ah = (unsigned char *)A_host, *Bh = (unsigned char *)B_host;
+  const unsigned char *Ah = (const unsigned char *)A_host;
+  unsigned char *Bh = (unsigned char *)B_host;
   int64_t c0 = 0;
   for (int64_t k = 0; k < C; k++) {
     const int v = k < rem ? 1 : 0;
     const int64_t cc = subc[v];
     unsigned char *a_slab = (unsigned char *)A_dev + c0 * per * esize;
     unsigned char *b_chunk = (unsigned char *)B_dev + c0 * per * esize;
-    cudaError_t e;
-    if (modeA) {  // contiguous A slab
-      e = cudaMemcpyAsync(a_slab, Ah + c0 * per * esize, (size_t)(cc * per * esize),
-                          cudaMemcpyHostToDevice, hp->h2d);
-    } else {      // strided A slab: rows of inner_q*cc elements
-      const size_t w = (size_t)(inner_q * cc * esize);
-      e = cudaMemcpy2DAsync(a_slab, w, Ah + c0 * inner_q * esize, (size_t)(inner_q * nq * esize), w,
-                            (size_t)(N / (inner_q * nq)), cudaMemcpyHostToDevice, hp->h2d);
-    }
+    const size_t wa = (size_t)(inA * cc * esize), wb = (size_t)(inB * cc * esize);
+    cudaError_t e = cudaMemcpy2DAsync(a_slab, wa, Ah + c0 * inA * esize,
+                                      (size_t)(inA * nc * esize), wa, (size_t)rowsA,
+                                      cudaMemcpyHostToDevice, hp->h2d);
     if (e != cudaSuccess) return TTLG_ERR_CUDA;
     cudaEventRecord(hp->evA[k], hp->h2d);
     cudaStreamWaitEvent(hp->comp, hp->evA[k], 0);
@@ -284,14 +292,8 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
     if (st != TTLG_OK) return st;
     cudaEventRecord(hp->evB[k], hp->comp);
     cudaStreamWaitEvent(hp->d2h, hp->evB[k], 0);
-    if (modeA) {  // the chunk's B rows are strided in B: rows of inner_b*cc elements
-      const size_t w = (size_t)(inner_b * cc * esize);
-      e = cudaMemcpy2DAsync(Bh + c0 * inner_b * esize, (size_t)(inner_b * na * esize), b_chunk, w, w,
-                            (size_t)(N / (inner_b * na)), cudaMemcpyDeviceToHost, hp->d2h);
-    } else {      // contiguous range of B
-      e = cudaMemcpyAsync(Bh + c0 * per * esize, b_chunk, (size_t)(cc * per * esize),
-                          cudaMemcpyDeviceToHost, hp->d2h);
-    }
+    e = cudaMemcpy2DAsync(Bh + c0 * inB * esize, (size_t)(inB * nc * esize), b_chunk, wb, wb,
+                          (size_t)rowsB, cudaMemcpyDeviceToHost, hp->d2h);
     if (e != cudaSuccess) return TTLG_ERR_CUDA;
     c0 += cc;
   }

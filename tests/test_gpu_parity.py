@@ -268,7 +268,9 @@ def test_full_exactly_once_index_encoding():
                                          ([40, 50, 60], [0, 2, 1], 8),          # small: 1 stream
                                          ([33, 17, 2048, 9], [2, 3, 0, 1], 4),
                                          ([512, 64, 8, 128], [1, 3, 2, 0], 4),  # mode A
-                                         ([16, 4, 16, 20, 16, 80], [5, 4, 3, 2, 1, 0], 8)])
+                                         ([16, 4, 16, 20, 16, 80], [5, 4, 3, 2, 1, 0], 8),
+                                         ([80, 64, 80, 64], [3, 2, 1, 0], 8),   # reversal: middle split
+                                         ([40, 30, 50, 70], [1, 3, 0, 2], 4)])
 def test_execute_host_pipeline(ext, perm, eb):
     """ttlg_execute_host: chunked H2D / kernel / D2H over internal streams."""
     n = int(np.prod(ext))
