@@ -842,6 +842,71 @@ __global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParam
   }
 }
 
+// k_inter (the mirror image: structure of arrays -> array of structures): the
+// fused problem [M, n1] perm (1 0), or [M, n1, nb] perm (1 0 2), with
+// N1 = n1 <= 8 and M a multiple of K.  A thread's slice is K x N1: column
+// block q of each of the N1 input rows, A[M*(r + N1*b) + K*q] (r < N1), ONE
+// 16-byte vector each (every load instruction: 512 contiguous bytes across
+// the warp), regrouped in registers (position u of row r is output element
+// u*N1 + r) and written as ONE contiguous output run of N1*K elements,
+// B[N1*(K*q + M*b) ...], as N1 16-byte vectors.
+template <int S, int N1>
+__global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParams P,
+                                               const void *__restrict__ Av,
+                                               void *__restrict__ Bv) {
+  constexpr int K = 16 / S;
+  constexpr int E = N1 * K;
+  constexpr int WPE = S / 4;
+  const uint4 *A = reinterpret_cast<const uint4 *>(Av);
+  uint4 *B = reinterpret_cast<uint4 *>(Bv);
+  const uint32_t nq = P.gdiv[0].div;  // M / K
+  const uint32_t total = P.num_tiles;
+  pdl_trigger();
+  pdl_wait();
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < total;
+       c += gridDim.x * blockDim.x) {
+    const uint32_t b = fdiv1(c, P.gdiv[0]);
+    const uint32_t q = c - b * nq;
+    uint32_t w[E * WPE];  // w[(r*K + u)*WPE + h]: position u of row r
+    const uint4 *src = A + ((size_t)b * N1) * nq + q;
+#pragma unroll
+    for (int r = 0; r < N1; r++) {
+      const uint4 v = __ldcs(src + (size_t)r * nq);
+      w[4 * r + 0] = v.x;
+      w[4 * r + 1] = v.y;
+      w[4 * r + 2] = v.z;
+      w[4 * r + 3] = v.w;
+    }
+    uint4 *dst = B + (size_t)c * N1;  // output run: N1 vectors (the batch is contiguous)
+#pragma unroll
+    for (int i = 0; i < N1; i++) {
+      uint32_t o[4];
+#pragma unroll
+      for (int x = 0; x < K; x++) {
+        const int e = i * K + x;           // output element index in the run
+        const int u = e / N1, r = e % N1;  // position u of input row r
+#pragma unroll
+        for (int h = 0; h < WPE; h++) o[x * WPE + h] = w[(r * K + u) * WPE + h];
+      }
+      __stcs(dst + i, make_uint4(o[0], o[1], o[2], o[3]));
+    }
+  }
+}
+
+template <int S>
+static const void *inter_ptr_s(int n1) {
+  switch (n1) {
+    case 2: return (const void *)k_inter<S, 2>;
+    case 3: return (const void *)k_inter<S, 3>;
+    case 4: return (const void *)k_inter<S, 4>;
+    case 5: return (const void *)k_inter<S, 5>;
+    case 6: return (const void *)k_inter<S, 6>;
+    case 7: return (const void *)k_inter<S, 7>;
+    case 8: return (const void *)k_inter<S, 8>;
+  }
+  return nullptr;
+}
+
 template <int S>
 static const void *deint_ptr_s(int n0) {
   switch (n0) {
@@ -857,6 +922,9 @@ static const void *deint_ptr_s(int n0) {
 }
 static const void *deint_ptr(int W, int n0) {
   return W == 8 ? deint_ptr_s<8>(n0) : (W == 4 ? deint_ptr_s<4>(n0) : nullptr);
+}
+static const void *inter_ptr(int W, int n1) {
+  return W == 8 ? inter_ptr_s<8>(n1) : (W == 4 ? inter_ptr_s<4>(n1) : nullptr);
 }
 
 // ---------------------------------------------------------------------------
@@ -942,7 +1010,8 @@ ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream
   const void *fn = plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
                        : plan->kind == KK_DEINT
-                             ? deint_ptr(plan->W, plan->kp.deint_n0)
+                             ? (plan->kp.deint_inter ? inter_ptr(plan->W, plan->kp.deint_n0)
+                                                     : deint_ptr(plan->W, plan->kp.deint_n0))
                              : kernel_ptr(plan->kind, plan->W, plan->kp.rsB == 0,
                                           plan->kp.xtab != 0);
   if (!fn) return TTLG_ERR_INTERNAL;

@@ -1055,36 +1055,43 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // factor measured for it on B200 (kDeintFactor, model.h) -- it competes
   // with the ranked candidates below.
   const int Kd = 16 / P.W;
+  // k_deint: the small extent is dim 0 (AoS -> SoA); k_inter: dim 1 (SoA -> AoS)
+  const bool two_d = P.W == P.esize && (P.d == 2 || (P.d == 3 && P.p[2] == 2)) && P.p[0] == 1 &&
+                     P.p[1] == 0;
+  const bool small0 = two_d && P.n[0] >= 2 && P.n[0] <= 8 && P.n[1] % Kd == 0;
+  const bool small1 = two_d && !small0 && P.n[1] >= 2 && P.n[1] <= 8 && P.n[0] % Kd == 0;
+  const bool inter = small1;
+  const int64_t dsmall = inter ? P.n[1] : P.n[0], dlong = inter ? P.n[0] : P.n[1];
   const bool deint_ok =
-      P.W == P.esize && (P.d == 2 || (P.d == 3 && P.p[2] == 2)) && P.p[0] == 1 && P.p[1] == 0 &&
-      P.n[0] >= 2 && P.n[0] <= 8 && P.n[1] % Kd == 0 && P.denseA == P.d - 1 &&
-      P.denseB == P.d - 1 && !forceW && (hv == 0 || hv == 4) &&
+      (small0 || small1) && P.denseA == P.d - 1 && P.denseB == P.d - 1 && !forceW &&
+      (hv == 0 || hv == 4) &&
       (force_schema == TTLG_SCHEMA_AUTO || force_schema == TTLG_SCHEMA_OA) &&
       !(hints && (hints->in_dim >= 0 || hints->in_block > 0 || hints->out_dim >= 0 ||
                   hints->out_block > 0 || (hints->threads && hints->threads != 256))) &&
-      N / ((int64_t)P.n[0] * Kd) < (1ll << 31);
+      N / (dsmall * Kd) < (1ll << 31);
   const double deint_t =
       deint_ok ? kDeintFactor * 2.0 * (double)N * P.W / (dev.hbm_gbs * 1e9) : 1e300;
   auto make_deint = [&](ttlg_plan_s *pl, ttlg_plan_info *info, double t) {
     TileParams K;
     memset(&K, 0, sizeof(K));
-    const int64_t nq = P.n[1] / Kd, chunks = N / ((int64_t)P.n[0] * Kd);
-    K.deint_n0 = (int32_t)P.n[0];
+    const int64_t nq = dlong / Kd, chunks = N / (dsmall * Kd);
+    K.deint_n0 = (int32_t)dsmall;
+    K.deint_inter = inter ? 1 : 0;
     K.gdiv[0] = make_fastdiv((uint32_t)nq);
     K.num_tiles = (uint32_t)chunks;
-    K.V = (int32_t)(P.n[0] * Kd);
-    K.LA = K.V;
-    K.LB = Kd;
-    K.RA = 1;
-    K.RB = (int32_t)P.n[0];
+    K.V = (int32_t)(dsmall * Kd);
+    K.LA = inter ? Kd : K.V;
+    K.LB = inter ? K.V : Kd;
+    K.RA = inter ? (int32_t)dsmall : 1;
+    K.RB = inter ? 1 : (int32_t)dsmall;
     K.tpc = 1;
     Tile T;
-    T.a = 1;
-    T.b = 0;
+    T.a = inter ? 0 : 1;
+    T.b = inter ? 1 : 0;
     T.ok = true;
     for (int k = 0; k < P.d; k++) T.t[k] = 1;
-    T.t[0] = P.n[0];
-    T.t[1] = Kd;
+    T.t[0] = inter ? Kd : P.n[0];
+    T.t[1] = inter ? P.n[1] : Kd;
     ModelInput mi;
     memset(&mi, 0, sizeof(mi));
     mi.kind = KK_DEINT;
@@ -1215,7 +1222,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     make_deint(nullptr, &sink->out[sink->n++], deint_t);
   // auto choice up to n0 = 6: at n0 = 8 k_quad's 4 x 4 register transposes win
   // (exp49: 5.45 vs 5.13 TB/s), n0 = 7 is unmeasured
-  if (deint_ok && P.n[0] <= 6 && deint_t < win_t) {
+  if (deint_ok && dsmall <= 6 && deint_t < win_t) {
     make_deint(plan, &plan->info, deint_t);
     return TTLG_OK;
   }

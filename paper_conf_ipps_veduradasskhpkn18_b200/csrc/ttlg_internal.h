@@ -47,7 +47,8 @@ enum KernelKind : int32_t {
   KK_TILE = 1,    // OD / OA / FMS: register-staged, one tile per CTA (k_tile)
   KK_PIPE = 2,    // OD / OA / FMS: cp.async double-buffered, persistent (k_pipe)
   KK_QUAD = 3,    // OD: 16-byte chunks in and out, K x K register transpose (k_quad)
-  KK_DEINT = 4,   // OA, input FVI <= 8 elements: [n0, M(, nb)] -> [M, n0(, nb)] (k_deint)
+  KK_DEINT = 4,   // [n0, M(, nb)] perm (1 0 (2)) with n0 <= 8 (k_deint, AoS -> SoA) or
+                  // n1 <= 8 (k_inter, SoA -> AoS): 16-byte accesses both ways
   KK_NUM = 5,
 };
 
@@ -109,7 +110,8 @@ struct TileParams {
   FastDiv fd_LA, fd_LB, fd_NT, fd_rsB;  // per-thread walk setup without hardware division
   int32_t qk, qnj;             // k_quad: chunk elements K (0: scalar kernels), column slots
   int32_t tpc;                 // tiles per CTA (consecutive tile indices)
-  int32_t deint_n0;            // k_deint: n0 (the structure size, 2..8)
+  int32_t deint_n0;            // k_deint: n0 (the structure size, 2..8); k_inter: n1
+  int32_t deint_inter;         // 1: k_inter (SoA -> AoS, the small dim is dim 1)
 };
 
 struct Problem {

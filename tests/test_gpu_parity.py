@@ -429,3 +429,19 @@ def test_deint_misaligned_pointers_fall_back():
     p.execute(A[1:].data_ptr(), B[1:].data_ptr(), torch.cuda.current_stream().cuda_stream)
     torch.cuda.synchronize()
     _assert_equal(_bits(B[1:]), oracle.transpose(_bits(A[1:]), ext, perm), "deint misaligned")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.parametrize("n1", [2, 3, 4, 5, 6, 7, 8])
+def test_inter_forced(n1, eb):
+    """k_inter (SoA -> AoS): [M, n1(, nb)] perm (1 0 (2)) with the small extent on dim 1."""
+    K = 16 // eb
+    for ext, perm in (([11 * K, n1, 7], [1, 0, 2]), ([250 * K, n1], [1, 0]), ([K, n1, 3], [1, 0, 2])):
+        got, exp, info = _run(ext, perm, eb, 700 + n1, plan_kwargs={"variant": 4}, canary=64)
+        # both extents small ([K, n1, 3] with n1 a multiple of K): the AoS -> SoA form wins
+        both = ext[0] <= 8 and n1 % K == 0
+        assert info["kernel"] == "deint" and (both or info["in_run"] == K), info
+        _assert_equal(got, exp, f"inter {ext} {perm}")
+    # the auto plan for an SoA -> AoS case with a tiny structure
+    got, exp, info = _run([4096, n1, 8], [1, 0, 2], eb, 800 + n1)
+    _assert_equal(got, exp, f"auto {info['kernel']}")
