@@ -795,9 +795,10 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
 // output is N0 runs of K elements, B[M*(r + N0*b) + K*q ...] for r < N0, each
 // written as ONE 16-byte vector after an in-register regrouping (element
 // u*N0 + r of the input run is position u of output row r).  No shared
-// memory, no shuffles: the warp's N0 load instructions together cover 512*N0
-// contiguous bytes (the later ones hit the lines the first ones brought into
-// L1), and every store instruction writes 512 contiguous bytes.
+// memory beyond a per-warp staging buffer, no shuffles: the warp's N0 load
+// instructions each read 512 contiguous bytes (staged through shared memory
+// to give every lane its own run), and every store instruction writes 512
+// contiguous bytes.
 // Parameters ride in TileParams: deint_n0 = N0, gdiv[0] = fastdiv(M/K),
 // num_tiles = chunks.
 template <int S, int N0>
@@ -811,45 +812,57 @@ __global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParam
   uint4 *B = reinterpret_cast<uint4 *>(Bv);
   const uint32_t nq = P.gdiv[0].div;  // M / K
   const uint32_t total = P.num_tiles;
+  __shared__ uint4 stage[256 * N0];
   pdl_trigger();
   pdl_wait();
-  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < total;
-       c += gridDim.x * blockDim.x) {
-    const uint32_t b = fdiv1(c, P.gdiv[0]);
-    const uint32_t q = c - b * nq;
-    // input run: N0 vectors starting at vector N0 * c (the batch is contiguous)
-    uint32_t w[E * WPE];
-    const uint4 *src = wadd(A, 0u) + (size_t)c * N0;
+  // whole warps iterate together (the staging is warp-wide)
+  const uint32_t lane = threadIdx.x & 31;
+  uint4 *wbuf = stage + (threadIdx.x >> 5) * 32 * N0;
+  const uint32_t nthreads = gridDim.x * blockDim.x;
+  const uint32_t span = (total + 31) / 32 * 32;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < span; c += nthreads) {
+    // the warp's 32 input runs are contiguous (consecutive c): N0 coalesced
+    // load instructions of 512 contiguous bytes each, staged in shared memory
+    // (16-byte slots XOR-swizzled by their 128-byte row: both phases
+    // conflict-free), then every lane reads back its own run
+    const uint32_t c0 = c - lane;
+    const uint32_t nvalid = min(32u, total - c0) * N0;
+    const uint4 *src = A + (size_t)c0 * N0;
 #pragma unroll
     for (int i = 0; i < N0; i++) {
-      const uint4 v = __ldcs(src + i);
+      const uint32_t slot = i * 32 + lane;
+      if (slot < nvalid) wbuf[slot ^ ((slot >> 3) & 7)] = __ldcs(src + slot);
+    }
+    __syncwarp();
+    uint32_t w[E * WPE];
+#pragma unroll
+    for (int i = 0; i < N0; i++) {
+      const uint32_t slot = lane * N0 + i;
+      const uint4 v = wbuf[slot ^ ((slot >> 3) & 7)];
       w[4 * i + 0] = v.x;
       w[4 * i + 1] = v.y;
       w[4 * i + 2] = v.z;
       w[4 * i + 3] = v.w;
     }
-    // output row r of batch b: vector index (r + N0*b) * (M/K) + q
-    uint4 *dst = B + ((size_t)b * N0) * nq + q;
+    __syncwarp();
+    if (c < total) {
+      const uint32_t b = fdiv1(c, P.gdiv[0]);
+      const uint32_t q = c - b * nq;
+      // output row r of batch b: vector index (r + N0*b) * (M/K) + q
+      uint4 *dst = B + ((size_t)b * N0) * nq + q;
 #pragma unroll
-    for (int r = 0; r < N0; r++) {
-      uint32_t o[4];
+      for (int r = 0; r < N0; r++) {
+        uint32_t o[4];
 #pragma unroll
-      for (int u = 0; u < K; u++)
+        for (int u = 0; u < K; u++)
 #pragma unroll
-        for (int h = 0; h < WPE; h++) o[u * WPE + h] = w[(u * N0 + r) * WPE + h];
-      __stcs(dst + (size_t)r * nq, make_uint4(o[0], o[1], o[2], o[3]));
+          for (int h = 0; h < WPE; h++) o[u * WPE + h] = w[(u * N0 + r) * WPE + h];
+        __stcs(dst + (size_t)r * nq, make_uint4(o[0], o[1], o[2], o[3]));
+      }
     }
   }
 }
 
-// k_inter (the mirror image: structure of arrays -> array of structures): the
-// fused problem [M, n1] perm (1 0), or [M, n1, nb] perm (1 0 2), with
-// N1 = n1 <= 8 and M a multiple of K.  A thread's slice is K x N1: column
-// block q of each of the N1 input rows, A[M*(r + N1*b) + K*q] (r < N1), ONE
-// 16-byte vector each (every load instruction: 512 contiguous bytes across
-// the warp), regrouped in registers (position u of row r is output element
-// u*N1 + r) and written as ONE contiguous output run of N1*K elements,
-// B[N1*(K*q + M*b) ...], as N1 16-byte vectors.
 template <int S, int N1>
 __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParams P,
                                                const void *__restrict__ Av,
@@ -861,12 +874,18 @@ __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParam
   uint4 *B = reinterpret_cast<uint4 *>(Bv);
   const uint32_t nq = P.gdiv[0].div;  // M / K
   const uint32_t total = P.num_tiles;
+  __shared__ uint4 stage[256 * N1];
   pdl_trigger();
   pdl_wait();
-  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < total;
-       c += gridDim.x * blockDim.x) {
-    const uint32_t b = fdiv1(c, P.gdiv[0]);
-    const uint32_t q = c - b * nq;
+  // whole warps iterate together (the staging is warp-wide); lanes past the
+  // end load nothing and store nothing
+  const uint32_t nthreads = gridDim.x * blockDim.x;
+  const uint32_t span = (total + 31) / 32 * 32;
+  for (uint32_t c = blockIdx.x * blockDim.x + threadIdx.x; c < span; c += nthreads) {
+    const bool live = c < total;
+    const uint32_t cl = live ? c : total - 1;
+    const uint32_t b = fdiv1(cl, P.gdiv[0]);
+    const uint32_t q = cl - b * nq;
     uint32_t w[E * WPE];  // w[(r*K + u)*WPE + h]: position u of row r
     const uint4 *src = A + ((size_t)b * N1) * nq + q;
 #pragma unroll
@@ -877,7 +896,12 @@ __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParam
       w[4 * r + 2] = v.z;
       w[4 * r + 3] = v.w;
     }
-    uint4 *dst = B + (size_t)c * N1;  // output run: N1 vectors (the batch is contiguous)
+    // the warp's 32 output runs are contiguous (consecutive c): stage them in
+    // shared memory (16-byte slots XOR-swizzled by their 128-byte row, both
+    // phases conflict-free) and write them back as N1 coalesced store
+    // instructions of 512 contiguous bytes each
+    const uint32_t lane = threadIdx.x & 31;
+    uint4 *wbuf = stage + (threadIdx.x >> 5) * 32 * N1;
 #pragma unroll
     for (int i = 0; i < N1; i++) {
       uint32_t o[4];
@@ -888,8 +912,19 @@ __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParam
 #pragma unroll
         for (int h = 0; h < WPE; h++) o[x * WPE + h] = w[(r * K + u) * WPE + h];
       }
-      __stcs(dst + i, make_uint4(o[0], o[1], o[2], o[3]));
+      const uint32_t slot = lane * N1 + i;
+      wbuf[slot ^ ((slot >> 3) & 7)] = make_uint4(o[0], o[1], o[2], o[3]);
     }
+    __syncwarp();
+    const uint32_t c0 = c - lane;  // chunk of lane 0
+    const uint32_t nvalid = min(32u, total - c0) * N1;
+    uint4 *dst = B + (size_t)c0 * N1;
+#pragma unroll
+    for (int i = 0; i < N1; i++) {
+      const uint32_t slot = i * 32 + lane;
+      if (slot < nvalid) __stcs(dst + slot, wbuf[slot ^ ((slot >> 3) & 7)]);
+    }
+    __syncwarp();
   }
 }
 
