@@ -1220,9 +1220,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   }
   if (deint_ok && sink && sink->shortlist && sink->n < sink->max)
     make_deint(nullptr, &sink->out[sink->n++], deint_t);
-  // auto choice up to n0 = 6: at n0 = 8 k_quad's 4 x 4 register transposes win
-  // (exp49: 5.45 vs 5.13 TB/s), n0 = 7 is unmeasured
-  if (deint_ok && dsmall <= 6 && deint_t < win_t) {
+  // with the warp-staged loads k_deint also wins at n0 = 7, 8 (exp66: 5.6-6.0
+  // vs 4.8-5.3 TB/s for the staged kernels / k_quad)
+  if (deint_ok && deint_t < win_t) {
     make_deint(plan, &plan->info, deint_t);
     return TTLG_OK;
   }
