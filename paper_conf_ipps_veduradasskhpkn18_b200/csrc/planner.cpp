@@ -613,6 +613,7 @@ static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) 
 // directly, including the balanced ceil(n/ceil(n/t)) variants).
 static const int64_t kRunTargets[] = {64, 128, 256, 512, 1024, 2048, 4096, 0};
 static const int64_t kTileTargets[] = {4096, 8192, 16384, 32768, 65536, 131072, 0};
+static const int64_t kDeepTargets[] = {8192, 16384, 32768, 65536, 0};
 
 static int cand_blocks(int64_t n, int64_t pre, int W, int64_t *out, int64_t forced,
                        const int64_t *targets) {
@@ -910,6 +911,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (ntop == kShort) admit = pool[order[kShort - 1]].lin;
   };
 
+  bool pipe_only = false;  // deep tiles: k_pipe candidates only
   // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB) x every kernel
   // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
@@ -961,7 +963,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       kinds[nk++] = KK_QUAD;
     } else {
       if (hv == 3) return;
-      if (hv != 2) kinds[nk++] = KK_TILE;
+      if (hv != 2 && !pipe_only) kinds[nk++] = KK_TILE;
       if (hv != 1) kinds[nk++] = KK_PIPE;
     }
     // block sizes: 256 and 512, plus (staged kernels) the multiple of the
@@ -1020,6 +1022,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (P.d > 1) {
     // ---- staged (OD / OA / FMS): enumerate input and output groups
     int64_t preA = 1;
+    int a_stop = -1;
     for (int a = 0; a <= P.denseA; a++) {
       const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0,
                                   kRunTargets);
@@ -1045,7 +1048,34 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         if (preB * P.W >= 4096 && !(hints && hints->out_dim > b)) break;
       }
       preA *= P.n[a];
-      if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) break;
+      if (preA * P.W >= 4096 && !(hints && hints->in_dim > a)) {
+        a_stop = a;
+        break;
+      }
+    }
+    // deep tiles: when the leading input block 0..a_stop (>= 4 KB) is also the
+    // leading output block (perm maps it onto itself, e.g. 1 0 2 4 3 5), the
+    // block is contiguous in both tensors; one more input dim blocked by tile
+    // volume gives tiles whose input run spans several such blocks and whose
+    // B-rows are adjacent in B (exp51: 24^6 1 0 2 4 3 5 4.1 -> 6.1 TB/s).
+    // k_pipe only: deep k_tile geometries were mis-ranked (exp53).
+    bool closed = a_stop >= 0 && a_stop + 1 <= P.denseA && !hints;
+    for (int i = 0; closed && i <= a_stop; i++) closed = P.p[i] <= a_stop;
+    if (closed) {
+      const int a = a_stop + 1;
+      const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, 0, kDeepTargets);
+      int64_t preB = 1;
+      pipe_only = true;
+      for (int b = 0; b <= P.denseB; b++) {
+        const int pb = P.p[b];
+        if (pb == a) break;  // the deep dim itself closes no output group here
+        const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, 0, kRunTargets);
+        for (int i = 0; i < nbA; i++)
+          for (int j = 0; j < nbB; j++) consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
+        preB *= P.n[pb];
+        if (preB * P.W >= 4096) break;
+      }
+      pipe_only = false;
     }
   }
   // ---- k_deint: [n0, M(, nb)] perm (1 0 (2)) with 2 <= n0 <= 8 (array of

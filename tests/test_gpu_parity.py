@@ -445,3 +445,10 @@ def test_inter_forced(n1, eb):
     # the auto plan for an SoA -> AoS case with a tiny structure
     got, exp, info = _run([4096, n1, 8], [1, 0, 2], eb, 800 + n1)
     _assert_equal(got, exp, f"auto {info['kernel']}")
+
+
+@pytest.mark.parametrize("ext", [[24, 24, 12, 4, 3, 2], [24, 24, 24, 3, 2, 2]])
+def test_closed_block_deep_tiles(ext):
+    """1 0 2 4 3 5 with a >= 4 KB leading block: the deep k_pipe tiles."""
+    got, exp, info = _run(ext, [1, 0, 2, 4, 3, 5], 8, 901, canary=64)
+    _assert_equal(got, exp, f"deep {info['kernel']} {info['tile_extents']}")

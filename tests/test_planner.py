@@ -237,3 +237,17 @@ def test_bench_reference_arm_contract():
     assert d["impl"] == "reference" and d["value"] > 0 and d["steps"] == 2
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0
+
+
+def test_deep_tiles_only_for_closed_leading_blocks():
+    """Input runs one dim past 4 KB (k_pipe only) are enumerated only when the
+    leading input block is also the leading output block (1 0 2 4 3 5 family)."""
+    d = ttlg.plan("f64", [24] * 6, [1, 0, 2, 4, 3, 5]).describe()
+    assert d["kernel"] == "pipe" and d["in_dim"] == 2 and d["tile_extents"][2] > 1
+    # not closed (perm[0..1] = 2 0): no deep candidate may appear
+    for c in ttlg.plan_candidates("f64", [16, 4, 16, 20, 16, 80], [2, 0, 4, 1, 5, 3]):
+        fe, te = c["fused_extents"], c["tile_extents"]
+        pre = 1
+        for k in range(c["in_dim"]):
+            pre *= fe[k]
+        assert pre * 8 < 4096 or c["in_dim"] == 0, c
