@@ -29,10 +29,16 @@ def main(launches="gpurun_out/launches.csv", bench="gpurun_out/bench.json",
     tot = sum(a[2] for a in acc.values())
     res = {k: a[0] / a[1] for k, a in acc.items()}
     share = {k: a[2] / tot for k, a in acc.items()}
-    json.dump({workload: res, "ncu_time_share": share,
-               "source": "ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,"
-                         "dram__bytes_write.sum, one bench step (profiles/*launches.csv)"},
-              open(out, "w"), indent=1)
+    import os
+    doc = json.load(open(out)) if os.path.exists(out) else {}
+    doc[workload] = res
+    doc.setdefault("ncu_time_share", {})
+    if not isinstance(doc["ncu_time_share"], dict) or "k_quad" in doc["ncu_time_share"]:
+        doc["ncu_time_share"] = {}
+    doc["ncu_time_share"][workload] = share
+    doc["source"] = ("ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,"
+                     "dram__bytes_write.sum, one bench step per workload (profiles/*launches*.csv)")
+    json.dump(doc, open(out, "w"), indent=1)
     print(res, share)
 
 
