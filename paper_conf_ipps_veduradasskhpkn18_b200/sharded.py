@@ -228,12 +228,14 @@ class P2PExchange:
         self.esize = out.element_size()
         dt = dtype if dtype is not None else api._dt_of_tensor(out)
         self._opened = []
+        self.subs = p2p_subproblems(self.sp, rank)
+        # plan first (no CUDA state yet): an unsupported sub-box raises before
+        # any peer mapping exists
+        self.plans = [api.plan_strided(dt, s.extents, self.sp.perm, s.in_strides, s.out_strides)
+                      for s in self.subs]
         if peer_ptrs is None:
             peer_ptrs = self._map_peers(out)
         self.peers = peer_ptrs
-        self.subs = p2p_subproblems(self.sp, rank)
-        self.plans = [api.plan_strided(dt, s.extents, self.sp.perm, s.in_strides, s.out_strides)
-                      for s in self.subs]
 
     def _map_peers(self, out):
         ptrs, self._opened = map_peer_slabs(out, self.group)
