@@ -5,7 +5,10 @@ Metric (BASELINE.json): effective transpose GB/s = 2*N*sizeof(elem)/time/1e9
 (PAPER.md L1501-1505), here summed over one "step" = one pass of the hot path
 over the workload: every case of the TTC-like 57-case suite (BASELINE config 2,
 SURVEY App. A synthetic re-creation), fp64, 200 MiB per tensor, each case one
-`ttlg_execute` of a pre-built plan (repeated-use mode, L1569-1593).
+`ttlg_execute` of a pre-built plan (repeated-use mode, L1569-1593); the
+step's 57 launches are captured once into a CUDA graph and replayed (the same
+kernels with the same parameter blocks; direct launches are timed as well and
+reported as `direct_launch`, `--no-graph` times only those).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--workload ttc57|ccsdt|smallfvi|c1]
   python bench.py --impl reference ...   (the oracle on the host cores)
@@ -334,6 +337,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
     ap.add_argument("--ref-cases-per-step", type=int, default=6)
+    ap.add_argument("--no-graph", action="store_true",
+                    help="time the step as direct launches only (default: the step's launches "
+                         "captured once into a CUDA graph and replayed; direct launches are "
+                         "timed too and reported as direct_launch)")
     ap.add_argument("--no-emulate", action="store_true",
                     help="sharded workload: skip the one-GPU emulation of P = 2/4/8")
     ap.add_argument("--tune", type=int, default=8,
@@ -406,6 +413,18 @@ def main():
 
     for _ in range(args.warmup):
         one_step()
+    graph = None
+    if not args.no_graph:
+        # the step captured once into a CUDA graph (kernel nodes with their
+        # parameter blocks baked in) and replayed: no per-launch host work
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph, stream=stream):
+            for i, p in enumerate(plans):
+                p.execute(As[i].data_ptr(), Bs[i].data_ptr(), stream.cuda_stream)
+        for _ in range(2):
+            graph.replay()
+        torch.cuda.synchronize()
     torch.cuda.synchronize()
 
     # ---- timed region (device events on the launching stream)
@@ -421,7 +440,11 @@ def main():
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     for s in range(args.steps):
-        one_step()
+        if graph is not None:
+            with torch.cuda.stream(stream):
+                graph.replay()
+        else:
+            one_step()
     t_end.record(stream)
     torch.cuda.synchronize()
     if world > 1:
@@ -432,6 +455,25 @@ def main():
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         elapsed_ms = float(t.item())
     launches = len(plans) * args.steps
+    direct = None
+    if graph is not None:
+        # the same K steps as direct launches (one ttlg_execute per case)
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        d0, d1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        d0.record(stream)
+        for _ in range(args.steps):
+            one_step()
+        d1.record(stream)
+        torch.cuda.synchronize()
+        dms = d0.elapsed_time(d1)
+        if world > 1:
+            t = torch.tensor([dms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dms = float(t.item())
+        direct = {"value": world * step_bytes * args.steps / (dms / 1e3) / 1e9, "unit": "GB/s",
+                  "ms_per_step": dms / args.steps}
     # per-kernel durations: the same K steps again, the launches of each kernel
     # grouped between ONE event pair per kernel and step (an event record
     # between two launches adds a bubble, so per-launch pairs would inflate
@@ -518,7 +560,8 @@ def main():
         torch.cuda.synchronize()
         tv = step_bytes * args.steps / (e0.elapsed_time(e1) / 1e3) / 1e9
         tuned = {"value": tv, "unit": "GB/s", "frac_of_d2d": tv / d2d_gbs,
-                 "model_regret_pct": 100.0 * (tv / (value / world) - 1.0),
+                 "model_regret_pct": 100.0 * (tv / ((direct["value"] if direct else value) /
+                                                    world) - 1.0),
                  "candidates_per_case": args.tune,
                  "api": "ttlg_plan_tune (measure mode over the model's short list)"}
         del tplans
@@ -591,7 +634,9 @@ def main():
             "data": "synthetic (SplitMix64 bit patterns, generated on device)",
             "config": {"workload": name, "cases_per_step": len(cases),
                        "bytes_per_step": step_bytes, "parallelism": f"replica x{world}",
-                       "mode": "repeated-use (pre-built plans)",
+                       "mode": "repeated-use (pre-built plans)" + (
+                           "; the step's launches captured once into a CUDA graph and replayed"
+                           if graph is not None else "; direct launches"),
                        "timing": "value: K steps between two events (no per-launch events); "
                                  "roofline/kernels: a second pass of K steps, each kernel's "
                                  "launches grouped between one event pair per step; cases / "
@@ -610,6 +655,7 @@ def main():
             "schemas": schemas,
             "model_err_pct": 100.0 * sum(errs) / len(errs),
             "tuned": tuned,
+            "direct_launch": direct,
             "clocks": clk,
             "e2e": e2e,
             "cpu_baseline": cpu,

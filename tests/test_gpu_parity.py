@@ -452,3 +452,33 @@ def test_closed_block_deep_tiles(ext):
     """1 0 2 4 3 5 with a >= 4 KB leading block: the deep k_pipe tiles."""
     got, exp, info = _run(ext, [1, 0, 2, 4, 3, 5], 8, 901, canary=64)
     _assert_equal(got, exp, f"deep {info['kernel']} {info['tile_extents']}")
+
+
+def test_cuda_graph_capture_replay():
+    """ttlg_execute launches can be captured into a CUDA graph (parameter
+    blocks are baked into the kernel nodes) and replayed: bit-exact, and the
+    plan may be destroyed after capture."""
+    cases = [([64, 48, 40], [2, 0, 1], 8), ([3, 256, 24], [1, 0, 2], 4), ([40, 30, 20], [0, 2, 1], 4)]
+    s = torch.cuda.Stream()
+    bufs = []
+    for k, (ext, perm, eb) in enumerate(cases):
+        n = int(np.prod(ext))
+        A = gen_tensor_torch(950 + k, n, eb, device=DEV)
+        bufs.append((A, torch.empty_like(A), ttlg.plan(_dt(eb), ext, perm)))
+    torch.cuda.synchronize()
+    for A, B, p in bufs:  # warm-up outside capture (one-time function attributes)
+        p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for A, B, p in bufs:
+            p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)
+    plans = [p for _, _, p in bufs]
+    for p in plans:
+        p.destroy()
+    for _, B, _ in bufs:
+        B.zero_()
+    g.replay()
+    torch.cuda.synchronize()
+    for (ext, perm, eb), (A, B, _) in zip(cases, bufs):
+        _assert_equal(_bits(B), oracle.transpose(_bits(A), ext, perm), f"graph {ext} {perm}")
