@@ -481,13 +481,25 @@ def main():
     kinds = sorted({kname(inf) for inf in infos})
     kev = {k: [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                for _ in range(args.steps)] for k in kinds}
+    kgraph = {}
+    if graph is not None:  # each kernel's launches as one graph, like the step
+        for k in kinds:
+            kgraph[k] = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(kgraph[k], stream=stream):
+                for i, p in enumerate(plans):
+                    if kname(infos[i]) == k:
+                        p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
+        torch.cuda.synchronize()
     with torch.cuda.stream(stream):
         for s in range(args.steps):
             for k in kinds:
                 kev[k][s][0].record(stream)
-                for i, p in enumerate(plans):
-                    if kname(infos[i]) == k:
-                        p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
+                if k in kgraph:
+                    kgraph[k].replay()
+                else:
+                    for i, p in enumerate(plans):
+                        if kname(infos[i]) == k:
+                            p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
                 kev[k][s][1].record(stream)
     # per-case durations (model error, per-case table): an event pair per launch
     for s in range(args.steps):
@@ -639,8 +651,9 @@ def main():
                            if graph is not None else "; direct launches"),
                        "timing": "value: K steps between two events (no per-launch events); "
                                  "roofline/kernels: a second pass of K steps, each kernel's "
-                                 "launches grouped between one event pair per step; cases / "
-                                 "model error: a third pass with an event pair per launch",
+                                 "launches grouped (as one graph in graph mode) between one "
+                                 "event pair per step; cases / model error: a third pass "
+                                 "with an event pair per launch",
                        "l2": l2_label},
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,
