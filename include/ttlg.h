@@ -92,9 +92,11 @@ typedef struct {
                                             (one tile per CTA), 2 = k_pipe (persistent,
                                             double-buffered), 3 = k_quad (OD in 16-byte
                                             chunks, K x K register transpose), 4 = k_deint
-                                            ([n0,M(,nb)] perm (1 0 (2)), 2 <= n0 <= 8,
-                                            M a multiple of 16/s: 16-byte accesses both
-                                            ways, no shared memory)                       */
+                                            / k_inter ([n0,M(,nb)] perm (1 0 (2)) with
+                                            2 <= n0 <= 8 and M a multiple of 16/s, or
+                                            2 <= M <= 8 and n0 a multiple of 16/s:
+                                            16-byte accesses both ways through a per-warp
+                                            staging buffer)                               */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
