@@ -10,7 +10,8 @@ step's 57 launches are captured once into a CUDA graph and replayed (the same
 kernels with the same parameter blocks; direct launches are timed as well and
 reported as `direct_launch`, `--no-graph` times only those).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--workload ttc57|ccsdt|smallfvi|c1]
+  python bench.py [--gpus N] [--steps K] [--warmup W]
+                  [--workload ttc57|ccsdt|smallfvi|c1|sharded|720-15|720-16|720-17|fig13]
   python bench.py --impl reference ...   (the oracle on the host cores)
 
 Inputs are generated on the device by the shared SplitMix64 generator
