@@ -118,14 +118,30 @@ def transpose_strided(A: np.ndarray, B: np.ndarray, extents: Sequence[int],
     return B
 
 
-def source_index(extents: Sequence[int], perm: Sequence[int], linB) -> np.ndarray:
-    """For each output linear index, the input linear index it is copied from."""
+def source_index(extents: Sequence[int], perm: Sequence[int], linB,
+                 threads: int = 1) -> np.ndarray:
+    """For each output linear index, the input linear index it is copied from.
+    threads > 1 splits the index list into contiguous pieces evaluated
+    concurrently (each piece is the same C loop; ctypes releases the GIL)."""
     linB = np.ascontiguousarray(np.asarray(linB, dtype=np.int64))
     linA = np.empty_like(linB)
     ext, pr = _arrs(extents, perm)
-    rc = _load().oracle_source_index(len(extents), ext, pr, linB.ctypes.data,
-                                     linA.ctypes.data, linB.size)
-    if rc != 0:
+    lib = _load()
+
+    def piece(lo, hi):
+        return lib.oracle_source_index(len(extents), ext, pr,
+                                       linB.ctypes.data + 8 * lo, linA.ctypes.data + 8 * lo,
+                                       hi - lo)
+    n = linB.size
+    threads = max(1, min(int(threads), n // 65536 or 1))
+    if threads == 1:
+        rcs = [piece(0, n)]
+    else:
+        from concurrent.futures import ThreadPoolExecutor
+        cuts = [n * t // threads for t in range(threads + 1)]
+        with ThreadPoolExecutor(threads) as ex:
+            rcs = list(ex.map(lambda t: piece(cuts[t], cuts[t + 1]), range(threads)))
+    if any(rc != 0 for rc in rcs):
         raise ValueError("oracle: invalid rank/extents/perm")
     return linA
 

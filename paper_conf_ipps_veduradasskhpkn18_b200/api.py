@@ -66,8 +66,9 @@ class Plan:
         self.dtype = _dtype_code(dtype)
         self.extents = [int(e) for e in extents]
         self.perm = [int(p) for p in perm]
+        self.strided = in_strides is not None or out_strides is not None
         ext, pr = arrays(self.extents, self.perm)
-        if in_strides is not None or out_strides is not None:
+        if self.strided:
             # sub-tensor form (ttlg_plan_strided): strides in elements
             d = len(self.extents)
 
@@ -253,6 +254,13 @@ def transpose_tensor(x, perm_t: Sequence[int], out=None, plan_: Optional[Plan] =
     stream = torch.cuda.current_stream(x.device).cuda_stream
     with torch.cuda.device(x.device):
         if plan_ is not None:
+            # the plan must describe exactly this (dtype, extents, perm) on dense
+            # tensors: a mismatched plan would address past the end of out
+            if (plan_.dtype != _dt_of_tensor(x) or plan_.extents != ext or plan_.perm != perm
+                    or plan_.strided):
+                raise ValueError("plan_ does not match x's dtype / shape / perm_t")
+            if not (x.is_contiguous() and out.is_contiguous()):
+                raise ValueError("plan_ needs contiguous x and out")
             plan_.execute(x.data_ptr(), out.data_ptr(), stream)
         elif x.is_contiguous() and out.is_contiguous():
             transpose(_dt_of_tensor(x), ext, perm, x.data_ptr(), out.data_ptr(), stream)

@@ -140,22 +140,46 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
     return TTLG_ERR_DEVICE;
   }
   if ((a | b) % (uintptr_t)p->align) {
-    // widened / 16-byte-vector access needs aligned pointers: re-plan at the
-    // element width (elem_bytes_override also rules out k_quad)
-    ttlg_plan_s q;
-    ttlg_plan_hints h;
-    if (p->has_hints) {
-      h = p->hints;
-    } else {
+    // widened / 16-byte-vector access needs aligned pointers: run the plan's
+    // element-width twin (elem_bytes_override also rules out k_quad and
+    // k_deint), planned once on first use and kept in the plan.  Only the
+    // caller's schema / no_fusion hints carry over: slice, kernel and block
+    // hints describe the widened problem (ttlg_plan_tune's winners carry them).
+    ttlg_plan_s *q = p->fallback.load(std::memory_order_acquire);
+    if (!q) {
+      q = new (std::nothrow) ttlg_plan_s;
+      if (!q) return TTLG_ERR_NO_MEMORY;
+      ttlg_plan_hints h;
       ttlg_plan_hints_init(&h);
+      h.elem_bytes_override = s;
+      if (p->has_hints) {
+        h.schema = p->hints.schema;
+        h.no_fusion = p->hints.no_fusion;
+      }
+      const int64_t *isx = p->strided ? p->in_strides : nullptr;
+      const int64_t *osx = p->strided ? p->out_strides : nullptr;
+      ttlg_status st = plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false, isx, osx);
+      if (st != TTLG_OK && h.schema != TTLG_SCHEMA_AUTO) {
+        // a schema of the widened problem (e.g. OD on a squeezed pencil) need
+        // not exist at element width; the bytes are the same under any schema
+        h.schema = TTLG_SCHEMA_AUTO;
+        st = plan_into(q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false, isx, osx);
+      }
+      if (st != TTLG_OK) {
+        delete q;
+        return st;
+      }
+      ttlg_plan_s *expected = nullptr;
+      if (!p->fallback.compare_exchange_strong(expected, q, std::memory_order_acq_rel)) {
+        delete q;  // another thread installed one first
+        q = expected;
+      }
     }
-    h.elem_bytes_override = s;
-    if (h.variant == 3 || h.variant == 4) h.variant = 0;  // k_quad / k_deint need 16-byte alignment
-    ttlg_status st = plan_into(&q, (ttlg_dtype)p->dt, p->rank, p->ext, p->perm, &h, false,
-                               p->strided ? p->in_strides : nullptr,
-                               p->strided ? p->out_strides : nullptr);
-    if (st != TTLG_OK) return st;
-    return launch(&q, A, B, stream);
+    ttlg_status st = launch(q, A, B, stream);
+    if (st == TTLG_OK && getenv_sync()) {
+      if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return TTLG_ERR_CUDA;
+    }
+    return st;
   }
   ttlg_status st = launch(p, A, B, stream);
   if (st == TTLG_OK && getenv_sync()) {
@@ -183,14 +207,17 @@ struct HostPipe {
   cudaStream_t h2d = nullptr, comp = nullptr, d2h = nullptr;
   cudaEvent_t start = nullptr, done = nullptr, evA[kMaxChunks], evB[kMaxChunks];
   bool ok = false;
+  std::once_flag init;
   std::mutex mu;
 };
 HostPipe g_pipes[16];
 
+// The device's pipe (streams and events created once, on that device: the
+// caller has checked that `dev` is current).
 HostPipe *host_pipe(int dev) {
   if (dev < 0 || dev >= 16) return nullptr;
   HostPipe &p = g_pipes[dev];
-  if (!p.ok) {
+  std::call_once(p.init, [&p]() {
     bool good = cudaStreamCreateWithFlags(&p.h2d, cudaStreamNonBlocking) == cudaSuccess &&
                 cudaStreamCreateWithFlags(&p.comp, cudaStreamNonBlocking) == cudaSuccess &&
                 cudaStreamCreateWithFlags(&p.d2h, cudaStreamNonBlocking) == cudaSuccess &&
@@ -199,10 +226,10 @@ HostPipe *host_pipe(int dev) {
     for (int i = 0; good && i < kMaxChunks; i++)
       good = cudaEventCreateWithFlags(&p.evA[i], cudaEventDisableTiming) == cudaSuccess &&
              cudaEventCreateWithFlags(&p.evB[i], cudaEventDisableTiming) == cudaSuccess;
-    if (!good) return nullptr;
-    p.ok = true;
-  }
-  return &p;
+    if (!good) cudaGetLastError();
+    p.ok = good;
+  });
+  return p.ok ? &p : nullptr;
 }
 }  // namespace
 
@@ -215,6 +242,13 @@ static ttlg_status execute_host(const ttlg_plan_s *p, const void *A_host, void *
   for (int i = 0; i < d; i++) m[i] = p->ext[p->perm[i]];
   const int64_t nbytes = N * esize;
   if (p->device < 0) return TTLG_ERR_DEVICE;
+  {
+    int dev = -1;  // before any stream / event of the device's pipe is touched
+    if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) {
+      cudaGetLastError();
+      return TTLG_ERR_DEVICE;
+    }
+  }
   const int64_t want = std::min<int64_t>((int64_t)kMaxChunks, nbytes / (16ll << 20));
   // the split dim: widest narrower row (contiguous side = unbounded)
   int cd = -1, pos = -1;

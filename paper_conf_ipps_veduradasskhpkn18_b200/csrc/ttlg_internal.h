@@ -5,6 +5,8 @@
 
 #include <stdint.h>
 
+#include <atomic>
+
 #include "../../include/ttlg.h"
 
 #define TTLG_MAXD TTLG_MAX_RANK
@@ -165,6 +167,14 @@ struct ttlg_plan_s {
   // sub-tensor (ttlg_plan_strided) request: strides in elements as given
   bool strided;
   int64_t in_strides[TTLG_MAXD], out_strides[TTLG_MAXD];
+  // element-width plan for pointers not aligned to `align` (api.cpp execute):
+  // built once, on first use, and owned by this plan
+  mutable std::atomic<ttlg_plan_s *> fallback{nullptr};
+
+  ttlg_plan_s() = default;
+  ttlg_plan_s(const ttlg_plan_s &) = delete;
+  ttlg_plan_s &operator=(const ttlg_plan_s &) = delete;
+  ~ttlg_plan_s() { delete fallback.load(std::memory_order_acquire); }
 };
 
 namespace ttlg {

@@ -482,3 +482,44 @@ def test_cuda_graph_capture_replay():
     torch.cuda.synchronize()
     for (ext, perm, eb), (A, B, _) in zip(cases, bufs):
         _assert_equal(_bits(B), oracle.transpose(_bits(A), ext, perm), f"graph {ext} {perm}")
+
+
+def test_tuned_plan_on_misaligned_views():
+    """A plan tuned on aligned buffers (its winner carries slice / kernel
+    hints of the widened problem) still runs on element-aligned views: the
+    element-width twin keeps only schema / no_fusion.  Tuning on
+    misaligned buffers works too, and the twin is built once per plan."""
+    stream = torch.cuda.current_stream().cuda_stream
+    for ext, perm, eb in (([64, 64, 64], [0, 2, 1], 8), ([4, 256, 96], [0, 2, 1], 4),
+                          ([64, 96], [1, 0], 4), ([3, 400, 8], [1, 0, 2], 4)):
+        n = int(np.prod(ext))
+        A = gen_tensor_torch(31, n + 1, eb, device=DEV)
+        B = torch.empty_like(A)
+        exp = oracle.transpose(_bits(A[1:]), ext, perm)
+        p = ttlg.plan(_dt(eb), ext, perm)
+        p.tune(A[:n].data_ptr(), B[:n].data_ptr(), stream, 6)
+        for _ in range(2):
+            B.zero_()
+            p.execute(A[1:].data_ptr(), B[1:].data_ptr(), stream)
+            torch.cuda.synchronize()
+            _assert_equal(_bits(B[1:]), exp, f"tuned, misaligned {ext} {perm}")
+        q = ttlg.plan(_dt(eb), ext, perm)
+        q.tune(A[1:].data_ptr(), B[1:].data_ptr(), stream, 6)
+        B.zero_()
+        q.execute(A[1:].data_ptr(), B[1:].data_ptr(), stream)
+        torch.cuda.synchronize()
+        _assert_equal(_bits(B[1:]), exp, f"tuned on misaligned {ext} {perm}")
+
+
+def test_transpose_tensor_rejects_mismatched_plan():
+    x = gen_tensor_torch(8, 6 * 7 * 8, 4, device=DEV).view(6, 7, 8)
+    ext, perm = ttlg.torch_to_c(list(x.shape), (2, 1, 0))
+    good = ttlg.plan("f32", ext, perm)
+    y = ttlg.transpose_tensor(x, (2, 1, 0), plan_=good)
+    torch.cuda.synchronize()
+    assert torch.equal(y.view(torch.int32).cpu(),
+                       x.permute(2, 1, 0).contiguous().view(torch.int32).cpu())
+    for bad in (ttlg.plan("f32", [8, 7, 7], perm), ttlg.plan("f64", ext, perm),
+                ttlg.plan("f32", ext, [1, 0, 2])):
+        with pytest.raises(ValueError):
+            ttlg.transpose_tensor(x, (2, 1, 0), plan_=bad)
