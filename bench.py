@@ -145,9 +145,16 @@ def run_reference(args, rank, world):
     """--impl reference: the oracle on the host cores (rank 0 only)."""
     if rank != 0:
         return
-    name, cases = _workload(args.workload)
     import oracle
-    from synth import gen_tensor_np, case_seed
+    from synth import gen_tensor_np, case_seed, configs
+    if args.workload == "sharded":
+        # config 5: one rank's slab at P = 8 ([64, 64, 64, 64, 16] fp32, 1 GiB),
+        # each of the five perms as a local transposition (the bounded sample)
+        name = "c5-8GiB-rank5-fp32 sharded (BASELINE config 5): one P=8 slab per case"
+        cases = [configs.Case(c.case_id, c.extents[:-1] + (c.extents[-1] // 8,), c.perm,
+                              c.elem_bytes, c.group) for c in configs.config5()]
+    else:
+        name, cases = _workload(args.workload)
     cores = len(os.sched_getaffinity(0))
     # each step = a bounded sample of the workload: the next m cases of the
     # suite, round-robin (warm-up steps advance too), so K steps sweep it
@@ -172,7 +179,9 @@ def run_reference(args, rank, world):
     line = {"impl": "reference", "metric": "effective transpose GB/s (2*N*s/time)",
             "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * sum(times) / len(times),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True,
+            "scaling": "strong" if args.workload == "sharded" else "weak", "vs_baseline": None,
+            "dtype": "f64" if cases[0].elem_bytes == 8 else "f32",
             "data": "synthetic (SplitMix64 bit patterns)",
             "config": {"workload": name,
                        "step": f"{m} cases of the suite per step, round-robin (bounded sample)"},
@@ -327,13 +336,28 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
         print(json.dumps(line), flush=True)
 
 
+def spawn_ranks(n: int) -> int:
+    """Re-run this command as n ranks under torch.distributed.run (rendezvous
+    on 127.0.0.1); returns the launcher's exit code."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={n}", "--master-addr=127.0.0.1", f"--master-port={port}",
+           os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ttlg", choices=["ttlg", "reference"])
-    ap.add_argument("--workload", default="ttc57")
+    ap.add_argument("--workload", default=None,
+                    help="default: ttc57 at N = 1 (BASELINE config 2, the headline); "
+                         "sharded (config 5, the north star's multi-GPU case) at N > 1")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=12.0)
@@ -349,11 +373,19 @@ def main():
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1 and args.impl != "reference":
+        # `bench.py --gpus N` without a launcher: start the N ranks ourselves
+        # (one process per GPU, the same command under torch.distributed.run)
+        sys.exit(spawn_ranks(args.gpus))
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if "WORLD_SIZE" in os.environ and args.gpus != world:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
+    if args.workload is None:
+        args.workload = "ttc57" if args.gpus == 1 else "sharded"
     if args.impl == "reference":
-        run_reference(args, rank, world)
+        run_reference(args, rank, args.gpus)
         return
 
     import numpy as np

@@ -1,0 +1,137 @@
+#!/usr/bin/env python
+"""Per-case floor table (VERDICT r1 "Next round" 2): every case of a workload
+timed on its own as ONE CUDA graph of R back-to-back `ttlg_execute` launches
+of its pre-built plan (no event pairs between launches), beside a graph of R
+same-size cudaMemcpyAsync device-to-device copies (the case-size-matched D2D
+denominator of the north star's ">= 90 % of D2D").
+
+  python tools/cases.py --workload c2 [--reps 20] [--trials 5] [--out f.json]
+
+Per case: GB/s = R * 2*N*s / t, the D2D GB/s of the same
+byte count, their ratio, the fraction of the measured HBM peak, the plan
+(schema, kernel, tile), predicted vs measured seconds (model error), and the
+strict Alg. 1 label is NOT used here (that is test infrastructure).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+
+def workload(name):
+    from synth import configs
+    table = {"c1": configs.config1, "c2": configs.config2, "c3": configs.config3,
+             "c4": configs.config4, "c5": configs.config5, "fig13": configs.fig13,
+             "720-15": lambda: configs.sweep720(15), "720-16": lambda: configs.sweep720(16),
+             "720-17": lambda: configs.sweep720(17)}
+    return table[name]()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", default="c2")
+    ap.add_argument("--reps", type=int, default=20)
+    ap.add_argument("--trials", type=int, default=5)
+    ap.add_argument("--out", default=None)
+    ap.add_argument("--only", default=None, help="comma-separated case ids")
+    ap.add_argument("--hints", default=None, help="json dict of plan hints for every case")
+    args = ap.parse_args()
+
+    import torch
+    import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
+    from synth import gen_tensor_torch, case_seed
+
+    peak = 6552.6
+    pp = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(pp):
+        peak = json.load(open(pp))["hbm_gbs"]
+    cases = workload(args.workload)
+    if args.only:
+        keep = {int(x) for x in args.only.split(",")}
+        cases = [c for c in cases if c.case_id in keep]
+    hints = json.loads(args.hints) if args.hints else {}
+    dev = torch.device("cuda:0")
+    s = torch.cuda.Stream(device=dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+
+    def time_graph(g):
+        with torch.cuda.stream(s):
+            for _ in range(2):
+                g.replay()
+            ts = []
+            for _ in range(args.trials):
+                e0.record(s)
+                g.replay()
+                e1.record(s)
+                e1.synchronize()
+                ts.append(e0.elapsed_time(e1) * 1e-3)
+        return statistics.median(ts)
+
+    rows, bufs = [], {}
+    d2d_cache = {}
+    t_start = time.time()
+    for c in cases:
+        key = (c.n_elems, c.elem_bytes)
+        if key not in bufs:
+            bufs.clear()
+            torch.cuda.empty_cache()
+            A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
+            bufs[key] = (A, torch.empty_like(A))
+        A, B = bufs[key]
+        p = ttlg.plan("f64" if c.elem_bytes == 8 else "f32", c.extents, c.perm, **hints)
+        info = p.describe()
+        with torch.cuda.stream(s):
+            p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)  # warm (function attributes)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(args.reps):
+                p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)
+        t = time_graph(g) / args.reps
+        del g
+        nbytes = c.alg_bytes
+        if nbytes not in d2d_cache:
+            gd = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(gd, stream=s):
+                for _ in range(args.reps):
+                    B.copy_(A)
+            d2d_cache[nbytes] = nbytes / (time_graph(gd) / args.reps) / 1e9
+            del gd
+        gbs = nbytes / t / 1e9
+        d2d = d2d_cache[nbytes]
+        rows.append({"case": c.label(), "schema": info["schema"], "kernel": info["kernel"],
+                     "access_bytes": info["access_bytes"], "threads": info["threads"],
+                     "tile": info["tile_extents"][:info["fused_rank"]],
+                     "fused": info["fused_extents"][:info["fused_rank"]],
+                     "fperm": info["fused_perm"][:info["fused_rank"]],
+                     "us": t * 1e6, "gbs": gbs, "d2d_gbs": d2d, "frac_d2d": gbs / d2d,
+                     "frac_peak": gbs / peak, "pred_us": info["predicted_seconds"] * 1e6,
+                     "model_err": abs(info["predicted_seconds"] - t) / t})
+        print(json.dumps(rows[-1]), flush=True)
+    tot_b = sum(c.alg_bytes for c in cases)
+    tot_t = sum(r["us"] for r in rows) * 1e-6
+    summ = {"workload": args.workload, "reps": args.reps, "trials": args.trials, "peak": peak,
+            "timing": "per case: one CUDA graph of `reps` back-to-back ttlg_execute launches "
+                      "(median of `trials` replays); D2D: a graph of `reps` same-size "
+                      "device-to-device copies",
+            "aggregate_gbs": tot_b / tot_t / 1e9,
+            "min_frac_d2d": min(r["frac_d2d"] for r in rows),
+            "below_0.9_d2d": [r["case"] for r in rows if r["frac_d2d"] < 0.9],
+            "mean_model_err": statistics.mean(r["model_err"] for r in rows),
+            "wall_s": time.time() - t_start, "cases": rows}
+    print(json.dumps({k: v for k, v in summ.items() if k != "cases"}), flush=True)
+    if args.out:
+        os.makedirs(os.path.dirname(args.out) or ".", exist_ok=True)
+        with open(args.out, "w") as f:
+            json.dump(summ, f, indent=1)
+
+
+if __name__ == "__main__":
+    main()
