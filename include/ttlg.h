@@ -164,6 +164,20 @@ ttlg_status ttlg_plan_strided(ttlg_plan_t *out, ttlg_dtype dt, int rank, const i
  * pointers, element-aligned, non-overlapping. */
 ttlg_status ttlg_execute(ttlg_plan_t plan, const void *A, void *B, void *stream);
 
+/* Batched repeated-use execution: the same plan on `count` (A[i], B[i]) pairs
+ * in ONE kernel launch (grid.y = count, at most TTLG_MAX_BATCH pairs per
+ * launch; larger counts take ceil(count / TTLG_MAX_BATCH) launches).  Used by
+ * the fused sharded exchange, where rank p's P sub-transpositions have the
+ * same shape and differ only in the A sub-box and the destination (peer) B
+ * slab.  Arrays are caller-owned host arrays of device pointers; every pair
+ * obeys ttlg_execute's rules, and no A[i] may overlap any B[j]
+ * (TTLG_ERR_ALIASING).  Outputs B[i] must not overlap each other (not
+ * checked: the result would depend on the write order).  count < 1 or NULL
+ * arrays -> TTLG_ERR_INVALID_VALUE. */
+#define TTLG_MAX_BATCH 16
+ttlg_status ttlg_execute_batch(ttlg_plan_t plan, int32_t count, const void *const *A,
+                               void *const *B, void *stream);
+
 ttlg_status ttlg_plan_destroy(ttlg_plan_t plan);
 
 /* Single-use: plan + execute + destroy, no caching, no host sync. */

@@ -26,7 +26,8 @@ EXPORTS = ["ttlg_plan", "ttlg_plan_ex", "ttlg_plan_hints_init", "ttlg_execute",
            "ttlg_plan_destroy", "ttlg_transpose", "ttlg_execute_host", "ttlg_predict_time",
            "ttlg_plan_describe", "ttlg_status_string", "ttlg_schema_name", "ttlg_version",
            "ttlg_model_source", "ttlg_plan_candidates", "ttlg_plan_tune", "ttlg_plan_strided",
-           "ttlg_ipc_export", "ttlg_ipc_open", "ttlg_ipc_close"]
+           "ttlg_ipc_export", "ttlg_ipc_open", "ttlg_ipc_close", "ttlg_execute_batch"]
+MAX_BATCH = 16
 IPC_HANDLE_BYTES = 64
 
 
@@ -102,6 +103,8 @@ def _load():
         "ttlg_ipc_open": ([ctypes.c_char_p, ctypes.c_int64, ctypes.POINTER(P)], ctypes.c_int),
         "ttlg_ipc_close": ([P, ctypes.c_int64], ctypes.c_int),
         "ttlg_execute": ([P, P, P, P], ctypes.c_int),
+        "ttlg_execute_batch": ([P, ctypes.c_int32, ctypes.POINTER(P), ctypes.POINTER(P), P],
+                               ctypes.c_int),
         "ttlg_plan_destroy": ([P], ctypes.c_int),
         "ttlg_transpose": ([ctypes.c_int, ctypes.c_int, i64p, i32p, P, P, P], ctypes.c_int),
         "ttlg_execute_host": ([P, P, P, P, P, P], ctypes.c_int),

@@ -104,6 +104,16 @@ class Plan:
         check(lib.ttlg_execute(self._h, ctypes.c_void_p(A_ptr), ctypes.c_void_p(B_ptr),
                                ctypes.c_void_p(stream)), "ttlg_execute")
 
+    def execute_batch(self, A_ptrs: Sequence[int], B_ptrs: Sequence[int], stream: int = 0):
+        """The plan on len(A_ptrs) (A, B) pairs in one launch (ttlg_execute_batch)."""
+        n = len(A_ptrs)
+        if len(B_ptrs) != n:
+            raise ValueError("A_ptrs and B_ptrs must have the same length")
+        a = (ctypes.c_void_p * n)(*[ctypes.c_void_p(int(x)) for x in A_ptrs])
+        b = (ctypes.c_void_p * n)(*[ctypes.c_void_p(int(x)) for x in B_ptrs])
+        check(lib.ttlg_execute_batch(self._h, n, a, b, ctypes.c_void_p(stream)),
+              "ttlg_execute_batch")
+
     def execute_host(self, A_host: int, B_host: int, A_dev: int, B_dev: int, stream: int = 0):
         check(lib.ttlg_execute_host(self._h, ctypes.c_void_p(A_host), ctypes.c_void_p(B_host),
                                     ctypes.c_void_p(A_dev), ctypes.c_void_p(B_dev),

@@ -127,19 +127,29 @@ static bool getenv_sync() {
   return v == 1;
 }
 
-static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *stream) {
-  if (!p || !A || !B) return TTLG_ERR_INVALID_VALUE;
+// n (A, B) pairs of one plan (1 <= n <= kMaxBatch): one launch with grid.y = n
+static ttlg_status execute_n(const ttlg_plan_s *p, int n, const void *const *Av,
+                             void *const *Bv, void *stream) {
+  if (!p || n < 1 || n > kMaxBatch || !Av || !Bv) return TTLG_ERR_INVALID_VALUE;
   const int s = p->dt == TTLG_F64 ? 8 : 4;
-  const uintptr_t a = (uintptr_t)A, b = (uintptr_t)B;
-  if (a % s || b % s) return TTLG_ERR_INVALID_VALUE;
-  if (a < b + (uintptr_t)p->spanB && b < a + (uintptr_t)p->spanA) return TTLG_ERR_ALIASING;
+  uintptr_t any = 0;
+  for (int i = 0; i < n; i++) {
+    const uintptr_t a = (uintptr_t)Av[i], b = (uintptr_t)Bv[i];
+    if (!a || !b || a % s || b % s) return TTLG_ERR_INVALID_VALUE;
+    any |= a | b;
+  }
+  for (int i = 0; i < n; i++)
+    for (int j = 0; j < n; j++) {
+      const uintptr_t a = (uintptr_t)Av[i], b = (uintptr_t)Bv[j];
+      if (a < b + (uintptr_t)p->spanB && b < a + (uintptr_t)p->spanA) return TTLG_ERR_ALIASING;
+    }
   if (p->device < 0) return TTLG_ERR_DEVICE;
   int dev = -1;
   if (cudaGetDevice(&dev) != cudaSuccess || dev != p->device) {
     cudaGetLastError();
     return TTLG_ERR_DEVICE;
   }
-  if ((a | b) % (uintptr_t)p->align) {
+  if (any % (uintptr_t)p->align) {
     // widened / 16-byte-vector access needs aligned pointers: run the plan's
     // element-width twin (elem_bytes_override also rules out k_quad and
     // k_deint), planned once on first use and kept in the plan.  Only the
@@ -175,19 +185,23 @@ static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *s
         q = expected;
       }
     }
-    ttlg_status st = launch(q, A, B, stream);
+    ttlg_status st = launch(q, n, Av, Bv, stream);
     if (st == TTLG_OK && getenv_sync()) {
       if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return TTLG_ERR_CUDA;
     }
     return st;
   }
-  ttlg_status st = launch(p, A, B, stream);
+  ttlg_status st = launch(p, n, Av, Bv, stream);
   if (st == TTLG_OK && getenv_sync()) {
     if (cudaStreamSynchronize((cudaStream_t)stream) != cudaSuccess) return TTLG_ERR_CUDA;
   }
   return st;
 }
 
+
+static ttlg_status execute(const ttlg_plan_s *p, const void *A, void *B, void *stream) {
+  return execute_n(p, 1, &A, &B, stream);
+}
 
 // ---- host-buffer pipeline (ttlg_execute_host) --------------------------------
 // A is split along one input dim cd into C chunks.  Chunk k's input slab is
@@ -388,6 +402,25 @@ ttlg_status ttlg_plan(ttlg_plan_t *out, ttlg_dtype dt, int rank, const int64_t *
 
 ttlg_status ttlg_execute(ttlg_plan_t plan, const void *A, void *B, void *stream) {
   return execute(plan, A, B, stream);
+}
+
+ttlg_status ttlg_execute_batch(ttlg_plan_t plan, int32_t count, const void *const *A,
+                               void *const *B, void *stream) {
+  if (!plan || count < 1 || !A || !B) return TTLG_ERR_INVALID_VALUE;
+  // validate every pair (and cross-pair aliasing) before the first launch
+  for (int i = 0; i < count; i++)
+    for (int j = 0; j < count; j++) {
+      const uintptr_t a = (uintptr_t)A[i], b = (uintptr_t)B[j];
+      if (!a || !b) return TTLG_ERR_INVALID_VALUE;
+      if (a < b + (uintptr_t)plan->spanB && b < a + (uintptr_t)plan->spanA)
+        return TTLG_ERR_ALIASING;
+    }
+  for (int32_t i0 = 0; i0 < count; i0 += kMaxBatch) {
+    const int n = (int)std::min<int32_t>(kMaxBatch, count - i0);
+    ttlg_status st = execute_n(plan, n, A + i0, B + i0, stream);
+    if (st != TTLG_OK) return st;
+  }
+  return TTLG_OK;
 }
 
 ttlg_status ttlg_plan_destroy(ttlg_plan_t plan) {

@@ -219,8 +219,9 @@ __device__ __forceinline__ void build_rows(int R, int nr, const FastDiv *ext, co
 
 template <int W, int U, bool CS>
 __global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TileParams P,
-                                                const void *__restrict__ Av,
-                                                void *__restrict__ Bv) {
+                                                const __grid_constant__ BatchPtrs X) {
+  const void *__restrict__ Av = X.A[blockIdx.y];
+  void *__restrict__ Bv = X.B[blockIdx.y];
   using T = typename Vec<W>::T;
   extern __shared__ __align__(16) unsigned char smem[];
   int2 *tabB = reinterpret_cast<int2 *>(smem + P.off_tabB);
@@ -325,8 +326,9 @@ struct __align__(16) CtxS {
 
 template <int W, bool XT, bool PERSIST, bool SM2>
 __global__ void __launch_bounds__(512, PERSIST ? 2 : (XT ? 3 : 4)) k_pipe(const __grid_constant__ TileParams P,
-                                              const void *__restrict__ Av,
-                                              void *__restrict__ Bv) {
+                                              const __grid_constant__ BatchPtrs X) {
+  const void *__restrict__ Av = X.A[blockIdx.y];
+  void *__restrict__ Bv = X.B[blockIdx.y];
   using T = typename Vec<W>::T;
   extern __shared__ __align__(16) unsigned char smem[];
   const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
@@ -633,8 +635,9 @@ __device__ __forceinline__ void quad_transpose<4, 8>(uint2 &v, int q) {
 
 template <int S, int CB, int NJ>
 __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TileParams P,
-                                                 const void *__restrict__ Av,
-                                                 void *__restrict__ Bv) {
+                                                 const __grid_constant__ BatchPtrs X) {
+  const void *__restrict__ Av = X.A[blockIdx.y];
+  void *__restrict__ Bv = X.B[blockIdx.y];
   constexpr int K = CB / S, LGK = K == 4 ? 2 : 1;
   using C = typename Chunk<CB>::T;
   extern __shared__ __align__(16) unsigned char smem[];
@@ -803,8 +806,9 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
 // num_tiles = chunks.
 template <int S, int N0>
 __global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParams P,
-                                               const void *__restrict__ Av,
-                                               void *__restrict__ Bv) {
+                                               const __grid_constant__ BatchPtrs X) {
+  const void *__restrict__ Av = X.A[blockIdx.y];
+  void *__restrict__ Bv = X.B[blockIdx.y];
   constexpr int K = 16 / S;          // elements per 16-byte vector
   constexpr int E = N0 * K;          // elements per thread slice
   constexpr int WPE = S / 4;         // 32-bit words per element
@@ -865,8 +869,9 @@ __global__ void __launch_bounds__(256) k_deint(const __grid_constant__ TileParam
 
 template <int S, int N1>
 __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParams P,
-                                               const void *__restrict__ Av,
-                                               void *__restrict__ Bv) {
+                                               const __grid_constant__ BatchPtrs X) {
+  const void *__restrict__ Av = X.A[blockIdx.y];
+  void *__restrict__ Bv = X.B[blockIdx.y];
   constexpr int K = 16 / S;
   constexpr int E = N1 * K;
   constexpr int WPE = S / 4;
@@ -1041,7 +1046,9 @@ static bool pdl_enabled() {
   return v == 1;
 }
 
-ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream) {
+ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *const *B,
+                   void *stream) {
+  if (n < 1 || n > kMaxBatch) return TTLG_ERR_INVALID_VALUE;
   const void *fn = plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
                        : plan->kind == KK_DEINT
@@ -1070,9 +1077,14 @@ ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream
     }
   }
   TileParams kp = plan->kp;
-  void *args[] = {(void *)&kp, (void *)&A, (void *)&B};
+  BatchPtrs X;
+  for (int i = 0; i < kMaxBatch; i++) {
+    X.A[i] = A[i < n ? i : 0];
+    X.B[i] = B[i < n ? i : 0];
+  }
+  void *args[] = {(void *)&kp, (void *)&X};
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(plan->grid);
+  cfg.gridDim = dim3(plan->grid, n);
   cfg.blockDim = dim3(plan->threads);
   cfg.dynamicSmemBytes = (size_t)smem;
   cfg.stream = (cudaStream_t)stream;

@@ -116,6 +116,14 @@ struct TileParams {
   int32_t deint_inter;         // 1: k_inter (SoA -> AoS, the small dim is dim 1)
 };
 
+// Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;
+// ttlg_execute_batch) -- a __grid_constant__ kernel parameter like TileParams.
+constexpr int kMaxBatch = TTLG_MAX_BATCH;
+struct BatchPtrs {
+  const void *A[kMaxBatch];
+  void *B[kMaxBatch];
+};
+
 struct Problem {
   int esize;       // bytes per element as given (4/8)
   int W;           // access-element bytes after widening (4/8/16)
@@ -200,6 +208,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
 // api.cpp
 const DeviceProfile &device_profile(int device);
 // kernels.cu
-ttlg_status launch(const ttlg_plan_s *plan, const void *A, void *B, void *stream);
+// n pairs (1 <= n <= kMaxBatch) in one launch: grid (plan->grid, n)
+ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *const *B,
+                   void *stream);
 int kernel_regs(int kind, int W);  // registers per thread of a kernel variant (cached; 0 if unknown)
 }  // namespace ttlg

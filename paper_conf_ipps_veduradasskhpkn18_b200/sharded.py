@@ -230,9 +230,16 @@ class P2PExchange:
         self._opened = []
         self.subs = p2p_subproblems(self.sp, rank)
         # plan first (no CUDA state yet): an unsupported sub-box raises before
-        # any peer mapping exists
-        self.plans = [api.plan_strided(dt, s.extents, self.sp.perm, s.in_strides, s.out_strides)
-                      for s in self.subs]
+        # any peer mapping exists.  Every destination's sub-box has the same
+        # extents and strides (only the A offset and the target slab differ),
+        # so ONE plan serves all of them and run() issues ONE batched launch
+        # (ttlg_execute_batch: grid.y = destinations).
+        s0 = self.subs[0]
+        assert all(s.extents == s0.extents and s.in_strides == s0.in_strides and
+                   s.out_strides == s0.out_strides for s in self.subs)
+        self.plan = api.plan_strided(dt, s0.extents, self.sp.perm, s0.in_strides,
+                                     s0.out_strides)
+        self.plans = [self.plan] * len(self.subs)
         if peer_ptrs is None:
             peer_ptrs = self._map_peers(out)
         self.peers = peer_ptrs
@@ -242,13 +249,14 @@ class P2PExchange:
         return ptrs
 
     def predicted_seconds(self) -> float:
-        return sum(p.describe()["predicted_seconds"] for p in self.plans)
+        return len(self.subs) * self.plan.describe()["predicted_seconds"]
 
     def run(self, A_local, stream: int):
+        """All P sub-transpositions as one kernel launch (grid.y = P)."""
         a0 = A_local.data_ptr()
-        for s, p in zip(self.subs, self.plans):
-            p.execute(a0 + s.a_offset * self.esize,
-                      self.peers[s.dest] + s.b_offset * self.esize, stream)
+        self.plan.execute_batch([a0 + s.a_offset * self.esize for s in self.subs],
+                                [self.peers[s.dest] + s.b_offset * self.esize
+                                 for s in self.subs], stream)
 
     def close(self):
         unmap_peer_slabs(self._opened)

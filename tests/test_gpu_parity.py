@@ -523,3 +523,28 @@ def test_transpose_tensor_rejects_mismatched_plan():
                 ttlg.plan("f32", ext, [1, 0, 2])):
         with pytest.raises(ValueError):
             ttlg.transpose_tensor(x, (2, 1, 0), plan_=bad)
+
+
+@pytest.mark.parametrize("count", [1, 3, 16, 21])
+def test_execute_batch(count):
+    """ttlg_execute_batch: one plan on `count` independent (A, B) pairs, one
+    launch per 16 pairs (grid.y = pairs), each bit-exact; every kernel family."""
+    stream = torch.cuda.current_stream().cuda_stream
+    for ext, perm, eb, hints in (([64, 48, 40], [2, 0, 1], 8, {}),
+                                 ([64, 96], [1, 0], 4, {"variant": 3}),
+                                 ([40, 30, 20], [0, 2, 1], 4, {}),
+                                 ([3, 256, 24], [1, 0, 2], 4, {"variant": 4}),
+                                 ([24, 20, 12, 8], [3, 1, 0, 2], 8, {"variant": 2})):
+        n = int(np.prod(ext))
+        As = [gen_tensor_torch(1200 + i, n, eb, device=DEV) for i in range(count)]
+        Bs = [torch.empty_like(a) for a in As]
+        p = ttlg.plan(_dt(eb), ext, perm, **hints)
+        p.execute_batch([a.data_ptr() for a in As], [b.data_ptr() for b in Bs], stream)
+        torch.cuda.synchronize()
+        for i in range(count):
+            _assert_equal(_bits(Bs[i]), oracle.transpose(_bits(As[i]), ext, perm),
+                          f"batch {i}/{count} {ext} {perm} {p.describe()['kernel']}")
+    X, Y, Z = (torch.empty_like(As[0]) for _ in range(3))
+    with pytest.raises(ttlg.TtlgError) as e:   # the A of pair 0 is the B of pair 1
+        p.execute_batch([X.data_ptr(), Y.data_ptr()], [Z.data_ptr(), X.data_ptr()], stream)
+    assert e.value.code == 2
