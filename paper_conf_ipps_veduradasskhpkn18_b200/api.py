@@ -217,7 +217,8 @@ def candidate_hints(d: dict) -> dict:
          "in_block": d["tile_extents"][a], "out_dim": b,
          "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
     if d["kernel"] != "direct":
-        h["variant"] = {"tile": 1, "pipe": 2, "quad": 3, "deint": 4}[d["kernel"]]
+        h["variant"] = {"tile": 1, "pipe": 2, "quad": 3, "deint": 4, "bulkq": 5,
+                        "bulkg": 6}[d["kernel"]]
     return h
 
 

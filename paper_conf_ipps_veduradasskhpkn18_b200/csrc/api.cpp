@@ -504,7 +504,13 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
     h.out_dim = ci.out_dim;
     h.out_block = ci.tile_extents[ci.fused_perm[ci.out_dim]];
     h.threads = ci.threads;
-    h.variant = ci.kernel == KK_TILE ? 1 : (ci.kernel == KK_PIPE ? 2 : (ci.kernel == KK_QUAD ? 3 : 0));
+    h.variant = ci.kernel == KK_TILE    ? 1
+                : ci.kernel == KK_PIPE  ? 2
+                : ci.kernel == KK_QUAD  ? 3
+                : ci.kernel == KK_BULKQ ? 5
+                : ci.kernel == KK_BULKG ? 6
+                                        : 0;
+    if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = 0;  // consumers + producer
     if (ci.kernel == KK_DEINT) {  // no slice parameters: the structure size fixes the slice
       ttlg_plan_hints_init(&h);
       h.variant = 4;

@@ -933,6 +933,235 @@ __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParam
   }
 }
 
+// ---------------------------------------------------------------------------
+// k_bulk: the staged tile transposition (OD, Alg. 2; OA/FMS, Alg. 5
+// L948-1020 / Alg. 6) as a warp-specialised, persistent pipeline:
+//
+//   warp 0 (producer): for each of the CTA's tiles, waits until ring stage s
+//     is free (mbarrier empty[s]), decodes the tile, arms full[s] with the
+//     tile's byte count and moves every A-row of the tile global -> shared
+//     with ONE TMA bulk copy per row (cp.async.bulk ... mbarrier::complete_tx,
+//     SASS UBLKCP): no per-element load instructions at all;
+//   warps 1.. (consumers): wait on full[s], write the tile's B-rows with
+//     16-byte stores, then release the stage (one arrive per warp on empty[s]).
+//
+// Up to nstage tiles are in flight per CTA, so the loads of the next tiles
+// stream while the current one is written -- no CTA-wide barrier anywhere in
+// the steady state (the ring replaces k_pipe's cp.async double buffer).
+// Consumer modes:
+//   MODE 0 (quad, OD): as k_quad -- a group of K = 16/S lanes reads K 16-byte
+//     chunks (K consecutive input-run positions at K consecutive output
+//     positions), transposes the K x K block with xor-shuffles and writes K
+//     B-rows with one 16-byte store each;
+//   MODE 1 (gather, any schema): a thread owns one 16-byte chunk of the
+//     output run (K = 16/S consecutive output positions, their shared-memory
+//     offsets in registers) and writes it for B-rows r0, r0 + rsB, ...: K
+//     element reads from shared memory, one 16-byte store.
+// Requirements (planner): every A-row starts 16-byte aligned and is a whole
+// number of 16-byte chunks (also in partial tiles); MODE 1 likewise for
+// B-rows; 16-byte aligned pointers.
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n}\n"
+               ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(bar)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile("{\n .reg .pred p;\n"
+               "TTLG_WAIT_%=:\n"
+               " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+               " @!p bra TTLG_WAIT_%=;\n}\n" ::"r"(bar), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes,
+                                         uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+      ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+
+template <int S, int MODE>
+__global__ void __launch_bounds__(544, 1) k_bulk(const __grid_constant__ TileParams P,
+                                                 const __grid_constant__ BatchPtrs X) {
+  constexpr int K = 16 / S;
+  constexpr int LGK = K == 4 ? 2 : (K == 2 ? 1 : 0);
+  const unsigned char *A = reinterpret_cast<const unsigned char *>(X.A[blockIdx.y]);
+  unsigned char *B = reinterpret_cast<unsigned char *>(X.B[blockIdx.y]);
+  extern __shared__ __align__(128) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_bar = s0 + P.off_bar, s_data = s0 + P.off_data;
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int NS = P.nstage, NC = (int)(blockDim.x >> 5) - 1;  // consumer warps
+  auto full_bar = [&](int st) { return s_bar + 16u * st; };
+  auto empty_bar = [&](int st) { return s_bar + 16u * st + 8u; };
+
+  if (tid == 0) {
+    for (int st = 0; st < NS; st++) {
+      mbar_init(full_bar(st), 1);
+      mbar_init(empty_bar(st), NC);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  // row tables (Alg. 4's offsets as rows x columns), built once per CTA
+  build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk, reinterpret_cast<int2 *>(smem),
+             reinterpret_cast<int *>(smem + P.off_digB), S);
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA), S);
+#pragma unroll 1
+  for (int j = tid; j < P.LB; j += blockDim.x) {
+    int rem = j, sm = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+      sm += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
+      rem = cq;
+    }
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = sm * S;  // byte offset
+  }
+  __syncthreads();
+
+  if (warp == 0) {
+    // ---- producer: one TMA bulk copy per A-row
+    int st = 0;
+    uint32_t ph = 0;
+    const int RA = P.RA;
+    for (uint32_t tile = blockIdx.x, k = 0; tile < P.num_tiles; tile += gridDim.x, k++) {
+      if (k >= (uint32_t)NS) mbar_wait(empty_bar(st), ph ^ 1u);
+      const TileCtx c = decode_tile(P, tile);
+      const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+      const uint32_t rowb = (uint32_t)(P.LAunit * c.limA) * S;
+      uint32_t nrows = (uint32_t)RA;
+      if (!full) {
+        uint32_t cnt = 0;
+        for (int r = lane; r < RA; r += 32) cnt += lds_int(s_digB + 4 * r) < c.limB;
+        nrows = __reduce_add_sync(0xffffffffu, cnt);
+      }
+      if (lane == 0) {
+        ctx[st].bA = c.bA;
+        ctx[st].bB = c.bB;
+        ctx[st].limA = c.limA;
+        ctx[st].limB = c.limB;
+        mbar_expect_tx(full_bar(st), nrows * rowb);
+      }
+      __syncwarp();
+      const unsigned char *Ab = A + c.bA * S;
+      const uint32_t dst = s_data + (uint32_t)st * P.stage_bytes;
+#pragma unroll 1
+      for (int r = lane; r < RA; r += 32) {
+        const int2 t = lds_int2(s_tabA + 8 * r);
+        if (full || lds_int(s_digB + 4 * r) < c.limB)
+          bulk_g2s(dst + t.y, Ab + (int64_t)t.x * S, rowb, full_bar(st));
+      }
+      if (++st == NS) {
+        st = 0;
+        ph ^= 1u;
+      }
+    }
+    return;
+  }
+
+  // ---- consumers
+  const int ct = tid - 32, NTc = NC * 32, LB = P.LB, RB = P.RB;
+  int m0, j0, rs, nB;
+  uint32_t jc[K];
+  if constexpr (MODE == 0) {
+    // quad: output position j0 (one per thread), row quads m0, m0 + rsB, ...
+    m0 = (int)fdiv1(ct, P.fd_LB);
+    j0 = ct - m0 * LB;
+    rs = P.rsB;
+    const int RBq = RB / K;
+    nB = (m0 < rs && m0 < RBq) ? (int)fdiv1(RBq - 1 - m0, P.fd_rsB) + 1 : 0;
+    jc[0] = lds_int(s_jcol + 4 * (j0 < LB ? j0 : 0));
+  } else {
+    // gather: output chunk q = j0 / K (one per thread), B-rows m0, m0 + rsB, ...
+    const int LBc = LB / K;
+    m0 = (int)fdiv1(ct, P.fd_LB);
+    j0 = (ct - m0 * LBc) * K;
+    rs = P.rsB;
+    nB = (m0 < rs && m0 < RB) ? (int)fdiv1(RB - 1 - m0, P.fd_rsB) + 1 : 0;
+#pragma unroll
+    for (int u = 0; u < K; u++) jc[u] = lds_int(s_jcol + 4 * (j0 + u < LB ? j0 + u : 0));
+  }
+  const int q = j0 & (K - 1);
+  const int nBw = MODE == 0 ? __reduce_max_sync(0xffffffffu, nB) : nB;
+  int st = 0;
+  uint32_t ph = 0;
+  for (uint32_t tile = blockIdx.x; tile < P.num_tiles; tile += gridDim.x) {
+    mbar_wait(full_bar(st), ph);
+    TileCtx c;
+    c.bA = ctx[st].bA;
+    c.bB = ctx[st].bB;
+    c.limA = ctx[st].limA;
+    c.limB = ctx[st].limB;
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int lim = full ? LB : P.LBunit * c.limB;
+    const uint32_t sbuf = s_data + (uint32_t)st * P.stage_bytes;
+    if constexpr (MODE == 0) {
+      using C = typename Chunk<16>::T;
+      int m = m0;
+#pragma unroll 4
+      for (int k = 0; k < nBw; k++) {
+        const bool act = k < nB;
+        const int row = K * (act ? m : 0) + q;  // own B-row x+q after the transpose
+        const int2 t = lds_int2(s_tabB + 8 * row);
+        const bool rok = act && j0 < LB && (full || lds_int(s_digA + 4 * row) < c.limA);
+        C v = lds_T<C>(sbuf + (t.y - q * S) + jc[0]);
+        quad_transpose<S, 16>(v, q);
+        const int jb = j0 - q;
+        C *dst = reinterpret_cast<C *>(B + (c.bB + jb) * S);
+        stcs_p(wadd(dst, (uint32_t)t.x >> LGK), v, rok && (full || jb < lim));
+        m += rs;
+      }
+    } else {
+      const bool jok = full || j0 < lim;
+      int r = m0;
+#pragma unroll 4
+      for (int k = 0; k < nB; k++) {
+        const int2 t = lds_int2(s_tabB + 8 * r);
+        uint4 v;
+        const uint32_t sr = sbuf + t.y;
+        if constexpr (S == 16) {
+          v = lds_T<uint4>(sr + jc[0]);
+        } else if constexpr (S == 8) {
+          const uint2 a = lds_T<uint2>(sr + jc[0]), b = lds_T<uint2>(sr + jc[1]);
+          v = make_uint4(a.x, a.y, b.x, b.y);
+        } else {
+          v = make_uint4(lds_T<unsigned int>(sr + jc[0]), lds_T<unsigned int>(sr + jc[1]),
+                         lds_T<unsigned int>(sr + jc[2]), lds_T<unsigned int>(sr + jc[3]));
+        }
+        uint4 *dst = reinterpret_cast<uint4 *>(B + (c.bB + j0) * S);
+        stcs_p(wadd(dst, (uint32_t)t.x >> LGK), v,
+               jok && (full || lds_int(s_digA + 4 * r) < c.limA));
+        r += rs;
+      }
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty_bar(st));
+    if (++st == NS) {
+      st = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
+template <int S>
+static const void *bulk_ptr_s(int mode) {
+  return mode == 0 ? (const void *)k_bulk<S, 0> : (const void *)k_bulk<S, 1>;
+}
+static const void *bulk_ptr(int W, int kind) {
+  const int mode = kind == KK_BULKQ ? 0 : 1;
+  if (W == 4) return bulk_ptr_s<4>(mode);
+  if (W == 8) return bulk_ptr_s<8>(mode);
+  return mode == 1 ? (const void *)k_bulk<16, 1> : nullptr;
+}
+
 template <int S>
 static const void *inter_ptr_s(int n1) {
   switch (n1) {
@@ -1009,6 +1238,7 @@ int kernel_regs(int kind, int W) {
   // asks for every scored candidate
   static std::atomic<int> regs[KK_NUM][3] = {{{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
@@ -1020,7 +1250,9 @@ int kernel_regs(int kind, int W) {
     cudaFuncAttributes attr;
     const void *fn = kind == KK_QUAD    ? quad_ptr(W, 16, 1)
                      : kind == KK_DEINT ? deint_ptr(W == 8 ? 8 : 4, 4)
-                                        : kernel_ptr(kind, W, false, false);
+                     : (kind == KK_BULKQ || kind == KK_BULKG)
+                         ? bulk_ptr(W, kind)
+                         : kernel_ptr(kind, W, false, false);
     if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
       r = attr.numRegs;
     } else {
@@ -1051,6 +1283,8 @@ ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *c
   if (n < 1 || n > kMaxBatch) return TTLG_ERR_INVALID_VALUE;
   const void *fn = plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
+                       : (plan->kind == KK_BULKQ || plan->kind == KK_BULKG)
+                             ? bulk_ptr(plan->W, plan->kind)
                        : plan->kind == KK_DEINT
                              ? (plan->kp.deint_inter ? inter_ptr(plan->W, plan->kp.deint_n0)
                                                      : deint_ptr(plan->W, plan->kp.deint_n0))

@@ -25,6 +25,7 @@ struct ModelInput {
   double fillA;  // useful fraction of the tile grid (partial tiles)
   double conf_load, conf_store;  // smem wavefronts / ideal for one warp access (>= 1)
   int qk;                        // k_quad chunk elements (0: scalar kernels)
+  int nstage;                    // k_bulk: tile buffers in the ring
 };
 
 struct ModelFeatures {

@@ -179,6 +179,18 @@ static void dense_prefixes(Problem &P) {
     P.denseB++;
 }
 
+// k_bulk joins the automatic choice only with TTLG_BULK=1 until the model is
+// calibrated on it (forced with hints variant 5 / 6 otherwise)
+static bool bulk_auto() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_BULK");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+constexpr int kBulkMaxStages = 6;
+
 namespace {
 
 struct Tile {
@@ -222,7 +234,7 @@ Tile make_tile(const Problem &P, int a, int64_t ta, int b, int64_t tb) {
 
 int schema_of(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_DIRECT) return P.d == 1 ? TTLG_SCHEMA_COPY : TTLG_SCHEMA_FML;
-  if (kind == KK_QUAD) return TTLG_SCHEMA_OD;
+  if (kind == KK_QUAD || kind == KK_BULKQ) return TTLG_SCHEMA_OD;
   if (P.p[0] == 0) return TTLG_SCHEMA_FMS;
   for (int i = 0; i <= T.b; i++)
     if (P.p[i] <= T.a) return TTLG_SCHEMA_OA;  // input and output groups overlap
@@ -232,23 +244,78 @@ int schema_of(const Problem &P, const Tile &T, int kind) {
 int64_t ceil_div(int64_t x, int64_t y) { return (x + y - 1) / y; }
 
 // k_quad (vector chunks in and out, K x K register transpose): an OD tile
-// whose input FVI and output FVI extents and blocks are multiples of K (so
-// every A-row, B-row and tile base is chunk-aligned).  K = 16 / W (16-byte
-// chunks); fp32 tiles whose FVIs are only even use K = 2 (8-byte chunks).
-// Returns K, or 0 when no chunking applies.
+// (the two runs disjoint; a tile holds only the dims of its two runs) whose
+// every A-row and B-row starts on a chunk boundary and whose runs are whole
+// chunks -- then every global access is one K-element vector and a chunk of K
+// consecutive input-run positions is K consecutive B-rows.  Exactly:
+//   LA = LAunit * t_a and the partial LAunit * (n_a mod t_a) multiples of K,
+//   likewise LB (LBunit * t_pb, LBunit * (n_pb mod t_pb));
+//   the A-row digits (output-run dims) have A strides multiple of K, the
+//   B-row digits (input-run dims) B strides multiple of K;
+//   every grid stride t_k * s_k (tile bases) a multiple of K on both sides.
+// The input FVI itself need not be a multiple of K (e.g. [3, 4096, 4096]
+// fp32 `2 1 0` with t1 = 4m: A-rows of 12 m floats).  K = 16 / W (16-byte
+// chunks); fp32 tiles failing that use K = 2 (8-byte chunks).  Returns K, or
+// 0 when no chunking applies.
 int quad_k(const Problem &P, const Tile &T) {
   if (P.W != P.esize || P.p[0] == 0) return 0;
   for (int i = 0; i <= T.b; i++)
     if (P.p[i] <= T.a) return 0;  // groups overlap: not OD
-  const int p0 = P.p[0];
+  const int pb = P.p[T.b];
+  bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
+  for (int k = 0; k <= T.a; k++) inIS[k] = true;
+  for (int i = 0; i <= T.b; i++) inOS[P.p[i]] = true;
+  int64_t LAunit = 1, LBunit = 1;
+  for (int k = 0; k < T.a; k++) LAunit *= T.t[k];
+  for (int i = 0; i < T.b; i++) LBunit *= T.t[P.p[i]];
   for (int K = 16 / P.W; K >= 2; K /= 2) {
-    // P.kalign: sub-tensors need every row start chunk-aligned
-    if (P.kalign % K == 0 && P.n[0] % K == 0 && P.n[p0] % K == 0 && T.t[0] % K == 0 &&
-        T.t[p0] % K == 0)
-      return K;
+    bool ok = (LAunit * T.t[T.a]) % K == 0 && (LAunit * (P.n[T.a] % T.t[T.a])) % K == 0 &&
+              (LBunit * T.t[pb]) % K == 0 && (LBunit * (P.n[pb] % T.t[pb])) % K == 0;
+    for (int k = 0; k < P.d && ok; k++) {
+      if (T.t[k] > 1 && inOS[k] && P.sA[k] % K) ok = false;  // A-row digit
+      if (T.t[k] > 1 && inIS[k] && P.sB[k] % K) ok = false;  // B-row digit
+      if (P.n[k] > T.t[k] && ((T.t[k] * P.sA[k]) % K || (T.t[k] * P.sB[k]) % K))
+        ok = false;  // tile base
+    }
+    if (ok) return K;
     if (P.W == 8) break;  // fp64: 16-byte chunks only
   }
   return 0;
+}
+
+// k_bulk (TMA bulk row loads): every A-row of every tile (partial tiles
+// included) starts 16-byte aligned and is a whole number of 16-byte chunks;
+// consumer mode quad needs k_quad's 16-byte chunks on the B side, mode gather
+// the same row alignment for B-rows.  No padded input runs (a bulk copy lands
+// one contiguous row).
+static bool bulk_ok(const Problem &P, const Tile &T, int kind) {
+  const int W = P.W, pb = P.p[T.b];
+  bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
+  for (int k = 0; k <= T.a; k++) inIS[k] = true;
+  for (int i = 0; i <= T.b; i++) inOS[P.p[i]] = true;
+  int64_t LAunit = 1, LBunit = 1;
+  for (int k = 0; k < T.a; k++) LAunit *= T.t[k];
+  for (int i = 0; i < T.b; i++) LBunit *= T.t[P.p[i]];
+  if ((LAunit * T.t[T.a] * W) % 16 || (LAunit * (P.n[T.a] % T.t[T.a]) * W) % 16) return false;
+  for (int k = 0; k < P.d; k++) {
+    if (T.t[k] > 1 && !inIS[k] && (P.sA[k] * W) % 16) return false;  // A-row digit
+    if (P.n[k] > T.t[k] && (T.t[k] * P.sA[k] * W) % 16) return false;  // tile base
+  }
+  if (kind == KK_BULKQ) return P.W == P.esize && quad_k(P, T) == 16 / W;
+  if ((LBunit * T.t[pb] * W) % 16 || (LBunit * (P.n[pb] % T.t[pb]) * W) % 16) return false;
+  for (int k = 0; k < P.d; k++) {
+    if (T.t[k] > 1 && !inOS[k] && (P.sB[k] * W) % 16) return false;  // B-row digit
+    if (P.n[k] > T.t[k] && (T.t[k] * P.sB[k] * W) % 16) return false;  // tile base
+  }
+  return true;
+}
+
+// Smallest block factor >= t (<= n) that makes pre * t a multiple of K, or 0.
+static int64_t round_block(int64_t t, int64_t pre, int64_t n, int K) {
+  int64_t m = 1;
+  while ((pre * m) % K) m++;
+  const int64_t r = (t + m - 1) / m * m;
+  return r <= n ? r : 0;
 }
 
 // Shared-memory stride of the next output-only dim (the generalisation of the
@@ -289,9 +356,17 @@ struct TileSummary {
   int buf_bytes;  // one data buffer
 };
 
+// shared-memory layout unit (elements) of a staged kernel: k_quad / k_bulk keep
+// every A-row on a 16-byte (chunk) boundary
+static int layout_unit(const Problem &P, const Tile &T, int kind) {
+  if (kind == KK_QUAD) return quad_k(P, T);
+  if (kind == KK_BULKQ || kind == KK_BULKG) return 16 / P.W;
+  return 0;
+}
+
 static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S) {
   const int d = P.d, a = T.a, b = T.b;
-  const int qk = kind == KK_QUAD ? quad_k(P, T) : 0;
+  const int qk = layout_unit(P, T, kind);
   S.qk = qk;
   bool inIS[TTLG_MAXD] = {false};
   for (int k = 0; k <= a; k++) inIS[k] = true;
@@ -332,8 +407,10 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
 static bool build_params(const Problem &P, const Tile &T, int kind, int threads, int nbuf,
                          TileParams &K, const int *isdelta = nullptr) {
   memset(&K, 0, sizeof(K));
-  const int qk = kind == KK_QUAD ? quad_k(P, T) : 0;
+  const int qk = layout_unit(P, T, kind);
   if (kind == KK_QUAD && qk == 0) return false;
+  const bool bulk = kind == KK_BULKQ || kind == KK_BULKG;
+  if (bulk && (isdelta || !bulk_ok(P, T, kind))) return false;
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
   bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
@@ -476,7 +553,23 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     off += (bytes + 15) / 16 * 16;
     return (int32_t)o;
   };
-  if (kind != KK_DIRECT) {
+  if (bulk) {
+    // k_bulk: tables, nbuf decoded-tile slots and mbarrier pairs, then the
+    // ring of nbuf tile buffers (128-byte aligned)
+    take((int64_t)K.RA * 8);  // tabA at 0
+    K.off_tabB = take((int64_t)K.RB * 8);
+    K.off_jcol = take((int64_t)K.LB * 4);
+    K.off_digB = take((int64_t)K.RA * 4);
+    K.off_digA = take((int64_t)K.RB * 4);
+    K.off_ctx = take(32 * (int64_t)nbuf);
+    K.off_bar = take(16 * (int64_t)nbuf);
+    off = (off + 127) / 128 * 128;
+    K.stage_bytes = (int32_t)((smem_elems * P.W + 127) / 128 * 128);
+    K.off_data = (int32_t)off;
+    K.off_data2 = K.off_data;
+    off += (int64_t)K.stage_bytes * nbuf;
+    K.nstage = nbuf;
+  } else if (kind != KK_DIRECT) {
     take((int64_t)K.RA * 8);  // tabA at 0
     K.off_tabB = take((int64_t)K.RB * 8);
     K.off_jcol = take((int64_t)K.LB * 4);
@@ -503,6 +596,20 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   K.drB = threads / K.LB;
   K.dxB = threads % K.LB;
   K.rsB = threads / K.LB;
+  if (bulk) {
+    // consumers are threads - 32 (warp 0 produces); quad: one output position
+    // per consumer, gather: one 16-byte output chunk per consumer
+    const int ntc = threads - 32;
+    const int L = kind == KK_BULKQ ? K.LB : K.LB * P.W / 16;
+    if (L > ntc) return false;
+    K.qk = kind == KK_BULKQ ? qk : 0;
+    K.rsB = ntc / L;
+    K.fd_LB = make_fastdiv((uint32_t)L);
+    K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
+    K.fd_LA = make_fastdiv((uint32_t)K.LA);
+    K.fd_NT = make_fastdiv((uint32_t)ntc);
+    return true;
+  }
   if (kind == KK_QUAD) {  // the load walk runs over chunks
     K.qk = qk;
     K.qnj = K.LB <= threads ? 1 : (K.LB <= 2 * threads ? 2 : 4);
@@ -778,7 +885,17 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // model input of one (geometry, kernel, block size); false if it cannot launch
   auto make_mi = [&](ModelInput &mi, int &tpc, int kind, int schema, int threads,
                      const TileSummary &S, double cl, double cs) {
-    const int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
+    int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
+    mi.nstage = 0;
+    if (kind == KK_BULKQ || kind == KK_BULKG) {
+      // as many ring stages as fit next to the tables (2..kBulkMaxStages), one CTA per SM
+      const int buf = (S.buf_bytes + 127) / 128 * 128;
+      const int fixed = S.smem_base - S.buf_bytes + 256;
+      const int ns = std::min(kBulkMaxStages, (dev.smem_per_block_optin - fixed) / std::max(buf, 1));
+      if (ns < 2) return false;
+      mi.nstage = ns;
+      smem = fixed + ns * buf;
+    }
     if (smem > dev.smem_per_block_optin) return false;
     // k_quad: at most 4 output positions per thread, warp-wide shuffles (whole warps)
     if (kind == KK_QUAD && (S.LB > 4 * threads || threads % 32)) return false;
@@ -797,9 +914,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.smem_bytes = smem;
     mi.occ = occupancy(dev, threads, smem, kernel_regs(kind, P.W));
     if (mi.occ < 1) return false;
+    if (mi.nstage) mi.occ = 1;  // __launch_bounds__(544, 1)
     const int64_t slots = (int64_t)dev.sms * mi.occ;
     tpc = 1;
-    if (kind == KK_PIPE) {
+    if (mi.nstage) {
+      mi.grid = (int)std::min<int64_t>(S.tiles, slots);
+      if (hints && hints->grid > 0) mi.grid = hints->grid;
+    } else if (kind == KK_PIPE) {
       // persistent: one CTA per resident slot, striding over the tiles
       mi.grid = (int)std::min<int64_t>(S.tiles, slots);
       if (hints && hints->grid > 0) mi.grid = hints->grid;
@@ -822,6 +943,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                          double &cs, TileSummary &S) {
     for (int k = 0; k < TTLG_MAXD; k++) delta[k] = 0;
     cl = cs = 1.0;
+    if (group == KK_BULKQ || group == KK_BULKG) {
+      // feasibility at the largest consumer count; the ring is sized in make_mi
+      if (!build_params(P, T, group, 32 + 512, 1, K0)) return false;
+      S.smem_base = K0.smem_bytes;
+      S.buf_bytes = K0.stage_bytes;
+      return true;
+    }
     if (!build_params(P, T, group, thr_list[0], 1, K0)) return false;
     if (group == KK_DIRECT) return true;
     if (group == KK_QUAD) {  // conflict-free by construction (16-byte slot j mod 8)
@@ -916,6 +1044,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
     if (hv == 4) return;  // k_deint forced: no staged / direct candidates
+    const bool bulk = group == KK_BULKQ || group == KK_BULKG;
+    if (bulk) {
+      if (forceW) return;  // element-width fallback plans: no 16-byte requirement
+      if (hv == 0 ? !bulk_auto() : hv != (group == KK_BULKQ ? 5 : 6)) return;
+    } else if (hv >= 5) {
+      return;  // k_bulk forced
+    }
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
       if (hints->in_block > 0 && hints->in_block != ta) return;
@@ -957,7 +1092,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (!build_exact(T, group, K0, delta, cl, cs, S)) return;
     }
     int kinds[2], nk = 0;
-    if (group == KK_DIRECT) {
+    if (bulk) {
+      kinds[nk++] = group;
+    } else if (group == KK_DIRECT) {
       kinds[nk++] = KK_DIRECT;
     } else if (group == KK_QUAD) {
       kinds[nk++] = KK_QUAD;
@@ -976,6 +1113,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         const int64_t m = (512 / LBc) * LBc;
         if (m >= 192 && m % 8 == 0 && m != 256) tl[ntl++] = (int)m;
       }
+    }
+    if (bulk) {  // producer warp + 256 / 512 consumers
+      tl[0] = 32 + 256;
+      tl[1] = 32 + 512;
+      ntl = 2;
     }
     for (int ki = 0; ki < nk; ki++) {
       for (int ti = 0; ti < ntl; ti++) {
@@ -1034,13 +1176,34 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         if (pb == a) {
           // the same dim closes both groups (overlap): one shared blocking
           // factor, drawn from both candidate lists
-          for (int i = 0; i < nbA; i++) consider(KK_TILE, a, blocksA[i], b, blocksA[i]);
-          for (int j = 0; j < nbB; j++) consider(KK_TILE, a, blocksB[j], b, blocksB[j]);
+          for (int i = 0; i < nbA; i++) {
+            consider(KK_TILE, a, blocksA[i], b, blocksA[i]);
+            consider(KK_BULKG, a, blocksA[i], b, blocksA[i]);
+          }
+          for (int j = 0; j < nbB; j++) {
+            consider(KK_TILE, a, blocksB[j], b, blocksB[j]);
+            consider(KK_BULKG, a, blocksB[j], b, blocksB[j]);
+          }
         } else {
           for (int i = 0; i < nbA; i++) {
             for (int j = 0; j < nbB; j++) {
               consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
               consider(KK_QUAD, a, blocksA[i], b, blocksB[j]);
+              consider(KK_BULKQ, a, blocksA[i], b, blocksB[j]);
+              consider(KK_BULKG, a, blocksA[i], b, blocksB[j]);
+              // k_quad needs whole chunks per run: the same slice with the
+              // blocking factors rounded up to a chunk multiple (e.g. t1 = 22
+              // -> 24 for [3, 4096, 4096] fp32 `2 1 0`)
+              if (P.W == P.esize && !(hints && (hints->in_block > 0 || hints->out_block > 0))) {
+                const int Kq = 16 / P.W;
+                const int64_t ra = round_block(blocksA[i], preA, P.n[a], Kq);
+                const int64_t rb = round_block(blocksB[j], preB, P.n[pb], Kq);
+                if (ra && rb && (ra != blocksA[i] || rb != blocksB[j])) {
+                  consider(KK_QUAD, a, ra, b, rb);
+                  consider(KK_BULKQ, a, ra, b, rb);
+                  consider(KK_BULKG, a, ra, b, rb);
+                }
+              }
             }
           }
         }
@@ -1240,7 +1403,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         padded |= delta[k] != 0;
       }
       TileParams K;
-      if (!build_params(P, e.T, e.group, e.mi.threads, e.kind == KK_PIPE ? 2 : 1, K,
+      if (!build_params(P, e.T, e.group, e.mi.threads,
+                        e.mi.nstage ? e.mi.nstage : (e.kind == KK_PIPE ? 2 : 1), K,
                         padded ? delta : nullptr))
         continue;
       K.tpc = e.tpc;
@@ -1267,7 +1431,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       delta[k] = B.delta[k];
       padded |= delta[k] != 0;
     }
-    if (!build_params(P, B.T, B.group, B.mi.threads, B.kind == KK_PIPE ? 2 : 1, K,
+    if (!build_params(P, B.T, B.group, B.mi.threads,
+                      B.mi.nstage ? B.mi.nstage : (B.kind == KK_PIPE ? 2 : 1), K,
                       padded ? delta : nullptr))
       return TTLG_ERR_INTERNAL;
     K.tpc = B.tpc;
@@ -1275,7 +1440,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->kind = B.kind;
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
-  plan->align = B.kind == KK_QUAD ? K.qk * P.W : P.W;
+  plan->align = B.kind == KK_QUAD ? K.qk * P.W
+                : (B.kind == KK_BULKQ || B.kind == KK_BULKG) ? 16
+                                                             : P.W;
   plan->threads = B.mi.threads;
   plan->grid = B.mi.grid;
   plan->nbytes = N * P.W;

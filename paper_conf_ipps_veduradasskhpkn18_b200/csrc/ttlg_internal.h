@@ -51,7 +51,11 @@ enum KernelKind : int32_t {
   KK_QUAD = 3,    // OD: 16-byte chunks in and out, K x K register transpose (k_quad)
   KK_DEINT = 4,   // [n0, M(, nb)] perm (1 0 (2)) with n0 <= 8 (k_deint, AoS -> SoA) or
                   // n1 <= 8 (k_inter, SoA -> AoS): 16-byte accesses both ways
-  KK_NUM = 5,
+  KK_BULKQ = 5,   // OD: TMA bulk row loads into an mbarrier ring, K x K register transposes,
+                  // 16-byte stores (k_bulk, consumer mode quad)
+  KK_BULKG = 6,   // any schema: TMA bulk row loads, 16-byte stores gathered from K
+                  // element reads (k_bulk, consumer mode gather)
+  KK_NUM = 7,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -114,6 +118,9 @@ struct TileParams {
   int32_t tpc;                 // tiles per CTA (consecutive tile indices)
   int32_t deint_n0;            // k_deint: n0 (the structure size, 2..8); k_inter: n1
   int32_t deint_inter;         // 1: k_inter (SoA -> AoS, the small dim is dim 1)
+  // k_bulk: ring of nstage tile buffers (stage_bytes apart, from off_data),
+  // 2 * nstage mbarriers at off_bar (full[s], empty[s]); warp 0 produces
+  int32_t nstage, stage_bytes, off_bar;
 };
 
 // Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;

@@ -333,7 +333,7 @@ _VARIANT_CASES = [
 ]
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3])
+@pytest.mark.parametrize("variant", [1, 2, 3, 5, 6])
 @pytest.mark.parametrize("ext,perm,eb", _VARIANT_CASES)
 def test_kernel_variants_forced(ext, perm, eb, variant):
     try:
@@ -548,3 +548,47 @@ def test_execute_batch(count):
     with pytest.raises(ttlg.TtlgError) as e:   # the A of pair 0 is the B of pair 1
         p.execute_batch([X.data_ptr(), Y.data_ptr()], [Z.data_ptr(), X.data_ptr()], stream)
     assert e.value.code == 2
+
+
+def _bulk_cases():
+    out = []
+    for grp in ("c2", "c3", "c4", "c5"):
+        out += [configs.scaled(c, 1 << 21) for c in configs.all_configs()[grp]]
+    return out + [configs.scaled(c, 1 << 18) for c in configs.sweep720(16)[::37]]
+
+
+@pytest.mark.parametrize("variant", [5, 6])
+@pytest.mark.parametrize("case", _bulk_cases(), ids=lambda c: c.label())
+def test_bulk_forced(case, variant):
+    """k_bulk (TMA bulk row loads into an mbarrier ring; 5 = quad consumers,
+    6 = gather consumers) forced on every config shape it applies to."""
+    try:
+        ttlg.plan(_dt(case.elem_bytes), case.extents, case.perm, variant=variant)
+    except ttlg.TtlgError:
+        pytest.skip("k_bulk not applicable (rows not 16-byte aligned)")
+    got, exp, info = _run(case.extents, case.perm, case.elem_bytes, case_seed(case.case_id),
+                          plan_kwargs={"variant": variant}, canary=64)
+    assert info["kernel"] == ("bulkq" if variant == 5 else "bulkg")
+    _assert_equal(got, exp, f"bulk {variant} {info}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_bulk_partial_tiles(eb):
+    """k_bulk with ragged tiles on both blocked dims (partial rows / row counts)."""
+    K = 16 // eb
+    n_ok = 0
+    for ext, perm in (([6 * K, 40, 7], [1, 0, 2]), ([4 * K, 30, 3 * K], [2, 1, 0]),
+                      ([2 * K, 50, 60], [0, 2, 1]), ([3, 4 * K * 11, 4 * K * 9], [2, 1, 0])):
+        for variant in (5, 6):
+            for ib, ob in ((None, None), (3, 5), (K, 2 * K), (2 * K, 3 * K)):
+                kw = {"variant": variant}
+                if ib:
+                    kw.update(in_dim=1, in_block=ib, out_dim=0, out_block=ob)
+                try:
+                    ttlg.plan(_dt(eb), ext, perm, **kw)
+                except ttlg.TtlgError:
+                    continue
+                got, exp, info = _run(ext, perm, eb, 95, plan_kwargs=kw, canary=32)
+                _assert_equal(got, exp, f"bulk partial {ext} {perm} {kw} {info}")
+                n_ok += 1
+    assert n_ok >= 6

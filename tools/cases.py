@@ -61,6 +61,10 @@ def main():
     ap.add_argument("--out", default=None)
     ap.add_argument("--only", default=None, help="comma-separated case ids")
     ap.add_argument("--hints", default=None, help="json dict of plan hints for every case")
+    ap.add_argument("--bulk", action="store_true",
+                    help="per case: the auto plan's slice with the k_bulk kernel (quad "
+                         "consumers for k_quad plans, else gather); the model's own k_bulk "
+                         "slice when the auto slice does not apply")
     args = ap.parse_args()
 
     import torch
@@ -104,7 +108,23 @@ def main():
             A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device=dev)
             bufs[key] = (A, torch.empty_like(A))
         A, B = bufs[key]
-        p = ttlg.plan("f64" if c.elem_bytes == 8 else "f32", c.extents, c.perm, **hints)
+        dt = "f64" if c.elem_bytes == 8 else "f32"
+        if args.bulk:
+            a = ttlg.plan(dt, c.extents, c.perm).describe()
+            h = ttlg.candidate_hints(a)
+            h.pop("threads", None)
+            h["variant"] = 5 if a["kernel"] == "quad" else 6
+            p = None
+            for hh in (h, {"variant": h["variant"]}, {"variant": 6}):
+                try:
+                    p = ttlg.plan(dt, c.extents, c.perm, **hh)
+                    break
+                except ttlg.TtlgError:
+                    continue
+            if p is None:
+                p = ttlg.plan(dt, c.extents, c.perm)
+        else:
+            p = ttlg.plan(dt, c.extents, c.perm, **hints)
         info = p.describe()
         with torch.cuda.stream(s):
             p.execute(A.data_ptr(), B.data_ptr(), s.cuda_stream)  # warm (function attributes)
