@@ -219,6 +219,8 @@ def candidate_hints(d: dict) -> dict:
     if d["kernel"] != "direct":
         h["variant"] = {"tile": 1, "pipe": 2, "quad": 3, "deint": 4, "bulkq": 5,
                         "bulkg": 6}[d["kernel"]]
+    if d["kernel"] in ("bulkq", "bulkg"):
+        h["threads"] = d["threads"] - 32   # consumer threads (warp 0 is the producer)
     return h
 
 

@@ -510,7 +510,7 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
                 : ci.kernel == KK_BULKQ ? 5
                 : ci.kernel == KK_BULKG ? 6
                                         : 0;
-    if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = 0;  // consumers + producer
+    if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = ci.threads - 32;  // consumers
     if (ci.kernel == KK_DEINT) {  // no slice parameters: the structure size fixes the slice
       ttlg_plan_hints_init(&h);
       h.variant = 4;

@@ -1002,9 +1002,12 @@ __global__ void __launch_bounds__(544, 1) k_bulk(const __grid_constant__ TilePar
   auto full_bar = [&](int st) { return s_bar + 16u * st; };
   auto empty_bar = [&](int st) { return s_bar + 16u * st + 8u; };
 
+  const bool tma = P.tma_rows != 0;
   if (tid == 0) {
     for (int st = 0; st < NS; st++) {
-      mbar_init(full_bar(st), 1);
+      // TMA rows: one arrive (+ the tile's transaction bytes); cp.async rows:
+      // one arrive per producer lane when its copies land, + lane 0's context arrive
+      mbar_init(full_bar(st), tma ? 1 : 33);
       mbar_init(empty_bar(st), NC);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -1027,8 +1030,58 @@ __global__ void __launch_bounds__(544, 1) k_bulk(const __grid_constant__ TilePar
   }
   __syncthreads();
 
+  if (warp == 0 && !tma) {
+    // ---- producer (short rows): 16-byte cp.async over the tile's chunks (a
+    // flat walk, chunk e = lane + 32 i -> A-row e / LAc, chunk e mod LAc),
+    // completion tracked by the stage's mbarrier (cp.async.mbarrier.arrive)
+    int st = 0;
+    uint32_t ph = 0;
+    const int LAc = P.LA / K, nch = P.RA * LAc;
+    const int r0 = (int)fdiv1(lane, P.fd_LA), x0 = lane - r0 * LAc;
+    const int dr = 32 / LAc, dx = 32 % LAc;
+    const int nA = lane < nch ? (nch - 1 - lane) / 32 + 1 : 0;
+    for (uint32_t tile = blockIdx.x, k = 0; tile < P.num_tiles; tile += gridDim.x, k++) {
+      if (k >= (uint32_t)NS) mbar_wait(empty_bar(st), ph ^ 1u);
+      const TileCtx c = decode_tile(P, tile);
+      const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+      const int limc = full ? LAc : (P.LAunit * c.limA) / K;
+      if (lane == 0) {
+        ctx[st].bA = c.bA;
+        ctx[st].bB = c.bB;
+        ctx[st].limA = c.limA;
+        ctx[st].limB = c.limB;
+        mbar_arrive(full_bar(st));
+      }
+      const uint4 *Ab = reinterpret_cast<const uint4 *>(A + c.bA * S);
+      const uint32_t dst = s_data + (uint32_t)st * P.stage_bytes;
+      int r = r0, x = x0;
+#pragma unroll 4
+      for (int i = 0; i < nA; i++) {
+        const int2 t = lds_int2(s_tabA + 8 * r);
+        const uint4 *g = wadd(Ab, ((uint32_t)t.x >> LGK) + x);
+        if (full)
+          cp_async<16>(dst + t.y + 16 * x, g);
+        else
+          cp_async_p<16>(dst + t.y + 16 * x, g, x < limc && lds_int(s_digB + 4 * r) < c.limB);
+        x += dx;
+        r += dr;
+        if (x >= LAc) {
+          x -= LAc;
+          r++;
+        }
+      }
+      asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(full_bar(st))
+                   : "memory");
+      if (++st == NS) {
+        st = 0;
+        ph ^= 1u;
+      }
+    }
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
+    return;
+  }
   if (warp == 0) {
-    // ---- producer: one TMA bulk copy per A-row
+    // ---- producer (long rows): one TMA bulk copy per A-row
     int st = 0;
     uint32_t ph = 0;
     const int RA = P.RA;

@@ -190,6 +190,16 @@ static bool bulk_auto() {
   return v == 1;
 }
 constexpr int kBulkMaxStages = 6;
+constexpr int64_t kBulkTmaRowBytes = 2048;
+// TTLG_BULK_TMA=0/1 forces cp.async / TMA rows in k_bulk (experiments); -1: by row length
+static int bulk_tma_mode() {
+  static int v = -2;
+  if (v == -2) {
+    const char *e = getenv("TTLG_BULK_TMA");
+    v = (e && (e[0] == '0' || e[0] == '1')) ? e[0] - '0' : -1;
+  }
+  return v;
+}
 
 namespace {
 
@@ -603,10 +613,14 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     const int L = kind == KK_BULKQ ? K.LB : K.LB * P.W / 16;
     if (L > ntc) return false;
     K.qk = kind == KK_BULKQ ? qk : 0;
+    // TMA bulk copies cost ~40 SM cycles each (measured: 256-byte rows move
+    // 1.9 TB/s): only rows of >= kBulkTmaRowBytes go through TMA
+    K.tma_rows = bulk_tma_mode() == 1 ||
+                 (bulk_tma_mode() < 0 && (int64_t)K.LAunit * T.t[T.a] * P.W >= kBulkTmaRowBytes);
     K.rsB = ntc / L;
+    K.fd_LA = make_fastdiv((uint32_t)(K.LA * P.W / 16));  // producer walk: chunks per A-row
     K.fd_LB = make_fastdiv((uint32_t)L);
     K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
-    K.fd_LA = make_fastdiv((uint32_t)K.LA);
     K.fd_NT = make_fastdiv((uint32_t)ntc);
     return true;
   }
@@ -888,6 +902,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
     mi.nstage = 0;
     if (kind == KK_BULKQ || kind == KK_BULKG) {
+      // one output position (quad) / 16-byte output chunk (gather) per consumer thread
+      if ((kind == KK_BULKQ ? S.LB : S.LB * P.W / 16) > threads - 32) return false;
       // as many ring stages as fit next to the tables (2..kBulkMaxStages), one CTA per SM
       const int buf = (S.buf_bytes + 127) / 128 * 128;
       const int fixed = S.smem_base - S.buf_bytes + 256;
@@ -1114,10 +1130,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         if (m >= 192 && m % 8 == 0 && m != 256) tl[ntl++] = (int)m;
       }
     }
-    if (bulk) {  // producer warp + 256 / 512 consumers
-      tl[0] = 32 + 256;
+    if (bulk) {  // producer warp + 256 / 512 consumers (hints->threads: the consumers)
+      tl[0] = 32 + ((hints && hints->threads) ? hints->threads : 256);
       tl[1] = 32 + 512;
-      ntl = 2;
+      ntl = (hints && hints->threads) ? 1 : 2;
     }
     for (int ki = 0; ki < nk; ki++) {
       for (int ti = 0; ti < ntl; ti++) {

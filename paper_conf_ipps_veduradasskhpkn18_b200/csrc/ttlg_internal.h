@@ -121,6 +121,7 @@ struct TileParams {
   // k_bulk: ring of nstage tile buffers (stage_bytes apart, from off_data),
   // 2 * nstage mbarriers at off_bar (full[s], empty[s]); warp 0 produces
   int32_t nstage, stage_bytes, off_bar;
+  int32_t tma_rows;  // 1: one TMA bulk copy per A-row; 0: 16-byte cp.async chunks
 };
 
 // Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;
