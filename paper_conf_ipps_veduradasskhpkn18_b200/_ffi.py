@@ -78,7 +78,8 @@ class PlanInfo(ctypes.Structure):
             "grid": self.grid, "threads": self.threads, "smem_bytes": self.smem_bytes,
             "bytes": self.bytes, "predicted_seconds": self.predicted_seconds,
             "candidates": self.candidates, "param_bytes": self.param_bytes,
-            "kernel": ["direct", "tile", "pipe", "quad", "deint", "bulkq", "bulkg"][self.kernel],
+            "kernel": ["direct", "tile", "pipe", "quad", "deint", "bulkq", "bulkg",
+                       "vec"][self.kernel],
             "occupancy": self.occupancy,
             "features": [float(x) for x in self.features[:self.num_features]],
         }

@@ -509,6 +509,7 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
                 : ci.kernel == KK_QUAD  ? 3
                 : ci.kernel == KK_BULKQ ? 5
                 : ci.kernel == KK_BULKG ? 6
+                : ci.kernel == KK_VEC   ? 7
                                         : 0;
     if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = ci.threads - 32;  // consumers
     if (ci.kernel == KK_DEINT) {  // no slice parameters: the structure size fixes the slice

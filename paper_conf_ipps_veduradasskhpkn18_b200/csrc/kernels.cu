@@ -789,6 +789,145 @@ __global__ void __launch_bounds__(512, 4) k_quad(const __grid_constant__ TilePar
   }
 }
 
+// k_vec (any schema -- OD, OA, FMS -- whose A-rows and B-rows all start on
+// 16-byte boundaries and are whole 16-byte chunks; DESIGN.md "vector
+// gathers"): the staged tile with 16-byte global accesses both ways but no
+// register transpose.  Load: the tile's A-rows move as 16-byte cp.async
+// chunks (as k_quad).  Store: a thread owns one 16-byte chunk of the output
+// run -- K = 16/S consecutive output positions, their shared-memory column
+// offsets held in registers -- and writes it for B-rows r0, r0 + rsB, ...:
+// K element reads from shared memory, one 16-byte st.global.cs.  This is the
+// Alg. 6 (FMS) data movement for pencils that are not a multiple of 16 bytes
+// (e.g. [3, 4096, 4096] fp32 `0 2 1`: 12-byte pencils, rows of 4m pencils),
+// with every global instruction moving 16 bytes instead of 4.
+template <int S>
+__global__ void __launch_bounds__(512, 4) k_vec(const __grid_constant__ TileParams P,
+                                                const __grid_constant__ BatchPtrs X) {
+  constexpr int K = 16 / S, LGK = K == 4 ? 2 : 1;
+  const unsigned char *A = reinterpret_cast<const unsigned char *>(X.A[blockIdx.y]);
+  unsigned char *B = reinterpret_cast<unsigned char *>(X.B[blockIdx.y]);
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_buf = s0 + P.off_data;
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
+  const int tid = threadIdx.x, NT = blockDim.x;
+  const bool decoder = tid == NT - 1;
+  const uint32_t first = blockIdx.x * (uint32_t)P.tpc;
+
+  auto put_ctx = [&](int slot, uint32_t tile) {
+    const TileCtx c = decode_tile(P, tile);
+    ctx[slot].bA = c.bA;
+    ctx[slot].bB = c.bB;
+    ctx[slot].limA = c.limA;
+    ctx[slot].limB = c.limB;
+  };
+  auto get_ctx = [&](int slot) {
+    TileCtx c;
+    c.bA = ctx[slot].bA;
+    c.bB = ctx[slot].bB;
+    c.limA = ctx[slot].limA;
+    c.limB = ctx[slot].limB;
+    return c;
+  };
+  pdl_trigger();
+  if (decoder && first < P.num_tiles) put_ctx(0, first);
+  build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk, reinterpret_cast<int2 *>(smem),
+             reinterpret_cast<int *>(smem + P.off_digB), S);
+  __syncthreads();  // tabA, digB, ctx[0] visible
+  pdl_wait();
+
+  const int LB = P.LB, LAc = P.LA / K, LBc = LB / K;
+  const int nChunks = P.V / K;
+  const int rA0 = (int)fdiv1(tid, P.fd_LA), cA0 = tid - rA0 * LAc;
+  const int nA = tid < nChunks ? (int)fdiv1(nChunks - 1 - tid, P.fd_NT) + 1 : 0;
+  const int drA = P.drA, dxA = P.dxA;
+  auto load = [&](const TileCtx &c, bool full) {
+    const uint4 *Ab = reinterpret_cast<const uint4 *>(A + c.bA * S);
+    const int limc = full ? LAc : (P.LAunit * c.limA) / K;
+    int r = rA0, cx = cA0;
+#pragma unroll 4
+    for (int k = 0; k < nA; k++) {
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const uint32_t soff = t.y + cx * 16;
+      const uint4 *g = wadd(Ab, ((uint32_t)t.x >> LGK) + cx);
+      if (full)
+        cp_async<16>(s_buf + soff, g);
+      else
+        cp_async_p<16>(s_buf + soff, g, cx < limc && lds_int(s_digB + 4 * r) < c.limB);
+      cx += dxA;
+      r += drA;
+      if (cx >= LAc) {
+        cx -= LAc;
+        r++;
+      }
+    }
+  };
+  TileCtx c = get_ctx(0);
+  bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+  if (first < P.num_tiles) load(c, full);
+  cp_async_commit();
+
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA), S);
+#pragma unroll 1
+  for (int j = tid; j < LB; j += NT) {
+    int rem = j, sm = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+      sm += (rem - cq * (int)P.j_div[k].div) * P.j_sS[k];
+      rem = cq;
+    }
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = sm * S;
+  }
+  __syncthreads();  // tabB, digA, jcol visible (the first tile's loads still in flight)
+
+  // store walk: output chunk q = tid mod LBc (positions K q .. K q + K - 1), B-rows m0 + k rs
+  const int m0 = (int)fdiv1(tid, P.fd_LB);
+  const int j0 = (tid - m0 * LBc) * K;
+  const int rs = P.rsB;
+  const int nB = (m0 < rs && m0 < P.RB) ? (int)fdiv1(P.RB - 1 - m0, P.fd_rsB) + 1 : 0;
+  uint32_t jc[K];
+#pragma unroll
+  for (int u = 0; u < K; u++) jc[u] = lds_int(s_jcol + 4 * (j0 + u < LB ? j0 + u : 0));
+
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = first + it;
+    if (tile >= P.num_tiles) break;
+    if (it > 0) {
+      __syncthreads();  // buffer drained, ctx[it & 1] visible
+      c = get_ctx(it & 1);
+      full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+      load(c, full);
+      cp_async_commit();
+    }
+    if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
+    cp_async_wait<0>();
+    __syncthreads();
+    const bool jok = full || j0 < P.LBunit * c.limB;
+    uint4 *dst = reinterpret_cast<uint4 *>(B + (c.bB + j0) * S);
+    int r = m0;
+#pragma unroll 4
+    for (int k = 0; k < nB; k++) {
+      const int2 t = lds_int2(s_tabB + 8 * r);
+      const uint32_t sr = s_buf + t.y;
+      uint4 v;
+      if constexpr (S == 8) {
+        const uint2 a = lds_T<uint2>(sr + jc[0]), b = lds_T<uint2>(sr + jc[1]);
+        v = make_uint4(a.x, a.y, b.x, b.y);
+      } else {
+        v = make_uint4(lds_T<unsigned int>(sr + jc[0]), lds_T<unsigned int>(sr + jc[1]),
+                       lds_T<unsigned int>(sr + jc[2]), lds_T<unsigned int>(sr + jc[3]));
+      }
+      stcs_p(wadd(dst, (uint32_t)t.x >> LGK), v,
+             jok && (full || lds_int(s_digA + 4 * r) < c.limA));
+      r += rs;
+    }
+  }
+}
+
 // k_deint (Orthogonal-Arbitrary with a tiny input FVI: array-of-structures ->
 // structure-of-arrays): the fused problem [n0, M] perm (1 0), or the batch
 // [n0, M, nb] perm (1 0 2), with N0 = n0 <= 8 and M a multiple of K = 16/S.
@@ -1292,7 +1431,7 @@ int kernel_regs(int kind, int W) {
   static std::atomic<int> regs[KK_NUM][3] = {{{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
-                                             {{-1}, {-1}, {-1}}};
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
   if (r >= 0) return r;
@@ -1305,6 +1444,7 @@ int kernel_regs(int kind, int W) {
                      : kind == KK_DEINT ? deint_ptr(W == 8 ? 8 : 4, 4)
                      : (kind == KK_BULKQ || kind == KK_BULKG)
                          ? bulk_ptr(W, kind)
+                     : kind == KK_VEC ? (W == 8 ? (const void *)k_vec<8> : (const void *)k_vec<4>)
                          : kernel_ptr(kind, W, false, false);
     if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
       r = attr.numRegs;
@@ -1338,6 +1478,8 @@ ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *c
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
                        : (plan->kind == KK_BULKQ || plan->kind == KK_BULKG)
                              ? bulk_ptr(plan->W, plan->kind)
+                       : plan->kind == KK_VEC
+                             ? (plan->W == 8 ? (const void *)k_vec<8> : (const void *)k_vec<4>)
                        : plan->kind == KK_DEINT
                              ? (plan->kp.deint_inter ? inter_ptr(plan->W, plan->kp.deint_n0)
                                                      : deint_ptr(plan->W, plan->kp.deint_n0))

@@ -39,7 +39,7 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
     read_bytes = tiles * fill * mi.RA * run_cost((int64_t)mi.LA * mi.W);
     runsA = tiles * fill * mi.RA;
     // flat load walk: ceil(V / threads) access elements (k_quad: 16-byte chunks) per thread
-    const double vk = mi.kind == KK_QUAD ? (double)mi.V / std::max(1, mi.qk) : (double)mi.V;
+    const double vk = mi.qk > 0 ? (double)mi.V / mi.qk : (double)mi.V;  // 16-byte chunks
     opsA = tiles * std::ceil(vk / mi.threads) * (mi.threads / 32.0);
   }
   const double write_bytes = tiles * fill * mi.RB * run_cost((int64_t)mi.LB * mi.W);
@@ -48,6 +48,10 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
   if (mi.kind == KK_DIRECT) {
     const double gB = group(mi.LB);
     opsB = tiles * mi.RB * std::ceil(mi.LB / gB) / (32.0 / gB);
+  } else if (mi.kind == KK_VEC || mi.kind == KK_BULKG) {
+    // one 16-byte output chunk per thread, B-rows strided by threads / chunks-per-row
+    const double rs = std::floor((double)mi.threads * std::max(1, mi.qk) / mi.LB);
+    opsB = tiles * std::ceil(mi.RB / std::max(1.0, rs)) * (mi.threads / 32.0);
   } else if (mi.LB <= mi.threads) {
     // one output position per thread, B-rows (k_quad: groups of K B-rows) strided by threads / LB
     const double rs = std::floor((double)mi.threads / mi.LB);

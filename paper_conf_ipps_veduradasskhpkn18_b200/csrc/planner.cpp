@@ -179,12 +179,12 @@ static void dense_prefixes(Problem &P) {
     P.denseB++;
 }
 
-// k_bulk joins the automatic choice only with TTLG_BULK=1 until the model is
-// calibrated on it (forced with hints variant 5 / 6 otherwise)
-static bool bulk_auto() {
+// k_bulk / k_vec join the automatic choice only with TTLG_NEW_KERNELS=1 until
+// the model is calibrated on them (forced with hints variant 5 / 6 / 7 otherwise)
+static bool new_kernels_auto() {
   static int v = -1;
   if (v < 0) {
-    const char *e = getenv("TTLG_BULK");
+    const char *e = getenv("TTLG_NEW_KERNELS");
     v = (e && e[0] == '1') ? 1 : 0;
   }
   return v == 1;
@@ -298,7 +298,7 @@ int quad_k(const Problem &P, const Tile &T) {
 // consumer mode quad needs k_quad's 16-byte chunks on the B side, mode gather
 // the same row alignment for B-rows.  No padded input runs (a bulk copy lands
 // one contiguous row).
-static bool bulk_ok(const Problem &P, const Tile &T, int kind) {
+static bool bulk_ok(const Problem &P, const Tile &T, int kind) {  // also k_vec (kind KK_VEC)
   const int W = P.W, pb = P.p[T.b];
   bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
   for (int k = 0; k <= T.a; k++) inIS[k] = true;
@@ -312,6 +312,7 @@ static bool bulk_ok(const Problem &P, const Tile &T, int kind) {
     if (P.n[k] > T.t[k] && (T.t[k] * P.sA[k] * W) % 16) return false;  // tile base
   }
   if (kind == KK_BULKQ) return P.W == P.esize && quad_k(P, T) == 16 / W;
+  if (kind == KK_VEC && W != 4 && W != 8) return false;
   if ((LBunit * T.t[pb] * W) % 16 || (LBunit * (P.n[pb] % T.t[pb]) * W) % 16) return false;
   for (int k = 0; k < P.d; k++) {
     if (T.t[k] > 1 && !inOS[k] && (P.sB[k] * W) % 16) return false;  // B-row digit
@@ -370,7 +371,7 @@ struct TileSummary {
 // every A-row on a 16-byte (chunk) boundary
 static int layout_unit(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_QUAD) return quad_k(P, T);
-  if (kind == KK_BULKQ || kind == KK_BULKG) return 16 / P.W;
+  if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_VEC) return 16 / P.W;
   return 0;
 }
 
@@ -421,6 +422,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   if (kind == KK_QUAD && qk == 0) return false;
   const bool bulk = kind == KK_BULKQ || kind == KK_BULKG;
   if (bulk && (isdelta || !bulk_ok(P, T, kind))) return false;
+  if (kind == KK_VEC && (isdelta || !bulk_ok(P, T, KK_VEC))) return false;
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
   bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
@@ -622,6 +624,20 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.fd_LB = make_fastdiv((uint32_t)L);
     K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
     K.fd_NT = make_fastdiv((uint32_t)ntc);
+    return true;
+  }
+  if (kind == KK_VEC) {
+    // load walk over 16-byte chunks; store walk: one output chunk per thread
+    const int K16 = 16 / P.W, LAc = K.LA / K16, LBc = K.LB / K16;
+    if (LBc > threads || threads % 32) return false;
+    K.qk = K16;
+    K.drA = threads / LAc;
+    K.dxA = threads % LAc;
+    K.fd_LA = make_fastdiv((uint32_t)LAc);
+    K.rsB = threads / LBc;
+    K.fd_LB = make_fastdiv((uint32_t)LBc);
+    K.fd_NT = make_fastdiv((uint32_t)threads);
+    K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
     return true;
   }
   if (kind == KK_QUAD) {  // the load walk runs over chunks
@@ -915,7 +931,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (smem > dev.smem_per_block_optin) return false;
     // k_quad: at most 4 output positions per thread, warp-wide shuffles (whole warps)
     if (kind == KK_QUAD && (S.LB > 4 * threads || threads % 32)) return false;
-    mi.qk = kind == KK_QUAD ? S.qk : 0;
+    if (kind == KK_VEC && (S.LB * P.W / 16 > threads || threads % 32)) return false;
+    mi.qk = (kind == KK_QUAD || kind == KK_VEC || kind == KK_BULKQ || kind == KK_BULKG) ? S.qk : 0;
     mi.kind = kind;
     mi.schema = schema;
     mi.W = P.W;
@@ -968,7 +985,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     if (!build_params(P, T, group, thr_list[0], 1, K0)) return false;
     if (group == KK_DIRECT) return true;
-    if (group == KK_QUAD) {  // conflict-free by construction (16-byte slot j mod 8)
+    if (group == KK_QUAD || group == KK_VEC) {  // chunk layout: no input-run padding
       S.smem_base = K0.smem_bytes;
       S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
       return true;
@@ -1061,11 +1078,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
     if (hv == 4) return;  // k_deint forced: no staged / direct candidates
     const bool bulk = group == KK_BULKQ || group == KK_BULKG;
-    if (bulk) {
+    if (bulk || group == KK_VEC) {
       if (forceW) return;  // element-width fallback plans: no 16-byte requirement
-      if (hv == 0 ? !bulk_auto() : hv != (group == KK_BULKQ ? 5 : 6)) return;
+      const int want = group == KK_BULKQ ? 5 : (group == KK_BULKG ? 6 : 7);
+      if (hv == 0 ? !new_kernels_auto() : hv != want) return;
     } else if (hv >= 5) {
-      return;  // k_bulk forced
+      return;  // k_bulk / k_vec forced
     }
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
@@ -1108,7 +1126,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (!build_exact(T, group, K0, delta, cl, cs, S)) return;
     }
     int kinds[2], nk = 0;
-    if (bulk) {
+    if (bulk || group == KK_VEC) {
       kinds[nk++] = group;
     } else if (group == KK_DIRECT) {
       kinds[nk++] = KK_DIRECT;
@@ -1194,10 +1212,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           // factor, drawn from both candidate lists
           for (int i = 0; i < nbA; i++) {
             consider(KK_TILE, a, blocksA[i], b, blocksA[i]);
+            consider(KK_VEC, a, blocksA[i], b, blocksA[i]);
             consider(KK_BULKG, a, blocksA[i], b, blocksA[i]);
           }
           for (int j = 0; j < nbB; j++) {
             consider(KK_TILE, a, blocksB[j], b, blocksB[j]);
+            consider(KK_VEC, a, blocksB[j], b, blocksB[j]);
             consider(KK_BULKG, a, blocksB[j], b, blocksB[j]);
           }
         } else {
@@ -1207,6 +1227,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
               consider(KK_QUAD, a, blocksA[i], b, blocksB[j]);
               consider(KK_BULKQ, a, blocksA[i], b, blocksB[j]);
               consider(KK_BULKG, a, blocksA[i], b, blocksB[j]);
+              consider(KK_VEC, a, blocksA[i], b, blocksB[j]);
               // k_quad needs whole chunks per run: the same slice with the
               // blocking factors rounded up to a chunk multiple (e.g. t1 = 22
               // -> 24 for [3, 4096, 4096] fp32 `2 1 0`)
@@ -1218,6 +1239,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                   consider(KK_QUAD, a, ra, b, rb);
                   consider(KK_BULKQ, a, ra, b, rb);
                   consider(KK_BULKG, a, ra, b, rb);
+                  consider(KK_VEC, a, ra, b, rb);
                 }
               }
             }
@@ -1457,7 +1479,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
   plan->align = B.kind == KK_QUAD ? K.qk * P.W
-                : (B.kind == KK_BULKQ || B.kind == KK_BULKG) ? 16
+                : (B.kind == KK_BULKQ || B.kind == KK_BULKG || B.kind == KK_VEC) ? 16
                                                              : P.W;
   plan->threads = B.mi.threads;
   plan->grid = B.mi.grid;

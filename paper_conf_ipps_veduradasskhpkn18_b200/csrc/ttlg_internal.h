@@ -55,7 +55,9 @@ enum KernelKind : int32_t {
                   // 16-byte stores (k_bulk, consumer mode quad)
   KK_BULKG = 6,   // any schema: TMA bulk row loads, 16-byte stores gathered from K
                   // element reads (k_bulk, consumer mode gather)
-  KK_NUM = 7,
+  KK_VEC = 7,     // any schema with 16-byte aligned rows: 16-byte cp.async loads, 16-byte
+                  // stores gathered from K element reads (k_vec)
+  KK_NUM = 8,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel

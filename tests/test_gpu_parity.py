@@ -333,7 +333,7 @@ _VARIANT_CASES = [
 ]
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 5, 6])
+@pytest.mark.parametrize("variant", [1, 2, 3, 5, 6, 7])
 @pytest.mark.parametrize("ext,perm,eb", _VARIANT_CASES)
 def test_kernel_variants_forced(ext, perm, eb, variant):
     try:
@@ -557,18 +557,19 @@ def _bulk_cases():
     return out + [configs.scaled(c, 1 << 18) for c in configs.sweep720(16)[::37]]
 
 
-@pytest.mark.parametrize("variant", [5, 6])
+@pytest.mark.parametrize("variant", [5, 6, 7])
 @pytest.mark.parametrize("case", _bulk_cases(), ids=lambda c: c.label())
 def test_bulk_forced(case, variant):
     """k_bulk (TMA bulk row loads into an mbarrier ring; 5 = quad consumers,
-    6 = gather consumers) forced on every config shape it applies to."""
+    6 = gather consumers) and k_vec (7: 16-byte cp.async loads, gathered
+    16-byte stores) forced on every config shape they apply to."""
     try:
         ttlg.plan(_dt(case.elem_bytes), case.extents, case.perm, variant=variant)
     except ttlg.TtlgError:
-        pytest.skip("k_bulk not applicable (rows not 16-byte aligned)")
+        pytest.skip("k_bulk / k_vec not applicable (rows not 16-byte aligned)")
     got, exp, info = _run(case.extents, case.perm, case.elem_bytes, case_seed(case.case_id),
                           plan_kwargs={"variant": variant}, canary=64)
-    assert info["kernel"] == ("bulkq" if variant == 5 else "bulkg")
+    assert info["kernel"] == {5: "bulkq", 6: "bulkg", 7: "vec"}[variant]
     _assert_equal(got, exp, f"bulk {variant} {info}")
 
 
@@ -579,7 +580,7 @@ def test_bulk_partial_tiles(eb):
     n_ok = 0
     for ext, perm in (([6 * K, 40, 7], [1, 0, 2]), ([4 * K, 30, 3 * K], [2, 1, 0]),
                       ([2 * K, 50, 60], [0, 2, 1]), ([3, 4 * K * 11, 4 * K * 9], [2, 1, 0])):
-        for variant in (5, 6):
+        for variant in (5, 6, 7):
             for ib, ob in ((None, None), (3, 5), (K, 2 * K), (2 * K, 3 * K)):
                 kw = {"variant": variant}
                 if ib:

@@ -110,15 +110,32 @@ GPU_CASES = [
 ]
 
 
-def _gpu_worker(rank, world, port, q):
+def _cases_for(world):
+    """GPU_CASES whose sharded extents P divides (plan_shards' precondition)."""
+    out = []
+    for ci, (ext, perm) in enumerate(GPU_CASES):
+        try:
+            plan_shards(ext, perm, world)
+        except ValueError:
+            continue
+        out.append((ci, (ext, perm)))
+    return out
+
+
+def _gpu_worker(rank, world, port, q, backend="gloo", own_device=False):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
-    torch.cuda.set_device(0)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dev = rank if own_device else 0
+    torch.cuda.set_device(dev)
+    if backend == "nccl":
+        dist.init_process_group("nccl", rank=rank, world_size=world,
+                                device_id=torch.device("cuda", dev))
+    else:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_ipps_veduradasskhpkn18_b200.sharded import P2PExchange
     try:
         results = []
-        for ci, (ext, perm) in enumerate(GPU_CASES):
+        for ci, (ext, perm) in _cases_for(world):
             sp = plan_shards(ext, perm, world)
             n = int(np.prod(ext))
             full = gen_tensor_np(300 + ci, n, 8)
@@ -137,8 +154,13 @@ def _gpu_worker(rank, world, port, q):
             torch.cuda.synchronize()
             dist.barrier()
             for B in (B1, B2):
-                gathered = [torch.empty(sp.n_local, dtype=torch.float64) for _ in range(world)]
-                dist.all_gather(gathered, B.cpu())
+                if backend == "nccl":
+                    gathered = [torch.empty_like(B) for _ in range(world)]
+                    dist.all_gather(gathered, B)
+                    gathered = [g.cpu() for g in gathered]
+                else:
+                    gathered = [torch.empty(sp.n_local, dtype=torch.float64) for _ in range(world)]
+                    dist.all_gather(gathered, B.cpu())
                 if rank == 0:
                     got = torch.cat(gathered).numpy().view(np.uint64)
                     results.append(bool(np.array_equal(got, expect)))
@@ -166,4 +188,28 @@ def test_sharded_gpu_two_processes_one_device():
     for p in procs:
         p.join(timeout=120)
     assert isinstance(res, list), res
-    assert len(res) == 2 * len(GPU_CASES) and all(res), res
+    assert len(res) == 2 * len(_cases_for(2)) and all(res), res
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_sharded_nccl_one_process_per_gpu(world):
+    """The multi-GPU path as bench.py runs it: one process per device, NCCL
+    all_to_all_single for the all-to-all exchange and CUDA IPC peer mappings
+    across devices (NVLink stores) for the fused exchange, both bit-exact
+    against the global oracle.  Needs `world` visible devices (skips otherwise:
+    every gpurun box of this build has one)."""
+    if torch.cuda.device_count() < world:
+        pytest.skip(f"needs {world} CUDA devices, {torch.cuda.device_count()} visible")
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_gpu_worker, args=(r, world, port, q, "nccl", True))
+             for r in range(world)]
+    for p in procs:
+        p.start()
+    res = q.get(timeout=900)
+    for p in procs:
+        p.join(timeout=120)
+    assert isinstance(res, list), res
+    assert len(res) == 2 * len(_cases_for(world)) and all(res), res

@@ -25,6 +25,10 @@ def main():
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--max-cand", type=int, default=120)
     ap.add_argument("--stride", type=int, default=1)
+    ap.add_argument("--variants", default="5,6",
+                    help="comma list of forced kernel variants to enumerate (0 = every "
+                         "non-bulk candidate)")
+    ap.add_argument("--only", default=None, help="comma-separated case ids")
     args = ap.parse_args()
 
     import torch
@@ -54,7 +58,12 @@ def main():
                 ts.append(e0.elapsed_time(e1) * 1e-3 / args.reps)
         return statistics.median(ts)
 
-    for c in workload(args.workload)[::args.stride]:
+    cases = workload(args.workload)[::args.stride]
+    if args.only:
+        keep = {int(x) for x in args.only.split(",")}
+        cases = [c for c in cases if c.case_id in keep]
+    variants = [int(v) for v in args.variants.split(",")]
+    for c in cases:
         dt = "f64" if c.elem_bytes == 8 else "f32"
         A = gen_tensor_torch(case_seed(c.case_id), c.n_elems, c.elem_bytes, device="cuda:0")
         B = torch.empty_like(A)
@@ -62,9 +71,10 @@ def main():
         ai = auto.describe()
         ta = gtime(auto, A, B)
         best = None
-        for v in (5, 6):
+        for v in variants:
             try:
-                cands = ttlg.plan_candidates(dt, c.extents, c.perm, variant=v)
+                cands = ttlg.plan_candidates(dt, c.extents, c.perm,
+                                             **({"variant": v} if v else {}))
             except ttlg.TtlgError:
                 continue
             if len(cands) > args.max_cand:
@@ -92,7 +102,7 @@ def main():
                     best = row
         print(json.dumps({"summary": c.label(), "auto_kernel": ai["kernel"],
                           "auto_gbs": c.alg_bytes / ta / 1e9,
-                          "best_bulk": None if best is None else
+                          "best": None if best is None else
                           {k: best[k] for k in ("kernel", "gbs", "tile", "threads", "LA_bytes",
                                                 "LB_bytes", "V_bytes")}}), flush=True)
         del A, B
