@@ -196,18 +196,19 @@ def run_reference(args, rank, world):
 def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
     """--workload sharded: BASELINE config 5, the 8 GiB rank-5 fp32 tensor
     [64,64,64,64,128] sharded on A's outermost dim across the ranks (one
-    process per GPU).  No-move perms: one local transposition per rank, no
-    communication.  Moved perms: the fused exchange (sub-transpositions storing
-    into the peers' B slabs over CUDA IPC / NVLink) and, for comparison, local
-    transpose -> NCCL all_to_all_single -> fold.  Also, on rank 0: the fused
-    exchange of P = 2/4/8 emulated on this one GPU (every peer slab local) --
-    the HBM-side cost of its sub-box launches."""
+    process per GPU; the default workload at N > 1).  No-move perms: one local
+    transposition per rank, no communication.  Moved perms: the model-chosen
+    exchange -- the fused one (ONE batched launch per rank whose
+    sub-transpositions store straight into the peers' B slabs over CUDA IPC /
+    NVLink) or local transpose -> NCCL all_to_all_single -> fold.  A step =
+    the five perms once.  At N = 1 also: the fused exchange of P = 2/4/8
+    emulated on this one GPU (every peer slab local) -- its HBM-side cost."""
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_veduradasskhpkn18_b200 as ttlg
     from paper_conf_ipps_veduradasskhpkn18_b200.sharded import (
         plan_shards, P2PExchange, map_peer_slabs, unmap_peer_slabs, sharded_transpose,
-        choose_exchange)
+        choose_exchange, NVLINK_GBS)
     from synth import configs, gen_tensor_torch, case_seed
 
     cases = configs.config5()
@@ -222,9 +223,12 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
     B = torch.empty_like(A)
     if world > 1:
         peers, opened = map_peer_slabs(B)
+        nccl_info = {"backend": dist.get_backend(), "communicator_size": dist.get_world_size()}
     else:
         peers, opened = [B.data_ptr()], []
+        nccl_info = None
     work = (torch.empty_like(A), torch.empty_like(A)) if world > 1 else None
+
     def make_ex(perm, out, ptrs, r, P):
         try:
             return P2PExchange(ext, perm, out, peer_ptrs=ptrs, rank=r, world=P)
@@ -244,12 +248,21 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
         e1.record(stream)
         torch.cuda.synchronize()
         ms = e0.elapsed_time(e1)
-        if world > 1:
+        if world > 1:  # the step time is the slowest rank's
             t = torch.tensor([ms], device=dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms = float(t.item())
             dist.barrier()
         return ms
+
+    def fns_for(c, ex):
+        def f_p2p():
+            ex.run(A, sptr)
+
+        def f_a2a():
+            with torch.cuda.stream(stream):
+                sharded_transpose(A, ext, c.perm, work=work)
+        return {"p2p": f_p2p, "local": f_p2p, "alltoall": f_a2a}
 
     per, other, modes = [], {}, {}
     clocks = ClockSampler(local_rank)
@@ -257,17 +270,10 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
     time.sleep(0.3)
     for c, ex in zip(cases, exs):
         key = "".join(map(str, c.perm))
-
-        def f_p2p(ex=ex):
-            ex.run(A, sptr)
-
-        def f_a2a(c=c):
-            with torch.cuda.stream(stream):
-                sharded_transpose(A, ext, c.perm, work=work)
         # model-driven choice between the fused exchange and the all-to-all
         mode = choose_exchange(ext, c.perm, world, "f32")["mode"] if world > 1 else "local"
         modes[key] = mode
-        fns = {"p2p": f_p2p, "local": f_p2p, "alltoall": f_a2a}
+        fns = fns_for(c, ex)
         for _ in range(args.warmup):
             fns[mode]()
         per.append(timed(fns[mode], args.steps))
@@ -280,6 +286,54 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
     clk = clocks.stop()
     total_ms = sum(per)
     value = 2 * n * 4 * len(cases) * args.steps / (total_ms / 1e3) / 1e9
+    per_gbs = {"".join(map(str, c.perm)): 2 * n * 4 * args.steps / (m / 1e3) / 1e9
+               for c, m in zip(cases, per)}
+    # roofline: the local (no-move) transpositions are HBM-bound -- bytes of one
+    # rank / that rank's time vs the measured HBM peak; moved perms are bound
+    # by NVLink: bus bandwidth = remote bytes per rank / time vs 770 GB/s
+    local_keys = [k for k in per_gbs if modes[k] == "local"]
+    hbm_achieved = (sum(2 * n_local * 4 * args.steps for _ in local_keys) /
+                    (sum(m for c, m in zip(cases, per) if "".join(map(str, c.perm)) in local_keys)
+                     / 1e3) / 1e9) if local_keys else None
+    nvlink = {}
+    for c, m in zip(cases, per):
+        k = "".join(map(str, c.perm))
+        if modes[k] != "local":
+            remote = n_local * 4 * (world - 1) / world * args.steps
+            nvlink[k] = {"mode": modes[k], "busbw_gbs": remote / (m / 1e3) / 1e9,
+                         "peak_gbs": NVLINK_GBS,
+                         "peak_source": "B200_PROFILING.md measured peer copy per direction"}
+
+    # end to end through the public API: each rank's slab from pinned host memory,
+    # the sharded transposition, its B slab back to pinned host memory
+    e2e = None
+    if args.e2e_steps > 0:
+        try:
+            hA = torch.empty(n_local, dtype=torch.float32, pin_memory=True)
+            hA.copy_(A)
+            hB = torch.empty(n_local, dtype=torch.float32, pin_memory=True)
+            torch.cuda.synchronize()
+
+            def e2e_step():
+                with torch.cuda.stream(stream):
+                    for c, ex in zip(cases, exs):
+                        mode = modes["".join(map(str, c.perm))]
+                        A.copy_(hA, non_blocking=True)
+                        fns_for(c, ex)[mode]()
+                        if world > 1 and mode == "p2p":
+                            # peers store into this rank's B: wait for all of them
+                            stream.synchronize()
+                            dist.barrier()
+                        hB.copy_(work[0] if mode == "alltoall" else B, non_blocking=True)
+            ms = timed(e2e_step, args.e2e_steps)
+            e2e = {"value": 2 * n * 4 * len(cases) * args.e2e_steps / (ms / 1e3) / 1e9,
+                   "unit": "GB/s", "h2d_bytes_per_step": len(cases) * n_local * 4 * world,
+                   "d2h_bytes_per_step": len(cases) * n_local * 4 * world,
+                   "steps": args.e2e_steps,
+                   "api": "per rank: pinned host slab -> H2D -> sharded transposition "
+                          "(P2PExchange.run / sharded_transpose) -> D2H of the B slab"}
+        except Exception as ex_:  # report, do not hide
+            e2e = {"value": None, "unit": "GB/s", "error": str(ex_)[:200]}
 
     emulated = {}
     if rank == 0 and world == 1 and not args.no_emulate:
@@ -304,12 +358,19 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
                 ms = timed(f_all, max(2, args.steps // 2))
                 emulated[f"P{P}:{''.join(map(str, c.perm))}"] = \
                     2 * n * 4 * max(2, args.steps // 2) / (ms / 1e3) / 1e9
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline([configs.Case(c.case_id, c.extents[:-1] + (c.extents[-1] // 8,),
+                                         c.perm, 4, c.group) for c in cases],
+                           budget_s=args.cpu_budget)
+        cpu["sample"] = "one P=8 slab [64,64,64,64,16] per perm: " + cpu["sample"]
     for ex in exs:
         if ex is not None:
             ex.close()
     unmap_peer_slabs(opened)
     if rank == 0:
         peak, peak_src, _ = _peaks()
+        launches = sum(1 if modes[k] != "alltoall" else 2 for k in modes) * args.steps
         line = {
             "metric": "effective transpose GB/s (2*N*s/time)", "value": value, "unit": "GB/s",
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
@@ -320,18 +381,25 @@ def run_sharded(args, rank, world, local_rank, dev):  # noqa: C901
                        "extents": ext, "perms": [list(c.perm) for c in cases],
                        "parallelism": f"shard x{world}",
                        "exchange": "per perm, model-chosen: local (no move) | p2p (fused "
-                                   "sub-transpositions storing over CUDA IPC) | alltoall "
-                                   "(local + NCCL all_to_all_single + fold)",
-                       "l2": "no flush: 8 GiB tensors (inputs larger than L2)"},
-            "gpu_launches": sum(len(ex.subs) if ex is not None and modes[k] != "alltoall" else 2
-                                for ex, k in zip(exs, modes)) * args.steps,
-            "per_perm_gbs": {"".join(map(str, c.perm)): 2 * n * 4 * args.steps / (m / 1e3) / 1e9
-                             for c, m in zip(cases, per)},
+                                   "sub-transpositions, one batched launch per rank storing "
+                                   "over CUDA IPC / NVLink) | alltoall (local + NCCL "
+                                   "all_to_all_single + fold)",
+                       "l2": "no flush: 8 GiB tensors (inputs larger than L2)",
+                       "process_group": nccl_info},
+            "gpu_launches": launches,
+            "per_perm_gbs": per_gbs,
             "modes": modes,
+            "roofline": {"bound": "hbm", "kernel": "local transpositions (no-move perms)",
+                         "achieved": hbm_achieved, "peak": peak, "peak_source": peak_src,
+                         "unit": "GB/s", "frac": hbm_achieved / peak if hbm_achieved else None,
+                         "traffic": None},
+            "nvlink": nvlink or None,
             "other_path_gbs": other or None,
             "p2p_emulated_one_gpu_gbs": emulated or None,
             "frac_of_peak": value / world / peak,
             "clocks": clk,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
         }
         print(json.dumps(line), flush=True)
 

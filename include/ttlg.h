@@ -119,10 +119,13 @@ typedef struct {
   int32_t candidates;                     /* number of candidates the model scored       */
   int32_t param_bytes;                    /* kernel-parameter blob size                  */
   int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe,
-                                             3 k_quad, 4 k_deint                         */
+                                             3 k_quad, 4 k_deint / k_inter, 5 k_bulk
+                                             (quad consumers), 6 k_bulk (gather
+                                             consumers), 7 k_vec                         */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[12];
+  int32_t stages;                         /* k_bulk: tile buffers in the ring; else 0    */
 } ttlg_plan_info;
 
 void ttlg_plan_hints_init(ttlg_plan_hints *hints);

@@ -60,7 +60,7 @@ class PlanInfo(ctypes.Structure):
                 ("predicted_seconds", ctypes.c_double), ("candidates", ctypes.c_int32),
                 ("param_bytes", ctypes.c_int32), ("kernel", ctypes.c_int32),
                 ("occupancy", ctypes.c_int32), ("num_features", ctypes.c_int32),
-                ("features", ctypes.c_double * 12)]
+                ("features", ctypes.c_double * 12), ("stages", ctypes.c_int32)]
 
     def to_dict(self) -> dict:
         d = self.fused_rank
@@ -80,7 +80,7 @@ class PlanInfo(ctypes.Structure):
             "candidates": self.candidates, "param_bytes": self.param_bytes,
             "kernel": ["direct", "tile", "pipe", "quad", "deint", "bulkq", "bulkg",
                        "vec"][self.kernel],
-            "occupancy": self.occupancy,
+            "occupancy": self.occupancy, "stages": self.stages,
             "features": [float(x) for x in self.features[:self.num_features]],
         }
 

@@ -98,10 +98,13 @@ ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev) {
 
 double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
   const ModelFeatures F = model_features(mi, dev);
-  const double *c = (mi.kind == KK_DIRECT) ? kCoefDirect
-                    : (mi.kind == KK_TILE) ? kCoefTile
-                    : (mi.kind == KK_QUAD) ? kCoefQuad
-                                           : kCoefPipe;
+  const double *c = (mi.kind == KK_DIRECT)  ? kCoefDirect
+                    : (mi.kind == KK_TILE)  ? kCoefTile
+                    : (mi.kind == KK_QUAD)  ? kCoefQuad
+                    : (mi.kind == KK_BULKQ) ? kCoefBulkQ
+                    : (mi.kind == KK_BULKG) ? kCoefBulkG
+                    : (mi.kind == KK_VEC)   ? kCoefVec
+                                            : kCoefPipe;
   double t = 0.0;
   for (int i = 0; i < kModelNumFeatures; i++) t += c[i] * F.f[i];
   // the model can never beat one pass of the algorithmic bytes at copy speed
@@ -140,6 +143,8 @@ void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d)
   d[13] = (RA + RB + (double)mi.LB) / th;          // per-CTA table entries per thread
   d[14] = mi.fillA;                                // useful fraction of the tile grid
   d[15] = std::ceil((double)mi.num_tiles / std::max(1, mi.grid));  // tiles per CTA
+  d[16] = std::log2(bytes);  // total traffic: launch-dominated / L2-resident below ~2x L2
+  d[17] = mi.nstage;         // k_bulk ring stages (0: other kernels)
 }
 
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {

@@ -36,7 +36,7 @@ struct ModelFeatures {
 ModelFeatures model_features(const ModelInput &mi, const DeviceProfile &dev);
 double predict_seconds(const ModelInput &mi, const DeviceProfile &dev);
 // ranking stage (boosted trees over model_descriptor); seconds
-constexpr int kGbtDesc = 16;  // descriptor length (tools/calibrate_gbt.py desc())
+constexpr int kGbtDesc = 18;  // descriptor length (tools/calibrate_gbt.py desc())
 void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d);
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
 void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);

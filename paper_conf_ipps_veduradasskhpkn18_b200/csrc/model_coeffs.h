@@ -12,5 +12,8 @@ constexpr double kCoefDirect[kModelNumFeatures] = {6.621356e-06, 8.801143e-01, 8
 constexpr double kCoefTile[kModelNumFeatures] = {8.564110e-06, 8.672552e-01, 4.235581e-02, 3.343247e-11, 0.000000e+00, 3.600222e-01, 8.875134e-02, 2.948236e-07, 3.549572e-10, 1.462520e-09};
 constexpr double kCoefPipe[kModelNumFeatures] = {7.472125e-06, 9.025470e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.375855e-01, 4.479036e-01, 0.000000e+00, 3.127622e-10, 1.671868e-09};
 constexpr double kCoefQuad[kModelNumFeatures] = {8.068869e-06, 8.957848e-01, 0.000000e+00, 1.501453e-10, 0.000000e+00, 3.723977e-01, 1.773548e-01, 2.590639e-07, 0.000000e+00, 2.316751e-09};
+constexpr double kCoefBulkQ[kModelNumFeatures] = {7.472125e-06, 9.025470e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.375855e-01, 4.479036e-01, 0.000000e+00, 3.127622e-10, 1.671868e-09};
+constexpr double kCoefBulkG[kModelNumFeatures] = {7.472125e-06, 9.025470e-01, 0.000000e+00, 0.000000e+00, 0.000000e+00, 1.375855e-01, 4.479036e-01, 0.000000e+00, 3.127622e-10, 1.671868e-09};
+constexpr double kCoefVec[kModelNumFeatures] = {8.564110e-06, 8.672552e-01, 4.235581e-02, 3.343247e-11, 0.000000e+00, 3.600222e-01, 8.875134e-02, 2.948236e-07, 3.549572e-10, 1.462520e-09};
 constexpr const char *kModelSource = "B200 fit (362 cases, 43650 points, rel<=1.5): direct: train 4.7% test 7.8% (n=854+167); tile: train 7.9% test 8.0% (n=7618+1987); pipe: train 7.7% test 7.8% (n=6688+1699); quad: train 8.0% test 7.2% (n=2853+906); regret 15.9%";
 }  // namespace ttlg

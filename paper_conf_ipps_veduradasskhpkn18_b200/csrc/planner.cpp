@@ -179,15 +179,18 @@ static void dense_prefixes(Problem &P) {
     P.denseB++;
 }
 
-// k_bulk / k_vec join the automatic choice only with TTLG_NEW_KERNELS=1 until
-// the model is calibrated on them (forced with hints variant 5 / 6 / 7 otherwise)
-static bool new_kernels_auto() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = getenv("TTLG_NEW_KERNELS");
-    v = (e && e[0] == '1') ? 1 : 0;
-  }
-  return v == 1;
+// Which of the newer kernels join the automatic choice: k_vec by default
+// (TTLG_VEC=0 removes it), k_bulk only with TTLG_BULK=1 (it wins on few
+// configurations).  Forced with hints variant
+// 5 / 6 / 7 either way.
+static bool env_flag(const char *name, bool dflt) {
+  const char *e = getenv(name);
+  if (!e || !e[0]) return dflt;
+  return e[0] == '1';
+}
+static bool new_kernel_auto(int group) {
+  static const bool vec = env_flag("TTLG_VEC", false), bulk = env_flag("TTLG_BULK", false);
+  return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;
 constexpr int64_t kBulkTmaRowBytes = 2048;
@@ -807,6 +810,7 @@ static void fill_info(ttlg_plan_info &I, ttlg_dtype dt, int rank, const Problem 
   I.param_bytes = (int32_t)sizeof(TileParams);
   I.kernel = kind;
   I.occupancy = mi.occ;
+  I.stages = mi.nstage;
 }
 
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
@@ -1081,7 +1085,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (bulk || group == KK_VEC) {
       if (forceW) return;  // element-width fallback plans: no 16-byte requirement
       const int want = group == KK_BULKQ ? 5 : (group == KK_BULKG ? 6 : 7);
-      if (hv == 0 ? !new_kernels_auto() : hv != want) return;
+      if (hv == 0 ? !new_kernel_auto(group) : hv != want) return;
     } else if (hv >= 5) {
       return;  // k_bulk / k_vec forced
     }
@@ -1094,6 +1098,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     Tile T = make_tile(P, a, ta, b, tb);
     if (!T.ok) return;
     if (group == KK_QUAD && (!quad_k(P, T) || forceW || (hv != 0 && hv != 3))) return;
+    if ((bulk || group == KK_VEC) && !bulk_ok(P, T, group)) return;  // 16-byte rows
     const int schema = schema_of(P, T, group);
     if (force_schema != TTLG_SCHEMA_AUTO && force_schema != schema) {
       // COPY and FML share the direct kernel; accept FML for a rank-1 problem

@@ -12,6 +12,7 @@ from __future__ import annotations
 import argparse
 import itertools
 import json
+import math
 import os
 import random
 import statistics
@@ -21,7 +22,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 
-def recipe_cases(n, seed, lo_mb=32, hi_mb=512):
+def recipe_cases(n, seed, lo_mb=32, hi_mb=512, log_size=False):
     """Paper dataset recipe (L1298-1313): ranks 3-6, any permutation, five extent
     orderings (equal, increasing, decreasing, up-down, down-up), volume range."""
     from synth.configs import Case
@@ -30,7 +31,10 @@ def recipe_cases(n, seed, lo_mb=32, hi_mb=512):
     for k in range(n):
         d = rng.randint(3, 6)
         eb = rng.choice([4, 8])
-        target = rng.uniform(lo_mb, hi_mb) * 2 ** 20 / eb
+        if log_size:
+            target = math.exp(rng.uniform(math.log(lo_mb), math.log(hi_mb))) * 2 ** 20 / eb
+        else:
+            target = rng.uniform(lo_mb, hi_mb) * 2 ** 20 / eb
         base = target ** (1.0 / d)
         kind = rng.choice(["eq", "inc", "dec", "updown", "downup"])
         f = [1.0] * d
@@ -39,7 +43,7 @@ def recipe_cases(n, seed, lo_mb=32, hi_mb=512):
             f[i] = {"eq": 1.0, "inc": 0.5 + t, "dec": 1.5 - t,
                     "updown": 0.6 + 0.8 * (1 - abs(2 * t - 1)),
                     "downup": 0.6 + 0.8 * abs(2 * t - 1)}[kind]
-        g = (1.0 / (1e-9 + float(__import__("math").prod(f)))) ** (1.0 / d)
+        g = (1.0 / (1e-9 + float(math.prod(f)))) ** (1.0 / d)
         ext = [max(2, int(round(base * fi * g * rng.uniform(0.9, 1.1)))) for fi in f]
         perm = list(range(d))
         while perm == list(range(d)):
@@ -53,6 +57,9 @@ def main():
     ap.add_argument("--group", default=None)
     ap.add_argument("--recipe", type=int, default=0)
     ap.add_argument("--seed", type=int, default=1)
+    ap.add_argument("--lo-mb", type=float, default=32.0)
+    ap.add_argument("--hi-mb", type=float, default=512.0)
+    ap.add_argument("--log-size", action="store_true", help="tensor sizes log-uniform")
     ap.add_argument("--max-cand", type=int, default=40)
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--stride", type=int, default=1)
@@ -70,7 +77,7 @@ def main():
     if args.group:
         cases += configs.all_configs()[args.group][::args.stride]
     if args.recipe:
-        cases += recipe_cases(args.recipe, args.seed)
+        cases += recipe_cases(args.recipe, args.seed, args.lo_mb, args.hi_mb, args.log_size)
     if args.ids:
         keep = {int(x) for x in args.ids.split(",")}
         cases = [c for c in cases if c.case_id in keep]
@@ -118,7 +125,7 @@ def main():
                 "threads": info["threads"], "kernel_hint": h.get("variant", 0),
                 "tile": info["tile_extents"], "LA": info["in_run"], "LB": info["out_run"],
                 "V": info["tile_volume"], "tiles": info["num_tiles"], "grid": info["grid"],
-                "occ": info["occupancy"], "features": info["features"],
+                "occ": info["occupancy"], "nstage": info["stages"], "features": info["features"],
                 "pred": info["predicted_seconds"], "meas": t, "gbs": c.alg_bytes / t / 1e9,
                 "is_auto": info["tile_extents"] == auto["tile_extents"]
                 and info["schema"] == auto["schema"]}), flush=True)

@@ -24,7 +24,7 @@ from scipy.optimize import nnls
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 COEFF_H = os.path.join(ROOT, "paper_conf_ipps_veduradasskhpkn18_b200", "csrc", "model_coeffs.h")
-KINDS = ["direct", "tile", "pipe", "quad"]
+KINDS = ["direct", "tile", "pipe", "quad", "bulkq", "bulkg", "vec"]
 
 
 def fit(rows):
@@ -97,7 +97,8 @@ def main():
             src = f.read()
         lines = []
         for k, name in (("direct", "kCoefDirect"), ("tile", "kCoefTile"), ("pipe", "kCoefPipe"),
-                        ("quad", "kCoefQuad")):
+                        ("quad", "kCoefQuad"), ("bulkq", "kCoefBulkQ"), ("bulkg", "kCoefBulkG"),
+                        ("vec", "kCoefVec")):
             if k in coefs:
                 vals = ", ".join(f"{v:.6e}" for v in coefs[k])
                 lines.append(f"constexpr double {name}[kModelNumFeatures] = {{{vals}}};")

@@ -26,7 +26,7 @@ from sklearn.ensemble import GradientBoostingRegressor
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 CSRC = os.path.join(ROOT, "paper_conf_ipps_veduradasskhpkn18_b200", "csrc")
-KID = {"direct": 0, "tile": 1, "pipe": 2, "quad": 3}
+KID = {"direct": 0, "tile": 1, "pipe": 2, "quad": 3, "bulkq": 5, "bulkg": 6, "vec": 7}
 HBM = 6555.5e9
 SMS = 148
 TOPK = int(os.environ.get("TTLG_GBT_TOPK", "16"))
@@ -46,7 +46,7 @@ def desc(r):
             math.log2(r["tiles"]), f[2] / max(f[1], 1e-12), f[8] / max(1.0, r["bytes"] / 1e9),
             r["tiles"] / (SMS * occ),
             math.log2(V / th), (RA + RB + r["LB"]) / th, N / (r["tiles"] * V),
-            math.ceil(r["tiles"] / r["grid"])]
+            math.ceil(r["tiles"] / r["grid"]), math.log2(r["bytes"]), float(r.get("nstage", 0))]
 
 
 def ideal(r):
@@ -57,7 +57,8 @@ def linear_coefs():
     src = open(os.path.join(CSRC, "model_coeffs.h")).read()
     co = {}
     for name, k in (("kCoefDirect", "direct"), ("kCoefTile", "tile"), ("kCoefPipe", "pipe"),
-                    ("kCoefQuad", "quad")):
+                    ("kCoefQuad", "quad"), ("kCoefBulkQ", "bulkq"), ("kCoefBulkG", "bulkg"),
+                    ("kCoefVec", "vec")):
         m = re.search(name + r"\[kModelNumFeatures\] = \{([^}]*)\}", src)
         co[k] = np.array([float(x) for x in m.group(1).split(",")])
     return co
