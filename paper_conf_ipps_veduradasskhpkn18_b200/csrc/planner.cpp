@@ -189,7 +189,7 @@ static bool env_flag(const char *name, bool dflt) {
   return e[0] == '1';
 }
 static bool new_kernel_auto(int group) {
-  static const bool vec = env_flag("TTLG_VEC", false), bulk = env_flag("TTLG_BULK", false);
+  static const bool vec = env_flag("TTLG_VEC", true), bulk = env_flag("TTLG_BULK", false);
   return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;

@@ -91,6 +91,20 @@ def main():
                                          learning_rate=args.lr, subsample=0.8,
                                          random_state=0).fit(X, y)
 
+    def per_schema(m, cs):
+        """Held-out mean |a-p|/a (L1414-1416) of every measured candidate, by
+        schema and by kernel; plus the error of each case's chosen plan."""
+        out = collections.defaultdict(list)
+        for c in cs:
+            rs = by[c]
+            P = m.predict(np.array([desc(r) for r in rs]))
+            for r, p in zip(rs, P):
+                e = abs(math.exp(p) * ideal(r) - r["meas"]) / r["meas"]
+                out["schema:" + r["schema"]].append(e)
+                out["kernel:" + r["kernel"]].append(e)
+                out["size:" + ("<16MB" if r["bytes"] < 16e6 else ">=16MB")].append(e)
+        return {k: (round(100 * float(np.mean(v)), 1), len(v)) for k, v in sorted(out.items())}
+
     def evaluate(m, cs):
         reg, err, gp, gb = [], [], [], []
         for c in cs:
@@ -114,6 +128,8 @@ def main():
     te = evaluate(m, list(test))
     print(f"train: regret {tr[0]:.1f}% err(top{TOPK}) {tr[1]:.1f}% picked {tr[2]:.0f} best {tr[3]:.0f}")
     print(f"test : regret {te[0]:.1f}% err(top{TOPK}) {te[1]:.1f}% picked {te[2]:.0f} best {te[3]:.0f}")
+    print("held-out error by schema / kernel / size (mean |a-p|/a %, n):")
+    print(json.dumps(per_schema(m, list(test))))
     if not args.write:
         return
     m = fit(rows)  # final model on all configurations
