@@ -85,7 +85,8 @@ typedef struct {
   int64_t out_block;                     /* blockB, 0 = auto                             */
   int32_t elem_bytes_override;           /* 0 = auto widening; else 4/8/16 access width
                                             (pins the width: no k_quad 16-byte chunks)   */
-  int32_t threads;                       /* 0 = auto; else threads per block             */
+  int32_t threads;                       /* 0 = auto; else threads per block (k_bulk:
+                                            consumer threads, 256 or 512)                 */
   int32_t grid;                          /* 0 = auto (persistent); else blocks           */
   int32_t no_fusion;                     /* 1 = skip index fusion (tests)                */
   int32_t variant;                       /* staged kernel: 0 = model choice, 1 = k_tile
@@ -96,7 +97,17 @@ typedef struct {
                                             2 <= n0 <= 8 and M a multiple of 16/s, or
                                             2 <= M <= 8 and n0 a multiple of 16/s:
                                             16-byte accesses both ways through a per-warp
-                                            staging buffer)                               */
+                                            staging buffer), 5 = k_bulk with quad
+                                            consumers (OD; TMA bulk row loads into an
+                                            mbarrier ring), 6 = k_bulk with gather
+                                            consumers (any schema), 7 = k_vec (16-byte
+                                            cp.async loads, 16-byte stores gathered from
+                                            16/s element reads); 5-7 need every A-row
+                                            (6, 7: and B-row) 16-byte aligned and whole
+                                            16-byte chunks, else TTLG_ERR_UNSUPPORTED.
+                                            The automatic choice considers 0-4 and 7
+                                            (env TTLG_VEC=0 drops 7; TTLG_BULK=1 adds
+                                            5, 6)                                          */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */

@@ -116,6 +116,7 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 
 // ---- ranking stage: boosted regression trees (model_gbt.h) --------------------
 #include "model_gbt.h"
+#include "model_gbt2.h"
 
 namespace ttlg {
 
@@ -155,9 +156,12 @@ double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 
 // The candidates' traversals of one tree are independent: interleaving them
 // (tree-major) lets the core overlap their dependent node loads.
-void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
+template <int NT, int D>
+static void gbt_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out,
+                      double init, const int8_t (&F_)[NT][(1 << D) - 1],
+                      const float (&T_)[NT][(1 << D) - 1], const float (&V_)[NT][1 << D]) {
   constexpr int kB = 32;
-  constexpr int NI = (1 << kGbtDepth) - 1;
+  constexpr int NI = (1 << D) - 1;
   float d[kB][kGbtDesc];
   double s[kB];
   for (int b0 = 0; b0 < n; b0 += kB) {
@@ -166,20 +170,20 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
       double dd[kGbtDesc];
       model_descriptor(mis[b0 + c], dev, dd);
       for (int k = 0; k < kGbtDesc; k++) d[c][k] = (float)dd[k];  // sklearn splits on float32
-      s[c] = kGbtInit;
+      s[c] = init;
     }
-    for (int t = 0; t < kGbtTrees; t++) {
-      const int8_t *F = kGbtF[t];
-      const float *T = kGbtT[t];
+    for (int t = 0; t < NT; t++) {
+      const int8_t *F = F_[t];
+      const float *T = T_[t];
       // level-major: the m walks of one level are independent load chains
       int idx[kB];
       for (int c = 0; c < m; c++) idx[c] = 0;
-      for (int l = 0; l < kGbtDepth; l++)
+      for (int l = 0; l < D; l++)
         for (int c = 0; c < m; c++) {
           const int i = idx[c];
           idx[c] = 2 * i + 1 + (d[c][F[i]] > T[i]);
         }
-      for (int c = 0; c < m; c++) s[c] += kGbtV[t][idx[c] - NI];
+      for (int c = 0; c < m; c++) s[c] += V_[t][idx[c] - NI];
     }
     for (int c = 0; c < m; c++) {
       const ModelInput &mi = mis[b0 + c];
@@ -187,6 +191,14 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
       out[b0 + c] = std::exp(std::max(s[c], 0.0)) * ideal;  // never below one pass at copy speed
     }
   }
+}
+
+void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
+  gbt_batch<kGbtTrees, kGbtDepth>(mis, n, dev, out, kGbtInit, kGbtF, kGbtT, kGbtV);
+}
+
+void predict_ranked2_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
+  gbt_batch<kGbt2Trees, kGbt2Depth>(mis, n, dev, out, kGbt2Init, kGbt2F, kGbt2T, kGbt2V);
 }
 
 }  // namespace ttlg

@@ -40,6 +40,11 @@ constexpr int kGbtDesc = 18;  // descriptor length (tools/calibrate_gbt.py desc(
 void model_descriptor(const ModelInput &mi, const DeviceProfile &dev, double *d);
 double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev);
 void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
+// second tree set (model_gbt2.h: refit with k_vec / k_bulk and small tensors in the
+// data): decides whether a k_vec candidate beats the first set's winner
+void predict_ranked2_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
+// k_vec replaces the winner only when predicted this much faster by the second set
+constexpr double kVecMargin = 0.95;
 
 // k_deint (one streaming pass, 16-byte accesses both ways): time = this
 // factor x the one-pass ideal 2*N*s / HBM bandwidth -- measured on B200 at

@@ -906,6 +906,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   const bool listing = sink && !sink->shortlist;
   Entry pool[kShort];
   int order[kShort];  // pool slots sorted by the linear prediction
+  // k_vec candidates of the automatic choice rank in their own short list and
+  // must beat the main winner under the second tree set (model_gbt2.h)
+  constexpr int kVecShort = 4;
+  Entry vpool[kVecShort];
+  int nv = 0;  // vpool sorted by the linear prediction
   int ntop = 0, ncand = 0;
   double admit = 1e300;  // admission threshold: the worst short-list entry once full
 
@@ -1179,6 +1184,30 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           ci.num_features = kModelFeatureCount;
           for (int f = 0; f < kModelFeatureCount; f++) ci.features[f] = F.f[f];
         }
+        if (kind == KK_VEC && hv == 0) {
+          bool dup = false;
+          for (int i = 0; i < nv && !dup; i++) {
+            bool same = vpool[i].mi.threads == mi.threads;
+            for (int k = 0; k < P.d && same; k++) same = vpool[i].T.t[k] == T.t[k];
+            dup = same;
+          }
+          if (dup || (nv == kVecShort && tm >= vpool[nv - 1].lin)) continue;
+          int pos = nv < kVecShort ? nv++ : nv - 1;
+          while (pos > 0 && vpool[pos - 1].lin > tm) {
+            vpool[pos] = vpool[pos - 1];
+            pos--;
+          }
+          Entry &e = vpool[pos];
+          e.lin = tm;
+          e.mi = mi;
+          e.T = T;
+          e.kind = kind;
+          e.schema = schema;
+          e.tpc = tpc;
+          e.group = group;
+          for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = 0;
+          continue;
+        }
         if (tm < admit) insert(tm, mi, T, kind, schema, tpc, group, delta);
       }
     }
@@ -1359,6 +1388,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     make_deint(plan, &plan->info, deint_t);
     return TTLG_OK;
   }
+  if (ntop == 0 && nv > 0) {  // only k_vec slices (cannot happen with the staged kernels present)
+    for (int i = 0; i < nv; i++) {
+      pool[i] = vpool[i];
+      order[i] = i;
+    }
+    ntop = nv;
+    nv = 0;
+  }
   if (ntop == 0) {
     const bool forced = hints && (hints->schema != TTLG_SCHEMA_AUTO || hints->in_dim >= 0 ||
                                   hints->in_block > 0 || hints->out_dim >= 0 ||
@@ -1434,6 +1471,39 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       win = rid[i];
     }
   }
+  // k_vec challenge: refine its short list, then compare with the winner under
+  // the second tree set; it replaces the winner only when predicted faster by
+  // kVecMargin (round-1 choices stay unless k_vec clearly wins)
+  const Entry *Bp = &pool[win];
+  if (nv > 0 && !listing && pool[win].lin < 1e299) {
+    ModelInput cm[1 + kVecShort];
+    int cid[1 + kVecShort], m = 0;
+    cm[m] = pool[win].mi;
+    cid[m++] = -1;
+    for (int i = 0; i < nv; i++) {
+      Entry &e = vpool[i];
+      TileSummary S2;
+      TileParams K0;
+      int dl[TTLG_MAXD];
+      double cl, cs;
+      int tpc;
+      if (!summarize(P, e.T, e.group, S2) || !build_exact(e.T, e.group, K0, dl, cl, cs, S2) ||
+          !make_mi(e.mi, tpc, e.kind, e.schema, e.mi.threads, S2, cl, cs))
+        continue;
+      e.tpc = tpc;
+      cm[m] = e.mi;
+      cid[m++] = i;
+    }
+    double t2[1 + kVecShort];
+    predict_ranked2_batch(cm, m, dev, t2);
+    int bj = -1;
+    for (int j = 1; j < m; j++)
+      if (t2[j] < kVecMargin * t2[0] && (bj < 0 || t2[j] < t2[bj])) bj = j;
+    if (bj > 0) {
+      Bp = &vpool[cid[bj]];
+      win_t = win_t * t2[bj] / t2[0];  // in the first set's scale (deint comparison below)
+    }
+  }
   if (sink && sink->shortlist) {
     // the ranked short list (tree prediction in predicted_seconds)
     for (int i = 0; i < std::min(ntop, kGbtTopK) && sink->n < sink->max; i++) {
@@ -1463,7 +1533,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     make_deint(plan, &plan->info, deint_t);
     return TTLG_OK;
   }
-  const Entry &B = pool[win];
+  const Entry &B = *Bp;
   if (B.lin >= 1e299) return TTLG_ERR_INTERNAL;
   // rebuild the winner's parameter block
   TileParams K;

@@ -71,6 +71,8 @@ def main():
     ap.add_argument("--trees", type=int, default=100)
     ap.add_argument("--depth", type=int, default=5)
     ap.add_argument("--lr", type=float, default=0.2)
+    ap.add_argument("--sym", default="kGbt", help="C symbol prefix of the tree set")
+    ap.add_argument("--out", default="model_gbt.h", help="header name under csrc/")
     args = ap.parse_args()
     rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
     # k_deint is not ranked by the trees (its time is a measured factor, model.h)
@@ -170,28 +172,29 @@ def main():
     def flt(x):
         return "INFINITY" if x == float("inf") else f"{x!r}f"
 
-    with open(os.path.join(CSRC, "model_gbt.h"), "w") as f:
-        f.write("// model_gbt.h -- GENERATED by tools/calibrate_gbt.py: boosted regression trees\n"
+    P = args.sym
+    with open(os.path.join(CSRC, args.out), "w") as f:
+        f.write(f"// {args.out} -- GENERATED by tools/calibrate_gbt.py: boosted regression trees\n"
                 "// predicting log(time / one-pass ideal) from model_descriptor() (model.cpp).\n"
                 f"// Fitted on {len(rows)} B200 measurements ({len(cases)} configurations); held-out\n"
                 f"// 20%: selection regret {te[0]:.1f}%, mean |a-p|/a {te[1]:.1f}% (top-{TOPK} lists).\n"
                 f"// Complete trees of depth {D}: node i has children 2i+1 (x <= t) and 2i+2.\n"
                 "#pragma once\n#include <math.h>\n#include <stdint.h>\nnamespace ttlg {\n")
-        f.write(f"constexpr int kGbtTrees = {len(F)};\nconstexpr int kGbtDepth = {D};\n"
-                f"constexpr int kGbtTopK = {TOPK};\n")
-        f.write(f"constexpr double kGbtInit = {init!r};\n")
-        f.write(f'constexpr const char *kGbtSource = "GBT {len(F)} trees depth {D}, '
+        f.write(f"constexpr int {P}Trees = {len(F)};\nconstexpr int {P}Depth = {D};\n"
+                + (f"constexpr int {P}TopK = {TOPK};\n" if P == "kGbt" else ""))
+        f.write(f"constexpr double {P}Init = {init!r};\n")
+        f.write(f'constexpr const char *{P}Source = "GBT {len(F)} trees depth {D}, '
                 f'{len(rows)} points / {len(cases)} cases; test regret {te[0]:.1f}%, '
                 f'err {te[1]:.1f}%";\n')
-        f.write(f"constexpr int8_t kGbtF[{len(F)}][{NI}] = {{\n" +
+        f.write(f"constexpr int8_t {P}F[{len(F)}][{NI}] = {{\n" +
                 ",\n".join("{" + ",".join(map(str, r)) + "}" for r in F) + "};\n")
-        f.write(f"constexpr float kGbtT[{len(F)}][{NI}] = {{\n" +
+        f.write(f"constexpr float {P}T[{len(F)}][{NI}] = {{\n" +
                 ",\n".join("{" + ",".join(flt(x) for x in r) + "}" for r in T) + "};\n")
-        f.write(f"constexpr float kGbtV[{len(F)}][{NL}] = {{\n" +
+        f.write(f"constexpr float {P}V[{len(F)}][{NL}] = {{\n" +
                 ",\n".join("{" + ",".join(flt(x) for x in r) + "}" for r in V) + "};\n")
         f.write("}  // namespace ttlg\n")
     feats = F
-    print("wrote", os.path.join(CSRC, "model_gbt.h"), len(feats), "trees")
+    print("wrote", os.path.join(CSRC, args.out), len(feats), "trees")
 
 
 if __name__ == "__main__":

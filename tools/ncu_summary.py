@@ -31,13 +31,23 @@ def main():
             for k in KEYS:
                 if k in d:
                     print(f"  {k:70s} {d[k]} {units[hdr.index(k)]}")
-            stalls = [(float(d[k] or 0), k) for k in hdr
-                      if k.startswith("smsp__average_warp_latency_issue_stalled")
-                      and k.endswith(".ratio") or
-                      (k.startswith("smsp__warp_issue_stalled") and k.endswith("per_warp_active.pct"))]
+            for k in ("smsp__issue_active.avg.pct_of_peak_sustained_active",
+                      "dram__throughput.avg.pct_of_peak_sustained_elapsed"):
+                if k in d:
+                    print(f"  {k:70s} {d[k]} {units[hdr.index(k)]}")
+            # warps stalled per issued instruction, by reason (the top 8)
+            stalls = []
+            for k in hdr:
+                if (k.startswith("smsp__average_warps_issue_stalled_")
+                        and k.endswith("_per_issue_active.ratio")):
+                    try:
+                        stalls.append((float(d[k]), k[len("smsp__average_warps_issue_stalled_"):
+                                                      -len("_per_issue_active.ratio")]))
+                    except ValueError:
+                        pass
             stalls.sort(reverse=True)
             for v, k in stalls[:8]:
-                print(f"  stall {k:64s} {v:.2f}")
+                print(f"  stall {k:40s} {v:.2f} warps per issue")
 
 
 if __name__ == "__main__":
