@@ -212,7 +212,22 @@ def test_plan_candidates_every_config_case():
             cands = ttlg.plan_candidates(dt, c.extents, c.perm)
             assert cands, c.label()
             kinds = {d["kernel"] for d in cands}
-            assert kinds <= {"direct", "tile", "pipe", "quad", "deint"}
+            # k_bulk only when forced or TTLG_BULK=1
+            assert kinds <= {"direct", "tile", "pipe", "quad", "deint", "vec"}
+            for d in cands:
+                if d["kernel"] == "vec":   # every listed k_vec slice plans as itself
+                    assert d["access_bytes"] in (4, 8)
+    # forced k_bulk / k_vec listings hold only their kernel and every entry re-plans
+    for c in groups["c2"][::6]:
+        for v, name in ((5, "bulkq"), (6, "bulkg"), (7, "vec")):
+            try:
+                cands = ttlg.plan_candidates("f64", c.extents, c.perm, variant=v)
+            except ttlg.TtlgError:
+                continue
+            assert {d["kernel"] for d in cands} <= {name}
+            for d in cands[:5]:
+                info = ttlg.plan("f64", c.extents, c.perm, **d["hints"]).describe()
+                assert info["kernel"] == name and info["tile_extents"] == d["tile_extents"]
 
 
 def test_bench_reference_arm_contract():
@@ -251,3 +266,47 @@ def test_deep_tiles_only_for_closed_leading_blocks():
         for k in range(c["in_dim"]):
             pre *= fe[k]
         assert pre * 8 < 4096 or c["in_dim"] == 0, c
+
+
+def test_vec_and_bulk_applicability():
+    """k_vec / k_bulk move whole 16-byte chunks: every A-row (and B-row) of every
+    tile must start 16-byte aligned; odd fp64
+    extents never qualify, 12-byte pencils do with 4-pencil blocks."""
+    p = ttlg.plan("f32", [3, 4096, 4096], [0, 2, 1], variant=7).describe()
+    assert p["kernel"] == "vec"
+    t = p["tile_extents"]
+    assert (t[0] * t[1] * 4) % 16 == 0 and (t[0] * t[2] * 4) % 16 == 0
+    for v in (5, 6, 7):
+        with pytest.raises(ttlg.TtlgError) as e:
+            ttlg.plan("f64", [17, 17, 17], [2, 1, 0], variant=v)
+        assert e.value.code == 7
+    # quad consumers need an Orthogonal-Distinct tile
+    with pytest.raises(ttlg.TtlgError):
+        ttlg.plan("f32", [4, 64, 64], [0, 2, 1], variant=5, schema="FMS")
+    b = ttlg.plan("f64", [64, 96], [1, 0], variant=5).describe()
+    assert b["kernel"] == "bulkq" and b["stages"] >= 2 and b["threads"] in (288, 544)
+
+
+def test_generalised_quad_chunks():
+    """k_quad needs chunk-aligned rows, not FVI multiples of K: [3, 4096, 4096]
+    fp32 `2 1 0` runs in 16-byte chunks with t1 a multiple of 4."""
+    d = ttlg.plan("f32", [3, 4096, 4096], [2, 1, 0], variant=3).describe()
+    assert d["kernel"] == "quad"
+    assert (d["tile_extents"][0] * d["tile_extents"][1]) % 4 == 0
+    with pytest.raises(ttlg.TtlgError):
+        ttlg.plan("f32", [3, 4096, 4096], [2, 1, 0], variant=3, in_dim=1, in_block=21)
+
+
+def test_execute_batch_validation_without_gpu():
+    p = ttlg.plan("f64", [64, 64], [1, 0])
+    with pytest.raises(ttlg.TtlgError) as e:   # pair 1's B is pair 0's A
+        p.execute_batch([1 << 20, 1 << 28], [1 << 30, 1 << 20])
+    assert e.value.code == 2
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute_batch([1 << 20, (1 << 28) + 4], [1 << 30, 1 << 32])
+    assert e.value.code == 1                    # not element aligned
+    with pytest.raises(ttlg.TtlgError) as e:
+        p.execute_batch([1 << 20] * 3, [1 << 30, 1 << 31, 1 << 32])
+    assert e.value.code == 3                    # valid arguments, no device here
+    with pytest.raises(ValueError):
+        p.execute_batch([1 << 20], [])
