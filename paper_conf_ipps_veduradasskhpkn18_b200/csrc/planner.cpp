@@ -425,7 +425,12 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   if (kind == KK_QUAD && qk == 0) return false;
   const bool bulk = kind == KK_BULKQ || kind == KK_BULKG;
   if (bulk && (isdelta || !bulk_ok(P, T, kind))) return false;
-  if (kind == KK_VEC && (isdelta || !bulk_ok(P, T, KK_VEC))) return false;
+  if (kind == KK_VEC && !bulk_ok(P, T, KK_VEC)) return false;
+  // k_vec: isdelta[0] is not an input-run pad but extra chunk units on the
+  // first output-only dim's shared-memory stride (the gather-conflict search,
+  // vec_conflicts); its input run stays contiguous (16-byte cp.async chunks)
+  const int opad = (kind == KK_VEC && isdelta) ? isdelta[0] : 0;
+  if (kind == KK_VEC) isdelta = nullptr;
   const Strides S = strides_of(P);
   const int d = P.d, a = T.a, b = T.b, pb = P.p[T.b];
   bool inIS[TTLG_MAXD] = {false}, inOS[TTLG_MAXD] = {false};
@@ -498,10 +503,13 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   int64_t Q = 1, mult = 0;
   bool od = true;
   for (int i = 0; i <= b; i++) od &= !inIS[P.p[i]];
+  bool first_out = true;
   for (int i = 0; i <= b; i++) {
     const int k = P.p[i];
     if (!inIS[k] && T.t[k] > 1) {
-      const int64_t s = pad_stride(cur, Q, P.W, qk, od, mult);
+      int64_t s = pad_stride(cur, Q, P.W, qk, od, mult);
+      if (first_out) s += (int64_t)opad * qk;
+      first_out = false;
       sm[k] = s;
       cur = s * T.t[k];
     }
@@ -738,6 +746,39 @@ static void smem_conflicts(const TileParams &K, int W, double &load, double &sto
   }
 }
 
+// k_vec's gather: lane l of the first warp owns output chunk q = l mod LBc of
+// B-row l / LBc and reads positions K q + u (u < K): the worst wavefront ratio
+// over the K reads (1 = conflict-free)
+static double vec_conflicts(const TileParams &K, int W) {
+  const int Kc = 16 / W, LBc = K.LB / Kc;
+  auto offsets = [](int cnt, int n, const int32_t *ext, const int32_t *sS, int64_t *out) {
+    int dig[TTLG_MAXD] = {0};
+    int64_t s = 0;
+    for (int i = 0; i < cnt; i++) {
+      out[i] = s;
+      for (int k = 0; k < n; k++) {
+        s += sS[k];
+        if (++dig[k] < ext[k]) break;
+        s -= (int64_t)dig[k] * sS[k];
+        dig[k] = 0;
+      }
+    }
+  };
+  const int nr = std::min(31 / LBc + 1, K.RB), nc = std::min(K.LB, 32 * Kc);
+  int64_t rows[33], cols[32 * 4], addr[32];
+  offsets(nr, K.nrb, K.rb_ext, K.rb_sS, rows);
+  offsets(nc, K.nj, K.j_ext, K.j_sS, cols);
+  double worst = 1.0;
+  for (int u = 0; u < Kc; u++) {
+    for (int l = 0; l < 32; l++) {
+      const int r = std::min(l / LBc, nr - 1), j = std::min((l % LBc) * Kc + u, nc - 1);
+      addr[l] = rows[r] + cols[j];
+    }
+    worst = std::max(worst, wavefront_ratio(addr, W));
+  }
+  return worst;
+}
+
 static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) {
   int occ = dev.max_threads_per_sm / threads;
   const int per = smem + 1024;  // 1 KB reserved per CTA
@@ -908,7 +949,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   int order[kShort];  // pool slots sorted by the linear prediction
   // k_vec candidates of the automatic choice rank in their own short list and
   // must beat the main winner under the second tree set (model_gbt2.h)
-  constexpr int kVecShort = 4;
+  constexpr int kVecShort = 8;
   Entry vpool[kVecShort];
   int nv = 0;  // vpool sorted by the linear prediction
   int ntop = 0, ncand = 0;
@@ -994,7 +1035,32 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     }
     if (!build_params(P, T, group, thr_list[0], 1, K0)) return false;
     if (group == KK_DIRECT) return true;
-    if (group == KK_QUAD || group == KK_VEC) {  // chunk layout: no input-run padding
+    if (group == KK_VEC) {
+      // the gather's bank conflicts depend on the output-only stride: try a
+      // few extra chunk units on it and keep the least conflicted layout
+      double best = vec_conflicts(K0, P.W);
+      int bp = 0;
+      for (int m = 1; m < 8 && best > 1.0; m++) {
+        int d2[TTLG_MAXD] = {0};
+        d2[0] = m;
+        TileParams Kt;
+        if (!build_params(P, T, group, thr_list[0], 1, Kt, d2)) continue;
+        const double c2 = vec_conflicts(Kt, P.W);
+        if (c2 < best - 1e-9) {
+          best = c2;
+          bp = m;
+        }
+      }
+      if (bp) {
+        delta[0] = bp;
+        if (!build_params(P, T, group, thr_list[0], 1, K0, delta)) return false;
+      }
+      cs = best;
+      S.smem_base = K0.smem_bytes;
+      S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
+      return true;
+    }
+    if (group == KK_QUAD) {  // chunk layout: no input-run padding
       S.smem_base = K0.smem_bytes;
       S.buf_bytes = (int)(((int64_t)K0.smem_elems * P.W + 15) / 16 * 16);
       return true;
@@ -1277,6 +1343,22 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                 }
               }
             }
+          }
+        }
+        // small closed block: dims 0..a-1 (< 4 KB) map onto output positions
+        // 0..a-1 (e.g. the 16 x 16 block of 16^6 `1 0 2 3 5 4`): with the
+        // output run = that block, dim a blocked by tile volume (8-64 KB)
+        // gives tiles of t consecutive blocks, every B-row one block --
+        // contiguous in both tensors (deep k_pipe tiles, as below)
+        if (b == a - 1 && !hints) {
+          bool closed_small = true;
+          for (int i = 0; closed_small && i < a; i++) closed_small = P.p[i] < a;
+          if (closed_small) {
+            int64_t blocksD[32];
+            const int nbD = cand_blocks(P.n[a], preA, P.W, blocksD, 0, kDeepTargets);
+            pipe_only = true;
+            for (int i = 0; i < nbD; i++) consider(KK_TILE, a, blocksD[i], b, P.n[pb]);
+            pipe_only = false;
           }
         }
         preB *= P.n[pb];
