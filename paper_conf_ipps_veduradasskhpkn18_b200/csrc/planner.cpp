@@ -949,7 +949,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   int order[kShort];  // pool slots sorted by the linear prediction
   // k_vec candidates of the automatic choice rank in their own short list and
   // must beat the main winner under the second tree set (model_gbt2.h)
-  constexpr int kVecShort = 8;
+  constexpr int kVecShort = 16;
   Entry vpool[kVecShort];
   int nv = 0;  // vpool sorted by the linear prediction
   int ntop = 0, ncand = 0;
