@@ -45,6 +45,9 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
 void predict_ranked2_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
 // k_vec replaces the winner only when predicted this much faster by the second set
 constexpr double kVecMargin = 0.95;
+// ... and is considered only when the first set predicts its winner below this
+// fraction of the copy speed
+constexpr double kVecChallenge = 0.8;
 
 // k_deint (one streaming pass, 16-byte accesses both ways): time = this
 // factor x the one-pass ideal 2*N*s / HBM bandwidth -- measured on B200 at

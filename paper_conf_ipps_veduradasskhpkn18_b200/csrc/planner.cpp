@@ -1157,6 +1157,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (forceW) return;  // element-width fallback plans: no 16-byte requirement
       const int want = group == KK_BULKQ ? 5 : (group == KK_BULKG ? 6 : 7);
       if (hv == 0 ? !new_kernel_auto(group) : hv != want) return;
+      // in the automatic choice k_vec only challenges matching-FVI winners (below)
+      if (hv == 0 && group == KK_VEC && P.p[0] != 0 && !listing) return;
     } else if (hv >= 5) {
       return;  // k_bulk / k_vec forced
     }
@@ -1557,7 +1559,15 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // the second tree set; it replaces the winner only when predicted faster by
   // kVecMargin (round-1 choices stay unless k_vec clearly wins)
   const Entry *Bp = &pool[win];
-  if (nv > 0 && !listing && pool[win].lin < 1e299) {
+  // the challenge (refining up to kVecShort k_vec slices with their padding
+  // search, ~100 us of host time) runs for matching-FVI problems whose
+  // winner is predicted below kVecChallenge of the copy speed: k_vec's wins
+  // that the second tree set resolves are the FMS pencils of 12/20/28 bytes
+  // (bulk_sweep, exp r2e8/r2e13); single-use plans elsewhere stay cheap
+  const double ideal_t = 2.0 * (double)N * P.W / (dev.hbm_gbs * 1e9);
+  if (nv > 0 && !listing && P.p[0] == 0 && pool[win].lin < 1e299 &&
+      win_t > ideal_t / kVecChallenge) {
+    if (fast) nv = std::min(nv, 4);
     ModelInput cm[1 + kVecShort];
     int cid[1 + kVecShort], m = 0;
     cm[m] = pool[win].mi;
