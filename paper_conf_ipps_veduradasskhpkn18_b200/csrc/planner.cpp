@@ -793,6 +793,9 @@ static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) 
 // slowest dim of the group; reading R12 enumerates block factors
 // directly, including the balanced ceil(n/ceil(n/t)) variants).
 static const int64_t kRunTargets[] = {64, 128, 256, 512, 1024, 2048, 4096, 0};
+// single-use plans (fast effort): a coarser run-length grid keeps the screen
+// to ~1/3 of the candidates, so planning hides behind short kernels
+static const int64_t kRunTargetsFast[] = {128, 512, 2048, 0};
 static const int64_t kTileTargets[] = {4096, 8192, 16384, 32768, 65536, 131072, 0};
 static const int64_t kDeepTargets[] = {8192, 16384, 32768, 65536, 0};
 
@@ -1070,7 +1073,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // in the input run, i.e. overlapping groups (OA/FMS); OD tiles skip the search
     bool overlap = false;
     for (int i = 0; i <= T.b; i++) overlap |= P.p[i] <= T.a;
-    if (overlap && cl + cs > 2.0) {
+    if (overlap && cl + cs > 2.0 && !fast) {  // single use: no padding search
       const int lp = 128 / P.W;
       const int opts[6] = {1, 2, 3, lp / 2, lp / 2 + 1, lp - 1};
       for (int k = 1; k <= T.a && cl + cs > 2.0; k++) {
@@ -1219,7 +1222,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // output run LB nearest below 512 when 512 would leave >= 1/16 of the
     // threads idle in the store walk (each thread owns one output position)
     int tl[3] = {thr_list[0], thr_list[1], 0}, ntl = nthr;
-    if (group != KK_DIRECT && !(hints && hints->threads)) {
+    if (group != KK_DIRECT && !(hints && hints->threads) && !fast) {
       const int64_t LBc = S.LB;
       if (LBc < 512 && (512 % LBc) * 16 >= 512) {
         const int64_t m = (512 / LBc) * LBc;
@@ -1303,12 +1306,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int a_stop = -1;
     for (int a = 0; a <= P.denseA; a++) {
       const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0,
-                                  kRunTargets);
+                                  fast ? kRunTargetsFast : kRunTargets);
       int64_t preB = 1;
       for (int b = 0; b <= P.denseB; b++) {
         const int pb = P.p[b];
         const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0,
-                                    kRunTargets);
+                                    fast ? kRunTargetsFast : kRunTargets);
         if (pb == a) {
           // the same dim closes both groups (overlap): one shared blocking
           // factor, drawn from both candidate lists
@@ -1333,7 +1336,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
               // k_quad needs whole chunks per run: the same slice with the
               // blocking factors rounded up to a chunk multiple (e.g. t1 = 22
               // -> 24 for [3, 4096, 4096] fp32 `2 1 0`)
-              if (P.W == P.esize && !(hints && (hints->in_block > 0 || hints->out_block > 0))) {
+              if (P.W == P.esize && !fast &&
+                  !(hints && (hints->in_block > 0 || hints->out_block > 0))) {
                 const int Kq = 16 / P.W;
                 const int64_t ra = round_block(blocksA[i], preA, P.n[a], Kq);
                 const int64_t rb = round_block(blocksB[j], preB, P.n[pb], Kq);
@@ -1355,6 +1359,11 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         if (b == a - 1 && !hints) {
           bool closed_small = true;
           for (int i = 0; closed_small && i < a; i++) closed_small = P.p[i] < a;
+          // ... unless dims 0..a close a larger block that the >= 4 KB deep
+          // tiles below cover (16^6 `1 0 2 4 3 5`: [16,16,16] blocks win)
+          bool closed_next = a + 1 < P.d && preA * P.n[a] * P.W <= 65536;
+          for (int i = 0; closed_next && i <= a; i++) closed_next = P.p[i] <= a;
+          closed_small &= !closed_next;
           if (closed_small) {
             int64_t blocksD[32];
             const int nbD = cand_blocks(P.n[a], preA, P.W, blocksD, 0, kDeepTargets);
@@ -1658,7 +1667,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // second tree set, whose data includes 0.25-32 MB tensors (launch-bound,
   // L2-resident): the first set only ranks
   double t_report = win_t;
-  if (!listing) predict_ranked2_batch(&B.mi, 1, dev, &t_report);
+  if (!listing && !fast) predict_ranked2_batch(&B.mi, 1, dev, &t_report);  // single use: skip
   fill_info(plan->info, dt, rank, P, B.T, K, B.mi, B.schema, B.kind, t_report, ncand);
   {
     const ModelFeatures F = model_features(B.mi, dev);
