@@ -1564,24 +1564,31 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       win = rid[i];
     }
   }
-  // k_vec challenge: refine its short list, then compare with the winner under
-  // the second tree set; it replaces the winner only when predicted faster by
-  // kVecMargin (round-1 choices stay unless k_vec clearly wins)
+  // Second opinion for weak winners: when the first tree set predicts its
+  // winner below kVecChallenge of the copy speed, the second set (model_gbt2.h,
+  // refit with k_vec and the cal33 top candidates of configs 2-4 in its data)
+  // re-ranks the first set's short list together with the k_vec slices
+  // (matching-FVI problems: their own short list, refined here with the
+  // gather-conflict padding); its pick replaces the winner only when predicted
+  // kVecMargin faster.  Round-1 choices elsewhere are unchanged, and
+  // single-use plans (fast effort) consult only the k_vec slices.
   const Entry *Bp = &pool[win];
-  // the challenge (refining up to kVecShort k_vec slices with their padding
-  // search, ~100 us of host time) runs for matching-FVI problems whose
-  // winner is predicted below kVecChallenge of the copy speed: k_vec's wins
-  // that the second tree set resolves are the FMS pencils of 12/20/28 bytes
-  // (bulk_sweep, exp r2e8/r2e13); single-use plans elsewhere stay cheap
   const double ideal_t = 2.0 * (double)N * P.W / (dev.hbm_gbs * 1e9);
-  if (nv > 0 && !listing && P.p[0] == 0 && pool[win].lin < 1e299 &&
-      win_t > ideal_t / kVecChallenge) {
+  if (!listing && pool[win].lin < 1e299 && win_t > ideal_t / kVecChallenge &&
+      (nv > 0 || !fast)) {
+    const bool use_vec = nv > 0 && P.p[0] == 0;
     if (fast) nv = std::min(nv, 4);
-    ModelInput cm[1 + kVecShort];
-    int cid[1 + kVecShort], m = 0;
+    ModelInput cm[kGbtTopK + kVecShort];
+    const Entry *ce[kGbtTopK + kVecShort];
+    int m = 0;
     cm[m] = pool[win].mi;
-    cid[m++] = -1;
-    for (int i = 0; i < nv; i++) {
+    ce[m++] = &pool[win];
+    for (int i = 0; i < nrk && !fast; i++) {
+      if (rid[i] == win) continue;
+      cm[m] = rk[i];
+      ce[m++] = &pool[rid[i]];
+    }
+    for (int i = 0; use_vec && i < nv; i++) {
       Entry &e = vpool[i];
       TileSummary S2;
       TileParams K0;
@@ -1592,16 +1599,17 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           !make_mi(e.mi, tpc, e.kind, e.schema, e.mi.threads, S2, cl, cs))
         continue;
       e.tpc = tpc;
+      for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)dl[k];
       cm[m] = e.mi;
-      cid[m++] = i;
+      ce[m++] = &e;
     }
-    double t2[1 + kVecShort];
+    double t2[kGbtTopK + kVecShort];
     predict_ranked2_batch(cm, m, dev, t2);
-    int bj = -1;
+    int bj = 0;
     for (int j = 1; j < m; j++)
-      if (t2[j] < kVecMargin * t2[0] && (bj < 0 || t2[j] < t2[bj])) bj = j;
+      if (t2[j] < kVecMargin * t2[0] && t2[j] < t2[bj]) bj = j;
     if (bj > 0) {
-      Bp = &vpool[cid[bj]];
+      Bp = ce[bj];
       win_t = win_t * t2[bj] / t2[0];  // in the first set's scale (deint comparison below)
     }
   }
