@@ -793,9 +793,6 @@ static int occupancy(const DeviceProfile &dev, int threads, int smem, int regs) 
 // slowest dim of the group; reading R12 enumerates block factors
 // directly, including the balanced ceil(n/ceil(n/t)) variants).
 static const int64_t kRunTargets[] = {64, 128, 256, 512, 1024, 2048, 4096, 0};
-// single-use plans (fast effort): a coarser run-length grid keeps the screen
-// to ~1/3 of the candidates, so planning hides behind short kernels
-static const int64_t kRunTargetsFast[] = {128, 512, 2048, 0};
 static const int64_t kTileTargets[] = {4096, 8192, 16384, 32768, 65536, 131072, 0};
 static const int64_t kDeepTargets[] = {8192, 16384, 32768, 65536, 0};
 
@@ -1222,7 +1219,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // output run LB nearest below 512 when 512 would leave >= 1/16 of the
     // threads idle in the store walk (each thread owns one output position)
     int tl[3] = {thr_list[0], thr_list[1], 0}, ntl = nthr;
-    if (group != KK_DIRECT && !(hints && hints->threads) && !fast) {
+    if (group != KK_DIRECT && !(hints && hints->threads)) {
       const int64_t LBc = S.LB;
       if (LBc < 512 && (512 % LBc) * 16 >= 512) {
         const int64_t m = (512 / LBc) * LBc;
@@ -1306,12 +1303,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int a_stop = -1;
     for (int a = 0; a <= P.denseA; a++) {
       const int nbA = cand_blocks(P.n[a], preA, P.W, blocksA, hints ? hints->in_block : 0,
-                                  fast ? kRunTargetsFast : kRunTargets);
+                                  kRunTargets);
       int64_t preB = 1;
       for (int b = 0; b <= P.denseB; b++) {
         const int pb = P.p[b];
         const int nbB = cand_blocks(P.n[pb], preB, P.W, blocksB, hints ? hints->out_block : 0,
-                                    fast ? kRunTargetsFast : kRunTargets);
+                                    kRunTargets);
         if (pb == a) {
           // the same dim closes both groups (overlap): one shared blocking
           // factor, drawn from both candidate lists
@@ -1336,8 +1333,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
               // k_quad needs whole chunks per run: the same slice with the
               // blocking factors rounded up to a chunk multiple (e.g. t1 = 22
               // -> 24 for [3, 4096, 4096] fp32 `2 1 0`)
-              if (P.W == P.esize && !fast &&
-                  !(hints && (hints->in_block > 0 || hints->out_block > 0))) {
+              if (P.W == P.esize && !(hints && (hints->in_block > 0 || hints->out_block > 0))) {
                 const int Kq = 16 / P.W;
                 const int64_t ra = round_block(blocksA[i], preA, P.n[a], Kq);
                 const int64_t rb = round_block(blocksB[j], preB, P.n[pb], Kq);
@@ -1564,30 +1560,25 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       win = rid[i];
     }
   }
-  // Second opinion for weak winners: when the first tree set predicts its
-  // winner below kVecChallenge of the copy speed, the second set (model_gbt2.h,
-  // refit with k_vec and the cal33 top candidates of configs 2-4 in its data)
-  // re-ranks the first set's short list together with the k_vec slices
-  // (matching-FVI problems: their own short list, refined here with the
-  // gather-conflict padding); its pick replaces the winner only when predicted
-  // kVecMargin faster.  Round-1 choices elsewhere are unchanged, and
-  // single-use plans (fast effort) consult only the k_vec slices.
+  // k_vec challenge: when the first tree set predicts its winner below
+  // kVecChallenge of the copy speed on a matching-FVI problem, the second set
+  // (model_gbt2.h, refit with k_vec in its data) compares it with the k_vec
+  // slices (their own short list, refined here with the gather-conflict
+  // padding); a k_vec slice replaces the winner only when predicted
+  // kVecMargin faster.  (Letting the second set re-rank the whole short list
+  // -- r2e16 -- gained 0.3-0.7 % on the odd 720-perm sweeps but put the
+  // closed-block cases onto 3.8 TB/s k_tile plans: not kept.)
   const Entry *Bp = &pool[win];
   const double ideal_t = 2.0 * (double)N * P.W / (dev.hbm_gbs * 1e9);
-  if (!listing && pool[win].lin < 1e299 && win_t > ideal_t / kVecChallenge &&
-      (nv > 0 || !fast)) {
-    const bool use_vec = nv > 0 && P.p[0] == 0;
+  if (!listing && pool[win].lin < 1e299 && win_t > ideal_t / kVecChallenge && nv > 0 &&
+      P.p[0] == 0) {
+    const bool use_vec = true;
     if (fast) nv = std::min(nv, 4);
-    ModelInput cm[kGbtTopK + kVecShort];
-    const Entry *ce[kGbtTopK + kVecShort];
+    ModelInput cm[1 + kVecShort];
+    const Entry *ce[1 + kVecShort];
     int m = 0;
     cm[m] = pool[win].mi;
     ce[m++] = &pool[win];
-    for (int i = 0; i < nrk && !fast; i++) {
-      if (rid[i] == win) continue;
-      cm[m] = rk[i];
-      ce[m++] = &pool[rid[i]];
-    }
     for (int i = 0; use_vec && i < nv; i++) {
       Entry &e = vpool[i];
       TileSummary S2;
@@ -1603,7 +1594,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       cm[m] = e.mi;
       ce[m++] = &e;
     }
-    double t2[kGbtTopK + kVecShort];
+    double t2[1 + kVecShort];
     predict_ranked2_batch(cm, m, dev, t2);
     int bj = 0;
     for (int j = 1; j < m; j++)

@@ -208,7 +208,7 @@ constexpr int kModelFeatureCount = 10;
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
 // fast = the single-use effort level: refine the linear screen's best
 // kFastRefine candidates and rank kFastTopK of them with the trees
-constexpr int kFastRefine = 6, kFastTopK = 6;
+constexpr int kFastRefine = 12, kFastTopK = 8;
 // in_strides / out_strides (elements; NULL = dense): the sub-tensor form of
 // ttlg_plan_strided -- in_strides[k] per input dim, out_strides[i] per output dim
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
