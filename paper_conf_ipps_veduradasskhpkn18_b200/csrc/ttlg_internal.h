@@ -206,9 +206,10 @@ struct CandidateSink {
 constexpr int kModelFeatureCount = 10;
 // planner.cpp
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
-// fast = the single-use effort level: refine the linear screen's best
-// kFastRefine candidates and rank kFastTopK of them with the trees
-constexpr int kFastRefine = 12, kFastTopK = 8;
+// fast = the single-use effort level: the same screen, refinement and tree
+// ranking as a repeated-use plan (so both pick the same kernel), minus the
+// shared-memory padding search and the reported-prediction tree pass
+constexpr int kFastRefine = 32, kFastTopK = 16;
 // in_strides / out_strides (elements; NULL = dense): the sub-tensor form of
 // ttlg_plan_strided -- in_strides[k] per input dim, out_strides[i] per output dim
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
