@@ -48,6 +48,8 @@ constexpr double kVecMargin = 0.95;
 // ... and is considered only when the first set predicts its winner below this
 // fraction of the copy speed
 constexpr double kVecChallenge = 0.8;
+// plans moving less than this many bytes (2 N s) are ranked by the second set
+constexpr double kSmallTraffic = 32.0 * 1024 * 1024;
 
 // k_deint (one streaming pass, 16-byte accesses both ways): time = this
 // factor x the one-pass ideal 2*N*s / HBM bandwidth -- measured on B200 at

@@ -1553,7 +1553,13 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     rk[nrk] = e.mi;
     rid[nrk++] = order[i];
   }
-  predict_ranked_batch(rk, nrk, dev, rt);
+  // tensors below kSmallTraffic bytes of traffic (launch-dominated, L2-resident)
+  // are outside the first tree set's data (>= 16 MB); the second set's data
+  // include 0.25-32 MB tensors, so it ranks them
+  if (2.0 * (double)N * P.W < kSmallTraffic)
+    predict_ranked2_batch(rk, nrk, dev, rt);
+  else
+    predict_ranked_batch(rk, nrk, dev, rt);
   for (int i = 0; i < nrk; i++) {
     if (rt[i] < win_t) {
       win_t = rt[i];
