@@ -269,6 +269,69 @@ __global__ void __launch_bounds__(512) k_direct(const __grid_constant__ TilePara
   }
 }
 
+// k_rows (FML / COPY, Alg. 7, with rows that are not a
+// multiple of 16 bytes -- odd fp64 extents such as 127^4, 15^6, 17^6): the
+// k_direct tile, but each row is copied by a group of G lanes with 16-byte
+// loads and stores wherever the source and destination rows share their
+// 16-byte phase (for all-odd extents every row does: A and B offsets of a row
+// have the same parity), with the head (up to 16/S - 1 elements before the
+// first 16-byte boundary) and the tail copied element-wise; rows whose
+// phases differ are copied element-wise.  G = the power of two covering the
+// row's chunks (at most 32): groups of 4-32 lanes per row.
+template <int S>
+__global__ void __launch_bounds__(512) k_rows(const __grid_constant__ TileParams P,
+                                              const __grid_constant__ BatchPtrs X) {
+  using T = typename Vec<S>::T;
+  constexpr int K = 16 / S;
+  extern __shared__ __align__(16) unsigned char smem[];
+  int2 *tabB = reinterpret_cast<int2 *>(smem + P.off_tabB);
+  int *digA = reinterpret_cast<int *>(smem + P.off_digA);
+  const T *A = reinterpret_cast<const T *>(X.A[blockIdx.y]);
+  T *B = reinterpret_cast<T *>(X.B[blockIdx.y]);
+
+  pdl_trigger();
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk, tabB, digA);
+  __syncthreads();
+  pdl_wait();
+
+  const int LB = P.LB, G = P.qk;  // qk: lanes per row
+  const int lane = threadIdx.x & (G - 1), grp = threadIdx.x / G, ngrp = blockDim.x / G;
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
+    if (tile >= P.num_tiles) break;
+    const TileCtx c = decode_tile(P, tile);
+    const int lim = P.LAunit * c.limA;  // valid input elements of the tile
+    const int nrows = (lim + LB - 1) / LB;
+    const T *Ab = A + c.bA;
+    T *Bb = B + c.bB;
+#pragma unroll 1
+    for (int r = grp; r < nrows; r += ngrp) {
+      const int len = min(LB, lim - r * LB);
+      const T *src = Ab + (int64_t)r * LB;
+      T *dst = Bb + tabB[r].x;
+      const uintptr_t sb = (uintptr_t)src, db = (uintptr_t)dst;
+      if (((sb ^ db) & 15) == 0) {
+        const int head = min(len, (int)(((16 - (db & 15)) & 15) / S));
+        const int nc = (len - head) / K;
+        if (lane < head) st_stream<true>(dst + lane, ld_stream<true>(src + lane));
+        const uint4 *s16 = reinterpret_cast<const uint4 *>(src + head);
+        uint4 *d16 = reinterpret_cast<uint4 *>(dst + head);
+        int k = lane;
+        for (; k + G < nc; k += 2 * G) {  // two 16-byte chunks in flight per lane
+          const uint4 v0 = __ldcs(s16 + k), v1 = __ldcs(s16 + k + G);
+          __stcs(d16 + k, v0);
+          __stcs(d16 + k + G, v1);
+        }
+        if (k < nc) __stcs(d16 + k, __ldcs(s16 + k));
+        const int t0 = head + nc * K;
+        if (lane < len - t0) st_stream<true>(dst + t0 + lane, ld_stream<true>(src + t0 + lane));
+      } else {
+        for (int e = lane; e < len; e += G) st_stream<true>(dst + e, ld_stream<true>(src + e));
+      }
+    }
+  }
+}
+
 // shared-memory helpers on 32-bit shared addresses (no generic->shared
 // conversion per access)
 __device__ __forceinline__ int2 lds_int2(uint32_t a) {
@@ -1480,6 +1543,8 @@ ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *c
                              ? bulk_ptr(plan->W, plan->kind)
                        : plan->kind == KK_VEC
                              ? (plan->W == 8 ? (const void *)k_vec<8> : (const void *)k_vec<4>)
+                       : (plan->kind == KK_DIRECT && plan->kp.qk > 0)
+                             ? (plan->W == 8 ? (const void *)k_rows<8> : (const void *)k_rows<4>)
                        : plan->kind == KK_DEINT
                              ? (plan->kp.deint_inter ? inter_ptr(plan->W, plan->kp.deint_n0)
                                                      : deint_ptr(plan->W, plan->kp.deint_n0))

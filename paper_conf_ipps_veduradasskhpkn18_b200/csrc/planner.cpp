@@ -193,6 +193,15 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;
+// FML / COPY rows that are not 16-byte multiples go through k_rows (TTLG_ROWS=0: k_direct)
+static bool rows16_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_ROWS");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
 constexpr int64_t kBulkTmaRowBytes = 2048;
 // TTLG_BULK_TMA=0/1 forces cp.async / TMA rows in k_bulk (experiments); -1: by row length
 static int bulk_tma_mode() {
@@ -664,6 +673,13 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   K.fd_LB = make_fastdiv((uint32_t)K.LB);
   K.fd_NT = make_fastdiv((uint32_t)threads);
   K.fd_rsB = make_fastdiv((uint32_t)(K.rsB > 0 ? K.rsB : 1));
+  if (kind == KK_DIRECT && (P.W == 4 || P.W == 8) && rows16_enabled()) {
+    // k_rows: rows that are not 16-byte multiples (no widening possible) move
+    // in 16-byte chunks between a head and a tail; qk = lanes per row
+    int G = 4;
+    while (G < 32 && G * 16 < K.LB * P.W + 16) G *= 2;
+    K.qk = G;
+  }
   return true;
 }
 

@@ -593,3 +593,25 @@ def test_bulk_partial_tiles(eb):
                 _assert_equal(got, exp, f"bulk partial {ext} {perm} {kw} {info}")
                 n_ok += 1
     assert n_ok >= 6
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_rows_fml_unaligned_rows(eb):
+    """k_rows (FML rows that are not 16-byte multiples): same-phase rows in
+    16-byte chunks between an element-wise head and tail, different-phase rows
+    element-wise; all-odd extents, mixed parities, row lengths of 1-300
+    elements, partial tiles and misaligned base pointers."""
+    for ext, perm in (([127, 7, 9], [0, 2, 1]), ([15, 15, 15, 15], [0, 2, 1, 3]),
+                      ([17, 6, 9, 5], [0, 3, 2, 1]), ([127, 128, 5], [0, 2, 1]),
+                      ([3, 50, 7], [0, 2, 1]), ([301, 3, 4, 5], [0, 3, 1, 2]),
+                      ([1, 5, 13, 11], [0, 3, 2, 1]), ([129, 33], [0, 1])):
+        got, exp, info = _run(ext, perm, eb, 1300, canary=32)
+        _assert_equal(got, exp, f"rows {ext} {perm} {info['kernel']}")
+        n = int(np.prod(ext))
+        A = gen_tensor_torch(1301, n + 3, eb, device=DEV)
+        B = torch.empty_like(A)
+        p = ttlg.plan(_dt(eb), ext, perm)
+        p.execute(A[1:].data_ptr(), B[3:].data_ptr(), torch.cuda.current_stream().cuda_stream)
+        torch.cuda.synchronize()
+        _assert_equal(_bits(B[3:]), oracle.transpose(_bits(A[1:n + 1]), ext, perm),
+                      f"rows misaligned {ext} {perm}")
