@@ -193,12 +193,15 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;
-// FML / COPY rows that are not 16-byte multiples go through k_rows (TTLG_ROWS=0: k_direct)
+// FML / COPY rows that are not 16-byte multiples go through k_rows only with
+// TTLG_ROWS=1: measured (r2e20) it loses to k_direct's 8 loads in flight per
+// thread on rows < 1 KB (720-perm sweeps 0.61-0.78x) and gains 5 % on the
+// 1016-byte rows of 127^4 -- kept as an option, off by default
 static bool rows16_enabled() {
   static int v = -1;
   if (v < 0) {
     const char *e = getenv("TTLG_ROWS");
-    v = (e && e[0] == '0') ? 0 : 1;
+    v = (e && e[0] == '1') ? 1 : 0;
   }
   return v == 1;
 }

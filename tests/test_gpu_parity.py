@@ -12,6 +12,7 @@
   path, non-default streams.
 """
 import itertools
+import os
 
 import numpy as np
 import pytest
@@ -600,7 +601,16 @@ def test_rows_fml_unaligned_rows(eb):
     """k_rows (FML rows that are not 16-byte multiples): same-phase rows in
     16-byte chunks between an element-wise head and tail, different-phase rows
     element-wise; all-odd extents, mixed parities, row lengths of 1-300
-    elements, partial tiles and misaligned base pointers."""
+    elements, partial tiles and misaligned base pointers.  k_rows is opt-in
+    (TTLG_ROWS=1, read once per process): run in a child process."""
+    import subprocess
+    import sys
+    if os.environ.get("TTLG_ROWS") != "1":
+        r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", __file__ + "::"
+                            f"test_rows_fml_unaligned_rows[{eb}]"],
+                           env={**os.environ, "TTLG_ROWS": "1"}, capture_output=True, text=True)
+        assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-2000:]
+        return
     for ext, perm in (([127, 7, 9], [0, 2, 1]), ([15, 15, 15, 15], [0, 2, 1, 3]),
                       ([17, 6, 9, 5], [0, 3, 2, 1]), ([127, 128, 5], [0, 2, 1]),
                       ([3, 50, 7], [0, 2, 1]), ([301, 3, 4, 5], [0, 3, 1, 2]),
