@@ -1,34 +1,44 @@
 // kernels.cu -- sm_100a transposition kernels of the B200 TTLG library.
 //
-// Two kernel families, templated on the access width W = 4/8/16 bytes:
+// Every kernel reads its launch parameters from two __grid_constant__ blocks
+// (TileParams: the plan's tile geometry and tables; BatchPtrs: the (A, B)
+// pair of blockIdx.y, ttlg_execute_batch) and moves elements as bit patterns.
 //
 //  k_direct  (FML / COPY; Alg. 7): the tile is a
 //            contiguous run of A (input dims 0..a, a blocked); elements are
 //            read with coalesced streaming loads, U per thread in flight, and
 //            written straight to their output row (output run = the matching
 //            FVI, dim 0).  No shared memory for data, only the row table.
+//  k_rows    (option, TTLG_ROWS=1): k_direct's tile with rows that are not
+//            16-byte multiples moved in 16-byte chunks between a head and tail.
 //
 //  k_pipe    (OD / OA / FMS; Alg. 2, Alg. 4/5 L868-1020, Alg. 6
 //            L1022-1107): the tile (the paper's "slice") is the union of an
 //            input-prefix group and an output-prefix group.  Load phase: A-rows
 //            of LA contiguous elements are copied global -> shared with cp.async
-//            (LDGSTS, predicated PTX); store phase: B-rows of LB
-//            contiguous elements are read from shared memory through the column
-//            offsets and written coalesced.  Rows are processed warp-wise: a
-//            warp (or a power-of-two lane group of G <= 32 lanes when the run is
-//            short) owns a row, so the row-table lookup is a broadcast and the
-//            column offsets are register-resident -- the B200 form of the
-//            paper's compile-time-constant indexing (L1138-1155).  The
-//            shared-memory layout pads every output-only dim so that output
-//            position j lands in bank j mod (128/W): conflict-free column reads
-//            (generalising the 32x33 pad, L747-749, and FMS's pad, L1104-1107).
+//            (LDGSTS, predicated PTX); store phase: B-rows of LB contiguous
+//            elements are read from shared memory through the column offsets
+//            and written coalesced.  The shared-memory layout pads every
+//            output-only dim so that output position j lands in bank
+//            j mod (128/W): conflict-free column reads (generalising the 32x33
+//            pad, L747-749, and FMS's pad, L1104-1107).  Two grid strategies:
+//            PERSIST = false ("k_tile": one tile, or a few consecutive tiles,
+//            per CTA, many CTAs per SM) and PERSIST = true ("k_pipe":
+//            persistent CTAs with a double-buffered cp.async ring).
+//  k_quad    (OD): the same tile in 16-byte chunks both ways, K x K register
+//            transposes with xor-shuffles in the store phase.
+//  k_vec     (any schema with 16-byte aligned rows): 16-byte chunk loads,
+//            16-byte stores gathered from K element reads (FMS 12/20/28-byte
+//            pencils).
+//  k_bulk    (option; TMA experiment): persistent, warp-specialised -- one
+//            cp.async.bulk per A-row into an mbarrier ring, consumer warps
+//            drain with k_quad's transposes or k_vec's gathers.
+//  k_deint / k_inter (OA with a tiny FVI: AoS <-> SoA): 16-byte accesses
+//            both ways through per-warp swizzled staging buffers.
 //
-// Two grid strategies compete per candidate: PERSIST = false ("k_tile"): one
-// CTA per tile (or a few consecutive tiles, `tpc`), single buffer, many CTAs
-// per SM; PERSIST = true ("k_pipe"): persistent CTAs with a double-buffered
-// cp.async ring.  k_direct uses one CTA per tile.  Every CTA builds its row tables in shared memory
-// (the paper's texture-mapped offset arrays, L737-745) and decodes its tile
-// index with fast-divmod (the paper's decode/compute_base, L725-737).
+// Every staged CTA builds its row tables in shared memory (the paper's
+// texture-mapped offset arrays, L737-745) and decodes its tile index with
+// fast-divmod (the paper's decode/compute_base, L725-737).
 #include <cuda_runtime.h>
 
 #include <atomic>
