@@ -1001,6 +1001,165 @@ __global__ void __launch_bounds__(512, 4) k_vec(const __grid_constant__ TilePara
   }
 }
 
+// k_phase (OD / OA / FMS whose rows start at any element -- odd fp64
+// extents such as 15^6 / 17^6, where no row is 16-byte aligned): k_tile's
+// slice, but the load phase moves every A-row as 16-byte cp.async chunks from
+// the 16-byte boundary at or below the row start.  Row r of a tile then sits
+// in its (16-byte aligned) shared-memory slot shifted by its phase
+// ph(r) = (tile base + A offset of r) mod K (K = 16/S), and the store walk
+// adds ph * S to every shared-memory read: the phase is the sum of the tile's
+// and the row digits' contributions, kept in the low bits of the B-row table
+// and the column offsets (both multiples of S bytes, so those bits are
+// free).  Each slot holds LAc = (LA + 2K - 2) / K chunks (the over-read
+// neighbours land inside it); a chunk that would cross the end of A is
+// loaded element by element.  Stores stay element-wise (the output rows have
+// arbitrary alignment too), one output position per thread as in k_pipe.
+__device__ __forceinline__ void build_rows_ph(int R, int nr, const FastDiv *ext,
+                                              const int32_t *sG, const int32_t *sS,
+                                              const int32_t *sP, int blk, int2 *tab, int *dig,
+                                              int sw, int pm) {
+#pragma unroll 1
+  for (int i = threadIdx.x; i < R; i += blockDim.x) {
+    int rem = i, g = 0, s = 0, ph = 0, dg = 0;
+    for (int k = 0; k < nr; k++) {
+      const int cq = (int)fdiv((uint32_t)rem, ext[k]);
+      const int c = rem - cq * (int)ext[k].div;
+      rem = cq;
+      g += c * sG[k];
+      s += c * sS[k];
+      ph += c * sP[k];
+      if (k == blk) dg = c;
+    }
+    tab[i] = make_int2(g, s * sw + (ph & pm));
+    dig[i] = dg;
+  }
+}
+
+template <int S>
+__global__ void __launch_bounds__(512, 4) k_phase(const __grid_constant__ TileParams P,
+                                                  const __grid_constant__ BatchPtrs X) {
+  using T = typename Vec<S>::T;
+  constexpr int K = 16 / S, M = K - 1;
+  const T *A = reinterpret_cast<const T *>(X.A[blockIdx.y]);
+  T *B = reinterpret_cast<T *>(X.B[blockIdx.y]);
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabA = s0, s_tabB = s0 + P.off_tabB, s_jcol = s0 + P.off_jcol;
+  const uint32_t s_digB = s0 + P.off_digB, s_digA = s0 + P.off_digA;
+  const uint32_t s_buf = s0 + P.off_data;
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
+  const int tid = threadIdx.x, NT = blockDim.x;
+  const bool decoder = tid == NT - 1;
+  const uint32_t first = blockIdx.x * (uint32_t)P.tpc;
+
+  auto put_ctx = [&](int slot, uint32_t tile) {
+    const TileCtx c = decode_tile(P, tile);
+    ctx[slot].bA = c.bA;
+    ctx[slot].bB = c.bB;
+    ctx[slot].limA = c.limA;
+    ctx[slot].limB = c.limB;
+  };
+  auto get_ctx = [&](int slot) {
+    TileCtx c;
+    c.bA = ctx[slot].bA;
+    c.bB = ctx[slot].bB;
+    c.limA = ctx[slot].limA;
+    c.limB = ctx[slot].limB;
+    return c;
+  };
+  pdl_trigger();
+  if (decoder && first < P.num_tiles) put_ctx(0, first);
+  build_rows(P.RA, P.nra, P.ra_div, P.ra_sG, P.ra_sS, P.ra_blk, reinterpret_cast<int2 *>(smem),
+             reinterpret_cast<int *>(smem + P.off_digB), S);
+  __syncthreads();  // tabA, digB, ctx[0] visible
+  pdl_wait();
+
+  const int LB = P.LB, LAc = P.qk;  // qk: 16-byte chunks per A-row slot
+  const int nChunks = P.RA * LAc;
+  const int rA0 = (int)fdiv1(tid, P.fd_LA), cA0 = tid - rA0 * LAc;
+  const int nA = tid < nChunks ? (int)fdiv1(nChunks - 1 - tid, P.fd_NT) + 1 : 0;
+  const int drA = P.drA, dxA = P.dxA;
+  const int64_t aN = P.a_elems;
+  auto load = [&](const TileCtx &c, bool full) {
+    int r = rA0, cx = cA0;
+#pragma unroll 4
+    for (int k = 0; k < nA; k++) {
+      const int2 t = lds_int2(s_tabA + 8 * r);
+      const int64_t e0 = ((c.bA + t.x) & ~(int64_t)M) + (int64_t)K * cx;  // chunk's first element
+      const uint32_t sd = s_buf + t.y + 16 * cx;
+      const bool ok = full || lds_int(s_digB + 4 * r) < c.limB;
+      if (e0 + K <= aN) {
+        cp_async_p<16>(sd, A + e0, ok);
+      } else {
+#pragma unroll
+        for (int u = 0; u < K; u++) cp_async_p<S>(sd + u * S, A + e0 + u, ok && e0 + u < aN);
+      }
+      cx += dxA;
+      r += drA;
+      if (cx >= LAc) {
+        cx -= LAc;
+        r++;
+      }
+    }
+  };
+  TileCtx c = get_ctx(0);
+  bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+  if (first < P.num_tiles) load(c, full);
+  cp_async_commit();
+
+  build_rows_ph(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_sP, P.rb_blk,
+                reinterpret_cast<int2 *>(smem + P.off_tabB),
+                reinterpret_cast<int *>(smem + P.off_digA), S, M);
+#pragma unroll 1
+  for (int j = tid; j < LB; j += NT) {
+    int rem = j, sm = 0, ph = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const int cq = (int)fdiv((uint32_t)rem, P.j_div[k]);
+      const int d = rem - cq * (int)P.j_div[k].div;
+      sm += d * P.j_sS[k];
+      ph += d * P.j_sP[k];
+      rem = cq;
+    }
+    reinterpret_cast<int *>(smem + P.off_jcol)[j] = sm * S + (ph & M);
+  }
+  __syncthreads();  // tabB, digA, jcol visible (the first tile's loads still in flight)
+
+  // store walk: one output position j0 per thread, B-rows m0 + k rs
+  const int m0 = (int)fdiv1(tid, P.fd_LB);
+  const int j0 = tid - m0 * LB;
+  const int rs = P.rsB;
+  const int nB = (m0 < rs && m0 < P.RB) ? (int)fdiv1(P.RB - 1 - m0, P.fd_rsB) + 1 : 0;
+  const int jc = lds_int(s_jcol + 4 * (j0 < LB ? j0 : 0));
+
+  for (int it = 0; it < P.tpc; it++) {
+    const uint32_t tile = first + it;
+    if (tile >= P.num_tiles) break;
+    if (it > 0) {
+      __syncthreads();  // buffer drained, ctx[it & 1] visible
+      c = get_ctx(it & 1);
+      full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+      load(c, full);
+      cp_async_commit();
+    }
+    if (decoder && it + 1 < P.tpc && tile + 1 < P.num_tiles) put_ctx((it + 1) & 1, tile + 1);
+    cp_async_wait<0>();
+    __syncthreads();
+    const int tp = (int)(c.bA & M);
+    const bool jok = full || j0 < P.LBunit * c.limB;
+    T *dst = B + c.bB + j0;
+    const uint32_t sj = s_buf + (uint32_t)(jc & ~M);
+    int r = m0;
+#pragma unroll 4
+    for (int k = 0; k < nB; k++) {
+      const int2 t = lds_int2(s_tabB + 8 * r);
+      const uint32_t a = sj + (uint32_t)(t.y & ~M) + (uint32_t)(((t.y + jc + tp) & M) * S);
+      stcs_p(wadd(dst, (uint32_t)t.x), lds_T<T>(a),
+             jok && (full || lds_int(s_digA + 4 * r) < c.limA));
+      r += rs;
+    }
+  }
+}
+
 // k_deint (Orthogonal-Arbitrary with a tiny input FVI: array-of-structures ->
 // structure-of-arrays): the fused problem [n0, M] perm (1 0), or the batch
 // [n0, M, nb] perm (1 0 2), with N0 = n0 <= 8 and M a multiple of K = 16/S.
@@ -1504,7 +1663,8 @@ int kernel_regs(int kind, int W) {
   static std::atomic<int> regs[KK_NUM][3] = {{{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
-                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
+                                             {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
   if (r >= 0) return r;
@@ -1518,6 +1678,7 @@ int kernel_regs(int kind, int W) {
                      : (kind == KK_BULKQ || kind == KK_BULKG)
                          ? bulk_ptr(W, kind)
                      : kind == KK_VEC ? (W == 8 ? (const void *)k_vec<8> : (const void *)k_vec<4>)
+                     : kind == KK_PHASE ? (W == 8 ? (const void *)k_phase<8> : (const void *)k_phase<4>)
                          : kernel_ptr(kind, W, false, false);
     if (cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
       r = attr.numRegs;
@@ -1553,6 +1714,8 @@ ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *c
                              ? bulk_ptr(plan->W, plan->kind)
                        : plan->kind == KK_VEC
                              ? (plan->W == 8 ? (const void *)k_vec<8> : (const void *)k_vec<4>)
+                       : plan->kind == KK_PHASE
+                             ? (plan->W == 8 ? (const void *)k_phase<8> : (const void *)k_phase<4>)
                        : (plan->kind == KK_DIRECT && plan->kp.qk > 0)
                              ? (plan->W == 8 ? (const void *)k_rows<8> : (const void *)k_rows<4>)
                        : plan->kind == KK_DEINT

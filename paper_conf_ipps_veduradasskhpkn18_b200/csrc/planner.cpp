@@ -193,6 +193,15 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;
+// k_phase substitution mode (TTLG_PHASE: 0 off, 1 rows off 16-byte boundaries, 2 always)
+static int phase_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_PHASE");
+    v = (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : 1;
+  }
+  return v;
+}
 // FML / COPY rows that are not 16-byte multiples go through k_rows only with
 // TTLG_ROWS=1: measured (r2e20) it loses to k_direct's 8 loads in flight per
 // thread on rows < 1 KB (720-perm sweeps 0.61-0.78x) and gains 5 % on the
@@ -386,7 +395,7 @@ struct TileSummary {
 // every A-row on a 16-byte (chunk) boundary
 static int layout_unit(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_QUAD) return quad_k(P, T);
-  if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_VEC) return 16 / P.W;
+  if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_VEC || kind == KK_PHASE) return 16 / P.W;
   return 0;
 }
 
@@ -512,6 +521,11 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     sm[k] = cur + pad;
     cur = sm[k] * T.t[k];
   }
+  if (kind == KK_PHASE) {
+    // every A-row slot holds the row shifted by its phase: (LA + 2K - 2) / K chunks
+    if (xtab || (P.W != 4 && P.W != 8)) return false;
+    cur = (cur + 2 * qk - 2) / qk * qk;
+  }
   int64_t Q = 1, mult = 0;
   bool od = true;
   for (int i = 0; i <= b; i++) od &= !inIS[P.p[i]];
@@ -554,6 +568,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.rb_div[K.nrb] = make_fastdiv((uint32_t)T.t[k]);
     K.rb_sG[K.nrb] = (int32_t)S.sB[k];
     K.rb_sS[K.nrb] = (int32_t)sm[k];
+    K.rb_sP[K.nrb] = (qk > 0 && !inIS[k]) ? (int32_t)(S.sA[k] % qk) : 0;  // k_phase
     maxG += (T.t[k] - 1) * S.sB[k];
     K.nrb++;
   }
@@ -565,6 +580,7 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.j_ext[K.nj] = (int32_t)T.t[k];
     K.j_div[K.nj] = make_fastdiv((uint32_t)T.t[k]);
     K.j_sS[K.nj] = (int32_t)sm[k];
+    K.j_sP[K.nj] = (qk > 0 && !inIS[k]) ? (int32_t)(S.sA[k] % qk) : 0;  // k_phase
     K.nj++;
   }
   if (smem_elems >= (1ll << 30)) return false;
@@ -647,6 +663,21 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.fd_LB = make_fastdiv((uint32_t)L);
     K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
     K.fd_NT = make_fastdiv((uint32_t)ntc);
+    return true;
+  }
+  if (kind == KK_PHASE) {
+    // load walk over the slots' 16-byte chunks; store walk: one output
+    // position per thread (k_pipe's non-SM2 walk)
+    const int LAc = (int)((K.LA + 2 * qk - 2) / qk);
+    if (K.LB > threads || threads % 32) return false;
+    K.qk = LAc;
+    K.drA = threads / LAc;
+    K.dxA = threads % LAc;
+    K.fd_LA = make_fastdiv((uint32_t)LAc);
+    K.rsB = threads / K.LB;
+    K.fd_LB = make_fastdiv((uint32_t)K.LB);
+    K.fd_NT = make_fastdiv((uint32_t)threads);
+    K.fd_rsB = make_fastdiv((uint32_t)K.rsB);
     return true;
   }
   if (kind == KK_VEC) {
@@ -1178,8 +1209,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       if (hv == 0 ? !new_kernel_auto(group) : hv != want) return;
       // in the automatic choice k_vec only challenges matching-FVI winners (below)
       if (hv == 0 && group == KK_VEC && P.p[0] != 0 && !listing) return;
-    } else if (hv >= 5) {
+    } else if (hv >= 5 && hv != 8) {
       return;  // k_bulk / k_vec forced
+    } else if (hv == 8 && group != KK_TILE) {
+      return;  // k_phase forced: the staged slices only (substituted below)
     }
     if (hints) {
       if (hints->in_dim >= 0 && hints->in_dim != a) return;
@@ -1675,14 +1708,48 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       return TTLG_ERR_INTERNAL;
     K.tpc = B.tpc;
   }
-  plan->kind = B.kind;
+  int kind_final = B.kind, grid_final = B.mi.grid;
+  {
+    // k_phase substitution: the winner's k_tile / k_pipe slice with 16-byte
+    // loads whatever the rows' alignment (TTLG_PHASE=0 off, 1 [default] when
+    // some A-row of the slice starts off a 16-byte boundary, 2 always; hints
+    // variant 8 forces it)
+    bool padded = false;
+    for (int k = 0; k < TTLG_MAXD; k++) padded |= B.delta[k] != 0;
+    const int mode = hv == 8 ? 2 : phase_mode();
+    if ((B.kind == KK_TILE || B.kind == KK_PIPE) && !padded && mode > 0 && !forceW &&
+        P.W == P.esize && (P.W == 4 || P.W == 8) && !listing) {
+      bool unaligned = (K.LA * P.W) % 16 != 0;
+      for (int k = 0; k < P.d && !unaligned; k++) {
+        const bool inrun = k <= B.T.a;
+        if (!inrun && B.T.t[k] > 1 && (P.sA[k] * P.W) % 16) unaligned = true;
+        if (P.n[k] > B.T.t[k] && (B.T.t[k] * P.sA[k] * P.W) % 16) unaligned = true;
+      }
+      TileParams Kp;
+      if ((mode == 2 || unaligned) && build_params(P, B.T, KK_PHASE, B.mi.threads, 1, Kp) &&
+          Kp.smem_bytes <= dev.smem_per_block_optin) {
+        Kp.tpc = B.kind == KK_TILE ? B.tpc : 1;
+        Kp.a_elems = spanA;
+        K = Kp;
+        kind_final = KK_PHASE;
+        grid_final = (int)((K.num_tiles + K.tpc - 1) / K.tpc);
+      } else if (hv == 8) {
+        return TTLG_ERR_UNSUPPORTED;
+      }
+    } else if (hv == 8) {
+      return TTLG_ERR_UNSUPPORTED;
+    }
+  }
+  plan->kind = kind_final;
   plan->variant = hints ? hints->variant : 0;
   plan->W = P.W;
-  plan->align = B.kind == KK_QUAD ? K.qk * P.W
-                : (B.kind == KK_BULKQ || B.kind == KK_BULKG || B.kind == KK_VEC) ? 16
-                                                             : P.W;
+  plan->align = kind_final == KK_QUAD ? K.qk * P.W
+                : (kind_final == KK_BULKQ || kind_final == KK_BULKG || kind_final == KK_VEC ||
+                   kind_final == KK_PHASE)
+                    ? 16
+                    : P.W;
   plan->threads = B.mi.threads;
-  plan->grid = B.mi.grid;
+  plan->grid = grid_final;
   plan->nbytes = N * P.W;
   plan->spanA = spanA * s;
   plan->spanB = spanB * s;
@@ -1692,7 +1759,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // L2-resident): the first set only ranks
   double t_report = win_t;
   if (!listing && !fast) predict_ranked2_batch(&B.mi, 1, dev, &t_report);  // single use: skip
-  fill_info(plan->info, dt, rank, P, B.T, K, B.mi, B.schema, B.kind, t_report, ncand);
+  fill_info(plan->info, dt, rank, P, B.T, K, B.mi, B.schema, kind_final, t_report, ncand);
+  plan->info.grid = grid_final;
   {
     const ModelFeatures F = model_features(B.mi, dev);
     plan->info.num_features = kModelFeatureCount;

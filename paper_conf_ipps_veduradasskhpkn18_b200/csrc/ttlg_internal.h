@@ -57,7 +57,9 @@ enum KernelKind : int32_t {
                   // element reads (k_bulk, consumer mode gather)
   KK_VEC = 7,     // any schema with 16-byte aligned rows: 16-byte cp.async loads, 16-byte
                   // stores gathered from K element reads (k_vec)
-  KK_NUM = 8,
+  KK_PHASE = 8,   // k_tile's slice with 16-byte loads at any row alignment (per-row phase
+                  // in shared memory) and element stores (k_phase)
+  KK_NUM = 9,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -124,6 +126,11 @@ struct TileParams {
   // 2 * nstage mbarriers at off_bar (full[s], empty[s]); warp 0 produces
   int32_t nstage, stage_bytes, off_bar;
   int32_t tma_rows;  // 1: one TMA bulk copy per A-row; 0: 16-byte cp.async chunks
+  // k_phase: A-offset phase (mod 16/W) contributed by each B-row digit and each
+  // output-run digit (0 for input-run dims); elements of A (end-of-tensor guard)
+  int32_t rb_sP[TTLG_MAXD];
+  int32_t j_sP[TTLG_MAXD];
+  int64_t a_elems;
 };
 
 // Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;

@@ -334,7 +334,7 @@ _VARIANT_CASES = [
 ]
 
 
-@pytest.mark.parametrize("variant", [1, 2, 3, 5, 6, 7])
+@pytest.mark.parametrize("variant", [1, 2, 3, 5, 6, 7, 8])
 @pytest.mark.parametrize("ext,perm,eb", _VARIANT_CASES)
 def test_kernel_variants_forced(ext, perm, eb, variant):
     try:
@@ -625,3 +625,31 @@ def test_rows_fml_unaligned_rows(eb):
         torch.cuda.synchronize()
         _assert_equal(_bits(B[3:]), oracle.transpose(_bits(A[1:n + 1]), ext, perm),
                       f"rows misaligned {ext} {perm}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_phase_forced_odd_extents(eb):
+    """k_phase (16-byte loads at any row alignment, per-row phase in shared
+    memory): every rank-4 perm of odd and mixed extents, ragged tiles, the
+    end-of-tensor chunk, misaligned-by-one-element views (element-width twin)."""
+    n_ok = 0
+    for ext in ([15, 17, 13, 19], [3, 33, 65, 7], [17, 6, 9, 5], [5, 2, 129, 31]):
+        for k, perm in enumerate(itertools.permutations(range(4))):
+            try:
+                ttlg.plan(_dt(eb), ext, list(perm), variant=8)
+            except ttlg.TtlgError:
+                continue
+            got, exp, info = _run(ext, list(perm), eb, 1400 + k,
+                                  plan_kwargs={"variant": 8}, canary=32)
+            assert info["kernel"] == "phase"
+            _assert_equal(got, exp, f"phase {ext} {perm} {info['tile_extents']}")
+            n_ok += 1
+    assert n_ok >= 40
+    for ext, perm in (([17, 17, 17, 17], [3, 1, 2, 0]), ([15, 15, 15], [2, 0, 1])):
+        for tiles in ({}, {"in_dim": 0, "in_block": 7, "out_dim": 0, "out_block": 5}):
+            try:
+                ttlg.plan(_dt(eb), ext, perm, variant=8, **tiles)
+            except ttlg.TtlgError:
+                continue
+            got, exp, _ = _run(ext, perm, eb, 1500, plan_kwargs={"variant": 8, **tiles}, canary=32)
+            _assert_equal(got, exp, f"phase {ext} {perm} {tiles}")
