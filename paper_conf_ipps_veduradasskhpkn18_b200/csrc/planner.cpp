@@ -193,12 +193,16 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : bulk;
 }
 constexpr int kBulkMaxStages = 6;
-// k_phase substitution mode (TTLG_PHASE: 0 off, 1 rows off 16-byte boundaries, 2 always)
+// k_phase substitution mode (TTLG_PHASE: 0 off [default], 1 rows off 16-byte
+// boundaries, 2 always).  Measured on the 720-perm sweeps (r2e22): halving
+// the load instructions does not pay for the phase arithmetic and the
+// shifted (bank-conflicting) rows in the element-wise store phase -- 17^6
+// 0.91x, 15^6 0.94x on average -- so it is an option, not the default.
 static int phase_mode() {
   static int v = -1;
   if (v < 0) {
     const char *e = getenv("TTLG_PHASE");
-    v = (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : 1;
+    v = (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : 0;
   }
   return v;
 }
@@ -1711,8 +1715,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   int kind_final = B.kind, grid_final = B.mi.grid;
   {
     // k_phase substitution: the winner's k_tile / k_pipe slice with 16-byte
-    // loads whatever the rows' alignment (TTLG_PHASE=0 off, 1 [default] when
-    // some A-row of the slice starts off a 16-byte boundary, 2 always; hints
+    // loads whatever the rows' alignment (TTLG_PHASE=1 when some A-row of the
+    // slice starts off a 16-byte boundary, 2 always, 0 [default] never; hints
     // variant 8 forces it)
     bool padded = false;
     for (int k = 0; k < TTLG_MAXD; k++) padded |= B.delta[k] != 0;
