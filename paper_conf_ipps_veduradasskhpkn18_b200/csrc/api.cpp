@@ -83,10 +83,11 @@ static int current_device() {
 }
 
 constexpr double kFastPlanSeconds = 150e-6;
+constexpr double kFast2PlanSeconds = 35e-6;  // shorter than a fast-effort plan
 
 static ttlg_status plan_into(ttlg_plan_s *p, ttlg_dtype dt, int rank, const int64_t *ext,
                              const int32_t *perm, const ttlg_plan_hints *hints,
-                             bool fast = false, const int64_t *in_strides = nullptr,
+                             int fast = 0, const int64_t *in_strides = nullptr,
                              const int64_t *out_strides = nullptr) {
   const int dev = current_device();
   ttlg_status st = make_plan(p, dt, rank, ext, perm, hints, device_profile(dev), nullptr, fast,
@@ -438,7 +439,8 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
   if (st != TTLG_OK) return st;
   double bytes = 2.0 * (dt == TTLG_F64 ? 8 : 4);
   for (int k = 0; k < rank; k++) bytes *= (double)extents[k];
-  const bool fast = bytes / (device_profile(current_device()).hbm_gbs * 1e9) < kFastPlanSeconds;
+  const double pass = bytes / (device_profile(current_device()).hbm_gbs * 1e9);
+  const int fast = pass < kFast2PlanSeconds ? 2 : (pass < kFastPlanSeconds ? 1 : 0);
   st = plan_into(&p, dt, rank, extents, perm, nullptr, fast);
   if (st != TTLG_OK) return st;
   return execute(&p, A, B, stream);

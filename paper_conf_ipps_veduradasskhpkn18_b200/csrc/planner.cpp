@@ -910,7 +910,7 @@ static void fill_info(ttlg_plan_info &I, ttlg_dtype dt, int rank, const Problem 
 
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints,
-                      const DeviceProfile &dev, CandidateSink *sink, bool fast,
+                      const DeviceProfile &dev, CandidateSink *sink, int fast,
                       const int64_t *in_strides, const int64_t *out_strides) {
   ttlg_status st = validate(dt, rank, ext, perm);
   if (st != TTLG_OK) return st;
@@ -1562,7 +1562,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int nd = 0;
     // fast planning (single-use calls on small tensors): refine only the
     // linear screen's best few; the rest drop out
-    const int nref = fast ? std::min(ntop, kFastRefine) : ntop;
+    const int nref = fast >= 2 ? std::min(ntop, kFast2Refine)
+                     : fast   ? std::min(ntop, kFastRefine)
+                              : ntop;
     for (int i = nref; i < ntop; i++) pool[order[i]].lin = 1e300;
     for (int ii = 0; ii < nref; ii++) {
       Entry &e = pool[order[ii]];
@@ -1602,7 +1604,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   ModelInput rk[kGbtTopK];
   int rid[kGbtTopK], nrk = 0;
   double rt[kGbtTopK];
-  const int topk = fast ? kFastTopK : kGbtTopK;
+  const int topk = fast >= 2 ? kFast2TopK : (fast ? kFastTopK : kGbtTopK);
   for (int i = 0; i < std::min(ntop, topk); i++) {
     const Entry &e = pool[order[i]];
     if (e.lin >= 1e299) continue;

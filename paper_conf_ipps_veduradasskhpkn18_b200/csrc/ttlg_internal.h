@@ -213,15 +213,18 @@ struct CandidateSink {
 constexpr int kModelFeatureCount = 10;
 // planner.cpp
 ttlg_status validate(ttlg_dtype dt, int rank, const int64_t *ext, const int32_t *perm);
-// fast = the single-use effort level: the same screen, refinement and tree
-// ranking as a repeated-use plan (so both pick the same kernel), minus the
-// shared-memory padding search and the reported-prediction tree pass
+// fast = the single-use effort level.  1: the same screen, refinement and
+// tree ranking as a repeated-use plan (so both pick the same kernel), minus
+// the shared-memory padding search and the reported-prediction tree pass;
+// 2 (passes shorter than a plan, e.g. 15^6 fp64): also refine only the
+// linear screen's best kFast2Refine and rank kFast2TopK with the trees
 constexpr int kFastRefine = 32, kFastTopK = 16;
+constexpr int kFast2Refine = 8, kFast2TopK = 6;
 // in_strides / out_strides (elements; NULL = dense): the sub-tensor form of
 // ttlg_plan_strided -- in_strides[k] per input dim, out_strides[i] per output dim
 ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t *ext,
                       const int32_t *perm, const ttlg_plan_hints *hints, const DeviceProfile &dev,
-                      CandidateSink *sink = nullptr, bool fast = false,
+                      CandidateSink *sink = nullptr, int fast = 0,
                       const int64_t *in_strides = nullptr, const int64_t *out_strides = nullptr);
 // api.cpp
 const DeviceProfile &device_profile(int device);
