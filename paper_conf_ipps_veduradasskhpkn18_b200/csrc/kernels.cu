@@ -306,6 +306,9 @@ __global__ void __launch_bounds__(512) k_rows(const __grid_constant__ TileParams
 
   const int LB = P.LB, G = P.qk;  // qk: lanes per row
   const int lane = threadIdx.x & (G - 1), grp = threadIdx.x / G, ngrp = blockDim.x / G;
+  // NR rows per group in flight, up to 2 chunks of each per lane (rows of up
+  // to 2G chunks; longer rows loop their remaining chunks after the batch)
+  constexpr int NR = 4;
   for (int it = 0; it < P.tpc; it++) {
     const uint32_t tile = blockIdx.x * (uint32_t)P.tpc + it;
     if (tile >= P.num_tiles) break;
@@ -315,28 +318,52 @@ __global__ void __launch_bounds__(512) k_rows(const __grid_constant__ TileParams
     const T *Ab = A + c.bA;
     T *Bb = B + c.bB;
 #pragma unroll 1
-    for (int r = grp; r < nrows; r += ngrp) {
-      const int len = min(LB, lim - r * LB);
-      const T *src = Ab + (int64_t)r * LB;
-      T *dst = Bb + tabB[r].x;
-      const uintptr_t sb = (uintptr_t)src, db = (uintptr_t)dst;
-      if (((sb ^ db) & 15) == 0) {
-        const int head = min(len, (int)(((16 - (db & 15)) & 15) / S));
-        const int nc = (len - head) / K;
-        if (lane < head) st_stream<true>(dst + lane, ld_stream<true>(src + lane));
-        const uint4 *s16 = reinterpret_cast<const uint4 *>(src + head);
-        uint4 *d16 = reinterpret_cast<uint4 *>(dst + head);
-        int k = lane;
-        for (; k + G < nc; k += 2 * G) {  // two 16-byte chunks in flight per lane
-          const uint4 v0 = __ldcs(s16 + k), v1 = __ldcs(s16 + k + G);
-          __stcs(d16 + k, v0);
-          __stcs(d16 + k + G, v1);
+    for (int r = grp; r < nrows; r += NR * ngrp) {
+      const T *src[NR];
+      T *dst[NR];
+      int len[NR], head[NR], nc[NR];
+      uint4 v0[NR], v1[NR];
+#pragma unroll
+      for (int q = 0; q < NR; q++) {
+        const int rq = r + q * ngrp;
+        len[q] = rq < nrows ? min(LB, lim - rq * LB) : 0;
+        src[q] = Ab + (int64_t)rq * LB;
+        dst[q] = Bb + (len[q] > 0 ? tabB[rq].x : 0);
+        const uintptr_t sb = (uintptr_t)src[q], db = (uintptr_t)dst[q];
+        if (len[q] > 0 && ((sb ^ db) & 15) == 0) {
+          head[q] = min(len[q], (int)(((16 - (db & 15)) & 15) / S));
+          nc[q] = (len[q] - head[q]) / K;
+        } else {
+          head[q] = len[q];  // element-wise row (or none)
+          nc[q] = 0;
         }
-        if (k < nc) __stcs(d16 + k, __ldcs(s16 + k));
-        const int t0 = head + nc * K;
-        if (lane < len - t0) st_stream<true>(dst + t0 + lane, ld_stream<true>(src + t0 + lane));
-      } else {
-        for (int e = lane; e < len; e += G) st_stream<true>(dst + e, ld_stream<true>(src + e));
+        const uint4 *s16 = reinterpret_cast<const uint4 *>(src[q] + head[q]);
+        if (lane < nc[q]) v0[q] = __ldcs(s16 + lane);
+        if (lane + G < nc[q]) v1[q] = __ldcs(s16 + lane + G);
+      }
+#pragma unroll
+      for (int q = 0; q < NR; q++) {
+        if (len[q] == 0) continue;
+        uint4 *d16 = reinterpret_cast<uint4 *>(dst[q] + head[q]);
+        if (lane < nc[q]) __stcs(d16 + lane, v0[q]);
+        if (lane + G < nc[q]) __stcs(d16 + lane + G, v1[q]);
+        if (nc[q] > 2 * G) {  // long rows: 4 chunks per lane in flight
+          const uint4 *s16 = reinterpret_cast<const uint4 *>(src[q] + head[q]);
+          for (int k = lane + 2 * G; k < nc[q]; k += 4 * G) {
+            uint4 w[4];
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+              if (k + u * G < nc[q]) w[u] = __ldcs(s16 + k + u * G);
+#pragma unroll
+            for (int u = 0; u < 4; u++)
+              if (k + u * G < nc[q]) __stcs(d16 + k + u * G, w[u]);
+          }
+        }
+        // head (a misaligned row: the whole row) and tail, element-wise
+        for (int e = lane; e < head[q]; e += G) st_stream<true>(dst[q] + e, ld_stream<true>(src[q] + e));
+        const int t0 = head[q] + nc[q] * K;
+        for (int e = t0 + lane; e < len[q]; e += G)
+          st_stream<true>(dst[q] + e, ld_stream<true>(src[q] + e));
       }
     }
   }
@@ -1622,6 +1649,8 @@ static const void *inter_ptr(int W, int n1) {
 
 // ---------------------------------------------------------------------------
 // launch plumbing
+
+
 template <int W, bool XT>
 static const void *kernel_ptr_x(int kind, bool sm2) {
   if (kind == KK_PIPE)

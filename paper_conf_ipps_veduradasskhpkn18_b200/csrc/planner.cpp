@@ -209,7 +209,10 @@ static int phase_mode() {
 // FML / COPY rows that are not 16-byte multiples go through k_rows only with
 // TTLG_ROWS=1: measured (r2e20) it loses to k_direct's 8 loads in flight per
 // thread on rows < 1 KB (720-perm sweeps 0.61-0.78x) and gains 5 % on the
-// 1016-byte rows of 127^4 -- kept as an option, off by default
+// 1016-byte rows of 127^4; with 4 rows in flight per lane group (r2e25/26)
+// 127^4 reaches 5.73-5.76 TB/s (k_direct's plan: 4.58) but rows of 120-500 B
+// drop to 0.2-0.55x and the 0.5-16 KB rows of [n0, m, k] `0 2 1` to
+// 0.15-0.65x -- kept as an option, off by default
 static bool rows16_enabled() {
   static int v = -1;
   if (v < 0) {

@@ -31,7 +31,25 @@ def workload(name):
              "c4": configs.config4, "c5": configs.config5, "fig13": configs.fig13,
              "720-15": lambda: configs.sweep720(15), "720-16": lambda: configs.sweep720(16),
              "720-17": lambda: configs.sweep720(17)}
+    if name == "fmlrows":
+        return fml_rows()
     return table[name]()
+
+
+def fml_rows():
+    """FML rows that are not 16-byte multiples, 64-2048+ bytes long: [n0, m, k]
+    `0 2 1` (fp64 odd n0, fp32 n0 = 4j+-1), ~256 MB per tensor (k_direct vs k_rows)."""
+    from synth.configs import Case
+    out = []
+    shapes = [(8, n0) for n0 in (15, 31, 47, 63, 95, 127, 191, 255, 383, 511, 1023, 2047)] + \
+             [(4, n0) for n0 in (63, 127, 255, 511, 1023, 2047)]
+    for i, (s, n0) in enumerate(shapes):
+        m = max(3, int(round((256 * 2 ** 20 / (s * n0)) ** 0.5))) | 1
+        # all-odd extents: every row keeps its 16-byte phase (as 127^4)
+        out.append(Case(9000 + i, (n0, m, m + 2), (0, 2, 1), s, "fmlrows"))
+        if s == 8 and n0 in (127, 255, 1023):  # half the rows change phase
+            out.append(Case(9100 + i, (n0, m + 1, m + 2), (0, 2, 1), s, "fmlrows"))
+    return out
 
 
 _cudart = None
