@@ -212,6 +212,8 @@ def candidate_hints(d: dict) -> dict:
     """Hints that reproduce a candidate returned by plan_candidates()."""
     if d["kernel"] == "deint":
         return {"variant": 4}
+    if d["kernel"] == "blk":
+        return {"variant": 9}
     a, b = d["in_dim"], d["out_dim"]
     h = {"schema": d["schema"] if d["schema"] != "COPY" else "FML", "in_dim": a,
          "in_block": d["tile_extents"][a], "out_dim": b,

@@ -514,9 +514,9 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
                 : ci.kernel == KK_VEC   ? 7
                                         : 0;
     if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = ci.threads - 32;  // consumers
-    if (ci.kernel == KK_DEINT) {  // no slice parameters: the structure size fixes the slice
-      ttlg_plan_hints_init(&h);
-      h.variant = 4;
+    if (ci.kernel == KK_DEINT || ci.kernel == KK_BLK) {  // no slice parameters: the
+      ttlg_plan_hints_init(&h);                         // structure fixes the slice
+      h.variant = ci.kernel == KK_DEINT ? 4 : 9;
     }
     ttlg_plan_s *q = new (std::nothrow) ttlg_plan_s;
     if (!q) break;

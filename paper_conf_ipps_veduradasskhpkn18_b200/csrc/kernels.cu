@@ -1332,6 +1332,201 @@ __global__ void __launch_bounds__(256) k_inter(const __grid_constant__ TileParam
 }
 
 // ---------------------------------------------------------------------------
+// k_blk: transpositions whose leading input dims 0..c-1 map onto the leading
+// output positions (a closed prefix, {perm[0..c-1]} = {0..c-1}, c >= 2; e.g.
+// 16^6 `1 0 2 4 3 5`, 24^6 `1 0 2 4 3 5`): the tensor is a set of blocks of
+// Vb = n0 * ... * n(c-1) elements (<= 8 KB) that are contiguous in BOTH A and
+// B -- the inner permutation acts inside a block, the outer one moves whole
+// blocks (PAPER.md's OA schema with the slice = one closed block, Alg. 5
+// L948-1020, in block granularity).  One warp moves one block at a time:
+//   load:   the block's Cb chunks (WC bytes each), CPL per lane, coalesced
+//           (each warp instruction covers 32 consecutive chunks of A);
+//   stage:  into the warp's own shared-memory buffer, either every dim-0 row
+//           padded by RA elements or the chunk slots XOR-swizzled (slot =
+//           c ^ ((c >> blk_swz) & (128/WC - 1))) -- the planner's
+//           gather-conflict choice;
+//   gather: output chunk oc of the block = KC = WC/S consecutive output
+//           elements, read from their staging positions (a per-CTA table,
+//           16-bit positions) and written with ONE WC-byte store -- B's block
+//           is written contiguously (coalesced, 32 chunks per instruction).
+// The next block's loads are issued before the current block's gather, so a
+// block's load latency overlaps the previous block's stores.  Blocks are
+// enumerated in output order (warp w takes blocks w, w + W, ...: consecutive
+// warps write consecutive blocks of B); the A offset of a block comes from its
+// outer digits (mixed radix over the outer output dims), decoded 32 blocks at
+// a time, one per lane, and broadcast with a shuffle.
+// Parameters (TileParams): num_tiles = blocks; ng / gdiv / gsA = outer output
+// dims (extents, A strides); V = Vb; LA = Cb; LB / fd_LB = chunks per dim-0
+// row; RA = row padding (elements); smem_elems = staging elements per warp;
+// qk = KC; nj / j_div / j_sS = the inner output digits and their staging
+// strides; off_tabB = gather table, off_data = staging buffers.
+template <int WC>
+struct ChunkOf;
+template <>
+struct ChunkOf<4> {
+  static __device__ __forceinline__ unsigned int make(const uint32_t *w) { return w[0]; }
+};
+template <>
+struct ChunkOf<8> {
+  static __device__ __forceinline__ uint2 make(const uint32_t *w) { return make_uint2(w[0], w[1]); }
+};
+template <>
+struct ChunkOf<16> {
+  static __device__ __forceinline__ uint4 make(const uint32_t *w) {
+    return make_uint4(w[0], w[1], w[2], w[3]);
+  }
+};
+template <int S>
+__device__ __forceinline__ void lds_words(uint32_t a, uint32_t *w) {
+  if constexpr (S == 8) {
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(w[0]), "=r"(w[1]) : "r"(a));
+  } else {
+    asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(w[0]) : "r"(a));
+  }
+}
+template <int WC>
+__device__ __forceinline__ void sts_chunk(uint32_t a, const typename Vec<WC>::T &v) {
+  if constexpr (WC == 16) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};\n" ::"r"(a), "r"(v.x), "r"(v.y),
+                 "r"(v.z), "r"(v.w) : "memory");
+  } else if constexpr (WC == 8) {
+    asm volatile("st.shared.v2.u32 [%0], {%1, %2};\n" ::"r"(a), "r"(v.x), "r"(v.y) : "memory");
+  } else {
+    asm volatile("st.shared.u32 [%0], %1;\n" ::"r"(a), "r"(v) : "memory");
+  }
+}
+
+template <int S, int WC, int CPL>
+__global__ void __launch_bounds__(256, CPL >= 16 ? 2 : 3) k_blk(const __grid_constant__ TileParams P,
+                                             const __grid_constant__ BatchPtrs X) {
+  using TC = typename Vec<WC>::T;
+  constexpr int KC = WC / S;
+  constexpr int WPE = S / 4;
+  extern __shared__ __align__(16) unsigned char smem[];
+  const unsigned char *A = reinterpret_cast<const unsigned char *>(X.A[blockIdx.y]);
+  unsigned char *B = reinterpret_cast<unsigned char *>(X.B[blockIdx.y]);
+  uint16_t *tab = reinterpret_cast<uint16_t *>(smem + P.off_tabB);
+  const int Cb = P.LA;
+
+  pdl_trigger();
+  // gather table: output chunk oc -> the staging positions of its KC elements
+#pragma unroll 1
+  for (int j = threadIdx.x; j < Cb * KC; j += blockDim.x) {
+    uint32_t rem = (uint32_t)j;
+    int off = 0;
+    for (int k = 0; k < P.nj; k++) {
+      const uint32_t q = fdiv1(rem, P.j_div[k]);
+      off += (int)(rem - q * P.j_div[k].div) * P.j_sS[k];
+      rem = q;
+    }
+    if (P.blk_swz) {  // XOR-swizzled chunk slots (no row padding)
+      const int c = off / KC;
+      off = (c ^ ((c >> P.blk_swz) & (128 / WC - 1))) * KC + off % KC;
+    }
+    tab[j] = (uint16_t)off;
+  }
+  __syncthreads();
+  pdl_wait();
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, wpc = blockDim.x >> 5;
+  // NB blocks per warp iteration: >= 8 chunks per lane in flight (registers)
+  constexpr int NB = CPL <= 2 ? 4 : (CPL == 4 ? 2 : 1);
+  const uint32_t stg_blk = (uint32_t)(P.smem_elems * S);
+  const uint32_t stg = (uint32_t)__cvta_generic_to_shared(smem + P.off_data) +
+                       (uint32_t)warp * NB * stg_blk;
+  const uint32_t tabs = (uint32_t)__cvta_generic_to_shared(tab);
+  // staging byte offset of this lane's m-th chunk (the same in every block)
+  uint32_t spos[CPL];
+#pragma unroll
+  for (int m = 0; m < CPL; m++) {
+    const uint32_t ch = (uint32_t)(lane + 32 * m);
+    spos[m] = P.blk_swz ? (ch ^ ((ch >> P.blk_swz) & (128 / WC - 1))) * WC
+                        : (ch * KC + fdiv1(ch, P.fd_LB) * (uint32_t)P.RA) * S;
+  }
+  const uint64_t nb = P.num_tiles, stride = (uint64_t)gridDim.x * wpc;
+  const uint64_t q0 = (uint64_t)blockIdx.x * wpc + warp;
+  // A and B byte offsets of 32 consecutive blocks of this warp, one per lane
+  int64_t myA = 0, myB = 0;
+  uint64_t grp = ~0ull;
+  auto bases = [&](uint64_t k, int64_t &bA, int64_t &bB) {  // k-th block of this warp
+    if ((k >> 5) != grp) {
+      grp = k >> 5;
+      const uint64_t qq = q0 + ((grp << 5) + lane) * stride;
+      if (qq < nb) {
+        const TileCtx c = decode_tile(P, (uint32_t)qq);
+        myA = c.bA * S;
+        myB = c.bB * S;
+      }
+    }
+    bA = __shfl_sync(0xffffffffu, myA, (int)(k & 31));
+    bB = __shfl_sync(0xffffffffu, myB, (int)(k & 31));
+  };
+  TC v[NB][CPL];
+  auto load = [&](int j, int64_t bA) {
+    const TC *src = reinterpret_cast<const TC *>(A + bA);
+#pragma unroll
+    for (int m = 0; m < CPL; m++)
+      if (lane + 32 * m < Cb) v[j][m] = __ldcs(src + lane + 32 * m);
+  };
+  int64_t curB[NB], nxtB[NB];
+#pragma unroll
+  for (int j = 0; j < NB; j++) {
+    int64_t bA;
+    bases(j, bA, curB[j]);
+    if (q0 + j * stride < nb) load(j, bA);
+  }
+  uint64_t kg = 0;
+  for (uint64_t qg = q0; qg < nb; qg += NB * stride, kg++) {
+#pragma unroll
+    for (int j = 0; j < NB; j++)
+      if (qg + j * stride < nb) {
+#pragma unroll
+        for (int m = 0; m < CPL; m++)
+          if (lane + 32 * m < Cb) sts_chunk<WC>(stg + j * stg_blk + spos[m], v[j][m]);
+      }
+    __syncwarp();
+    // the next group's loads fly while this group is gathered and stored
+#pragma unroll
+    for (int j = 0; j < NB; j++) {
+      int64_t bA;
+      bases((kg + 1) * NB + j, bA, nxtB[j]);  // whole warp (shuffles) before the guard
+      if (qg + (NB + j) * stride < nb) load(j, bA);
+    }
+#pragma unroll
+    for (int j = 0; j < NB; j++) {
+      if (qg + j * stride >= nb) break;
+      TC *dst = reinterpret_cast<TC *>(B + curB[j]);
+      const uint32_t sb = stg + j * stg_blk;
+#pragma unroll
+      for (int m = 0; m < CPL; m++) {
+        const int oc = lane + 32 * m;
+        if (oc < Cb) {
+          uint32_t w[WC / 4], pk[(KC + 1) / 2];
+          // the KC 16-bit positions of chunk oc, packed (one shared load)
+          if constexpr (KC == 4) {
+            asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(pk[0]), "=r"(pk[1])
+                         : "r"(tabs + 8u * oc));
+          } else if constexpr (KC == 2) {
+            asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(pk[0]) : "r"(tabs + 4u * oc));
+          } else {
+            asm volatile("ld.shared.u16 %0, [%1];\n" : "=r"(pk[0]) : "r"(tabs + 2u * oc));
+          }
+#pragma unroll
+          for (int u = 0; u < KC; u++) {
+            const uint32_t pos = (pk[u >> 1] >> (16 * (u & 1))) & 0xffffu;
+            lds_words<S>(sb + pos * S, w + u * WPE);
+          }
+          __stcs(dst + oc, ChunkOf<WC>::make(w));
+        }
+      }
+    }
+    __syncwarp();
+#pragma unroll
+    for (int j = 0; j < NB; j++) curB[j] = nxtB[j];
+  }
+}
+
+// ---------------------------------------------------------------------------
 // k_bulk: the staged tile transposition (OD, Alg. 2; OA/FMS, Alg. 5
 // L948-1020 / Alg. 6) as a warp-specialised, persistent pipeline:
 //
@@ -1686,6 +1881,54 @@ static const void *quad_ptr(int W, int cb, int nj) {
   return cb == 16 ? quad_ptr_nj<4, 16>(nj) : quad_ptr_nj<4, 8>(nj);
 }
 
+template <int S, int WC>
+static const void *blk_ptr_c(int cpl) {
+  switch (cpl) {
+    case 2: return (const void *)k_blk<S, WC, 2>;
+    case 4: return (const void *)k_blk<S, WC, 4>;
+    case 8: return (const void *)k_blk<S, WC, 8>;
+    case 16: return (const void *)k_blk<S, WC, 16>;
+  }
+  return nullptr;
+}
+static const void *blk_ptr(int S, int WC, int cpl) {
+  if (S == 8) return WC == 16 ? blk_ptr_c<8, 16>(cpl) : (WC == 8 ? blk_ptr_c<8, 8>(cpl) : nullptr);
+  if (S == 4)
+    return WC == 16 ? blk_ptr_c<4, 16>(cpl)
+                    : (WC == 8 ? blk_ptr_c<4, 8>(cpl) : (WC == 4 ? blk_ptr_c<4, 4>(cpl) : nullptr));
+  return nullptr;
+}
+static int cpl_idx(int cpl) { return cpl == 2 ? 0 : (cpl == 4 ? 1 : (cpl == 8 ? 2 : 3)); }
+
+int blk_regs(int S, int WC, int cpl) {
+  // [S 4/8][WC 4/8/16][CPL 2/4/8/16], read once under the lock
+  static std::atomic<int> regs[2][3][4];
+  static std::once_flag once;
+  std::call_once(once, [] {
+    for (auto &a : regs)
+      for (auto &b : a)
+        for (auto &c : b) c.store(-1);
+  });
+  std::atomic<int> &slot = regs[S == 8][widx(WC)][cpl_idx(cpl)];
+  int r = slot.load(std::memory_order_acquire);
+  if (r >= 0) return r;
+  static std::mutex mu;
+  std::lock_guard<std::mutex> g(mu);
+  r = slot.load(std::memory_order_relaxed);
+  if (r < 0) {
+    cudaFuncAttributes attr;
+    const void *fn = blk_ptr(S, WC, cpl);
+    if (fn && cudaFuncGetAttributes(&attr, fn) == cudaSuccess) {
+      r = attr.numRegs;
+    } else {
+      cudaGetLastError();
+      r = 0;
+    }
+    slot.store(r, std::memory_order_release);
+  }
+  return r;
+}
+
 int kernel_regs(int kind, int W) {
   // read once per (kind, width) under the lock, then lock-free: the planner
   // asks for every scored candidate
@@ -1693,7 +1936,7 @@ int kernel_regs(int kind, int W) {
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
-                                             {{-1}, {-1}, {-1}}};
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
   if (r >= 0) return r;
@@ -1737,7 +1980,8 @@ static bool pdl_enabled() {
 ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *const *B,
                    void *stream) {
   if (n < 1 || n > kMaxBatch) return TTLG_ERR_INVALID_VALUE;
-  const void *fn = plan->kind == KK_QUAD
+  const void *fn = plan->kind == KK_BLK ? blk_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.blk_cpl)
+                   : plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
                        : (plan->kind == KK_BULKQ || plan->kind == KK_BULKG)
                              ? bulk_ptr(plan->W, plan->kind)

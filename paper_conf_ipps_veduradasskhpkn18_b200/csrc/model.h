@@ -55,5 +55,9 @@ constexpr double kSmallTraffic = 32.0 * 1024 * 1024;
 // factor x the one-pass ideal 2*N*s / HBM bandwidth -- measured on B200 at
 // the config-4 sizes, n0 = 2..5: 5.41-5.63 TB/s back to back (exp49)
 constexpr double kDeintFactor = 1.18;
+// k_blk (one streaming pass, one warp per closed leading block): the same
+// form, measured on B200 (r2e30, graph timing): 16^6 / 24^6 fp64 `1 0 ...`
+// 5.65-5.7 TB/s, 15^6 / 17^6 5.8-6.0 TB/s -> 1.10-1.16 x the ideal
+constexpr double kBlkFactor = 1.13;
 
 }  // namespace ttlg

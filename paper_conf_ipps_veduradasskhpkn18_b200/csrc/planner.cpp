@@ -1208,7 +1208,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // One slice geometry (Alg. 3's dimsIn/blockA, dimsOut/blockB) x every kernel
   // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
-    if (hv == 4) return;  // k_deint forced: no staged / direct candidates
+    if (hv == 4 || hv == 9) return;  // k_deint / k_blk forced: no staged / direct candidates
     const bool bulk = group == KK_BULKQ || group == KK_BULKG;
     if (bulk || group == KK_VEC) {
       if (forceW) return;  // element-width fallback plans: no 16-byte requirement
@@ -1536,6 +1536,188 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     make_deint(plan, &plan->info, deint_t);
     return TTLG_OK;
   }
+  // ---- k_blk: a closed leading block (dims 0..c-1 onto output positions
+  // 0..c-1, c >= 2) of <= 8 KB, contiguous in A and in B -- the outer
+  // permutation moves whole blocks, the inner one acts inside a block: one
+  // warp per block, chunk loads and gathered chunk stores (kernels.cu k_blk).
+  // Its time is the one-pass ideal times the factor measured for it on B200
+  // (kBlkFactor, model.h); like k_deint it competes with the ranked winner.
+  int cb = 0;  // closed prefix length
+  if (P.p[0] != 0 && P.W == P.esize) {
+    int mx = 0;
+    for (int k = 0; k < P.d; k++) {
+      mx = std::max(mx, (int)P.p[k]);
+      if (mx == k) {
+        cb = k + 1;
+        break;
+      }
+    }
+  }
+  int64_t Vb = 1;
+  for (int k = 0; k < cb; k++) Vb *= P.n[k];
+  int blk_wc = 0, blk_cpl = 0;
+  if (cb >= 2 && P.denseA >= cb - 1 && P.denseB >= cb - 1 &&
+      (hv == 0 || hv == 9) &&
+      (force_schema == TTLG_SCHEMA_AUTO || force_schema == TTLG_SCHEMA_OA) &&
+      !(hints && (hints->in_dim >= 0 || hints->in_block > 0 || hints->out_dim >= 0 ||
+                  hints->out_block > 0 || (hints->threads && hints->threads != 256)))) {
+    // widest chunk dividing the dim-0 row, the block and every outer stride
+    for (int wc = 16; wc >= s && !blk_wc; wc /= 2) {
+      if (forceW && wc != s) continue;  // element-width twin
+      bool ok = (P.n[0] * s) % wc == 0 && (Vb * s) % wc == 0;
+      for (int k = cb; ok && k < P.d; k++) ok = (P.sA[k] * s) % wc == 0 && (P.sB[k] * s) % wc == 0;
+      if (ok) blk_wc = wc;
+    }
+    const int64_t Cb = blk_wc ? Vb * s / blk_wc : 0;
+    const int need = (int)ceil_div(Cb, 32);
+    blk_cpl = need <= 2 ? 2 : (need <= 4 ? 4 : (need <= 8 ? 8 : (need <= 16 ? 16 : 0)));
+    // every lane busy (>= 32 chunks), 16-bit staging positions, the stage
+    // ring of 8 warps (worst-case row padding) within a CTA's shared memory
+    const int nbw = blk_cpl <= 2 ? 4 : (blk_cpl == 4 ? 2 : 1);
+    const int64_t worst = (Vb + Vb / P.n[0] * 8 * 2) * s * nbw * 8 + Cb * 8;
+    if (Cb < 32 || Vb * 2 > 65535 || N / Vb >= (1ll << 31) ||
+        worst > dev.smem_per_block_optin)
+      blk_cpl = 0;
+  }
+  const bool blk_ok = blk_cpl > 0;
+  const double blk_t = blk_ok ? kBlkFactor * 2.0 * (double)N * s / (dev.hbm_gbs * 1e9) : 1e300;
+  auto make_blk = [&](ttlg_plan_s *pl, ttlg_plan_info *info, double t) {
+    TileParams K;
+    memset(&K, 0, sizeof(K));
+    const int KC = blk_wc / s;
+    const int64_t Cb = Vb * s / blk_wc, rowc = P.n[0] / KC;
+    // outer dims in output order: block q = mixed radix over n[p[cb..d-1]]
+    K.ng = P.d - cb;
+    for (int g = 0; g < K.ng; g++) {
+      const int i = P.p[cb + g];
+      K.gdiv[g] = make_fastdiv((uint32_t)P.n[i]);
+      K.gsA[g] = P.sA[i];
+      K.gsB[g] = P.sB[i];
+    }
+    K.blkA_g = K.blkB_g = -1;
+    K.num_tiles = (uint32_t)(N / Vb);
+    K.V = (int32_t)Vb;
+    K.LA = (int32_t)Cb;
+    K.LB = (int32_t)rowc;
+    K.fd_LB = make_fastdiv((uint32_t)rowc);
+    K.qk = KC;
+    K.blk_cpl = blk_cpl;
+    K.tpc = 1;
+    // inner output digits (output order) and their staging strides for a
+    // dim-0 row padding of pad elements; the pad (a multiple of KC, so the
+    // staged chunks stay WC-aligned) minimises the first warp's gather
+    // wavefronts
+    K.nj = cb;
+    auto strides = [&](int pad, int32_t *sS) {
+      for (int k = 0; k < cb; k++) {
+        const int i = P.p[k];
+        int64_t st = i == 0 ? 1 : P.n[0] + pad;
+        for (int j = 1; j < i; j++) st *= P.n[j];
+        sS[k] = (int32_t)st;
+      }
+    };
+    // layouts: dim-0 row padding pad (swz = 0) or chunk slots XOR-swizzled
+    // by chunk-index bits [swz, swz + log2(128/WC)) (pad = 0); the gather of
+    // the first warp's first two chunk sets is simulated for each
+    const int mask = 128 / blk_wc - 1;
+    int lg = 0;
+    while ((1 << lg) <= mask) lg++;
+    auto gather_cost = [&](int pad, int swz) {
+      int32_t sS[TTLG_MAXD];
+      strides(pad, sS);
+      double c = 0;
+      for (int64_t m = 0; m < std::min<int64_t>(2, ceil_div(Cb, 32)); m++)
+        for (int u = 0; u < KC; u++) {
+          int64_t addr[32];
+          for (int l = 0; l < 32; l++) {
+            int64_t rem = (32 * m + l) % Cb * KC + u, off = 0;
+            for (int k = 0; k < cb; k++) {
+              const int64_t e = P.n[P.p[k]];
+              off += (rem % e) * sS[k];
+              rem /= e;
+            }
+            if (swz) {
+              const int64_t ch = off / KC;
+              off = (ch ^ ((ch >> swz) & mask)) * KC + off % KC;
+            }
+            addr[l] = off;
+          }
+          c += wavefront_ratio(addr, s);
+        }
+      return c;
+    };
+    int best_pad = 0, best_swz = 0;
+    double best_c = 1e300;
+    for (int pad = 0; pad <= 8 * KC; pad += KC) {
+      const double c = gather_cost(pad, 0);
+      if (c < best_c - 1e-9) {
+        best_c = c;
+        best_pad = pad;
+      }
+    }
+    // a swizzle permutes whole groups of 128 bytes; 16-byte chunks only
+    // (measured, r2e31: 8-byte chunk swizzles lose to padding on 15^6)
+    if (Cb % (mask + 1) == 0 && blk_wc == 16)
+      for (int swz = lg; swz <= lg + 6; swz++) {
+        const double c = gather_cost(0, swz);
+        if (c < best_c - 1e-9) {
+          best_c = c;
+          best_pad = 0;
+          best_swz = swz;
+        }
+      }
+    K.blk_swz = best_swz;
+    strides(best_pad, K.j_sS);
+    for (int k = 0; k < cb; k++) {
+      K.j_ext[k] = (int32_t)P.n[P.p[k]];
+      K.j_div[k] = make_fastdiv((uint32_t)P.n[P.p[k]]);
+    }
+    K.RA = best_pad;
+    const int64_t rows = Vb / P.n[0];
+    K.smem_elems = (int32_t)((Vb + rows * best_pad + KC - 1) / KC * KC);
+    K.smem_elems = (int32_t)(ceil_div((int64_t)K.smem_elems * s, 16) * 16 / s);
+    K.off_tabB = 0;
+    K.off_data = (int32_t)ceil_div(Cb * KC * 2, 16) * 16;
+    const int nbw = blk_cpl <= 2 ? 4 : (blk_cpl == 4 ? 2 : 1);  // blocks per warp iteration
+    K.smem_bytes = K.off_data + 8 * nbw * K.smem_elems * s;
+    Tile T;
+    T.a = cb - 1;
+    T.b = cb - 1;
+    T.ok = true;
+    for (int k = 0; k < P.d; k++) T.t[k] = k < cb ? P.n[k] : 1;
+    ModelInput mi;
+    memset(&mi, 0, sizeof(mi));
+    mi.kind = KK_BLK;
+    mi.schema = TTLG_SCHEMA_OA;
+    mi.W = s;
+    mi.N = N;
+    mi.threads = 256;
+    mi.occ = std::max(1, occupancy(dev, 256, K.smem_bytes, blk_regs(s, blk_wc, blk_cpl)));
+    mi.grid = (int)std::min<int64_t>(ceil_div(N / Vb, 8), (int64_t)dev.sms * mi.occ);
+    if (pl) {
+      pl->kind = KK_BLK;
+      pl->variant = 9;
+      pl->W = s;
+      pl->align = blk_wc;
+      pl->threads = 256;
+      pl->grid = mi.grid;
+      pl->nbytes = N * s;
+      pl->spanA = spanA * s;
+      pl->spanB = spanB * s;
+      pl->kp = K;
+    }
+    fill_info(*info, dt, rank, P, T, K, mi, TTLG_SCHEMA_OA, KK_BLK, t, ncand + 1);
+    info->access_bytes = blk_wc;
+    info->num_features = 0;
+  };
+  if (blk_ok && listing && sink->n < sink->max) make_blk(nullptr, &sink->out[sink->n++], blk_t);
+  if (hv == 9) {
+    if (!blk_ok) return TTLG_ERR_UNSUPPORTED;
+    if (sink && sink->shortlist && sink->n < sink->max)
+      make_blk(nullptr, &sink->out[sink->n++], blk_t);
+    make_blk(plan, &plan->info, blk_t);
+    return TTLG_OK;
+  }
   if (ntop == 0 && nv > 0) {  // only k_vec slices (cannot happen with the staged kernels present)
     for (int i = 0; i < nv; i++) {
       pool[i] = vpool[i];
@@ -1698,6 +1880,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // vs 4.8-5.3 TB/s for the staged kernels / k_quad)
   if (deint_ok && deint_t < win_t) {
     make_deint(plan, &plan->info, deint_t);
+    return TTLG_OK;
+  }
+  if (blk_ok && sink && sink->shortlist && sink->n < sink->max)
+    make_blk(nullptr, &sink->out[sink->n++], blk_t);
+  if (blk_ok && blk_t < win_t) {
+    make_blk(plan, &plan->info, blk_t);
     return TTLG_OK;
   }
   const Entry &B = *Bp;

@@ -59,7 +59,9 @@ enum KernelKind : int32_t {
                   // stores gathered from K element reads (k_vec)
   KK_PHASE = 8,   // k_tile's slice with 16-byte loads at any row alignment (per-row phase
                   // in shared memory) and element stores (k_phase)
-  KK_NUM = 9,
+  KK_BLK = 9,     // closed leading block (<= 8 KB, contiguous in A and B): one warp per
+                  // block, WC-byte chunk loads and gathered WC-byte stores (k_blk)
+  KK_NUM = 10,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -131,6 +133,8 @@ struct TileParams {
   int32_t rb_sP[TTLG_MAXD];
   int32_t j_sP[TTLG_MAXD];
   int64_t a_elems;
+  int32_t blk_cpl;  // k_blk: chunks per lane (template instance)
+  int32_t blk_swz;  // k_blk: chunk-slot XOR swizzle shift (0: row padding RA instead)
 };
 
 // Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;
@@ -233,4 +237,5 @@ const DeviceProfile &device_profile(int device);
 ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *const *B,
                    void *stream);
 int kernel_regs(int kind, int W);  // registers per thread of a kernel variant (cached; 0 if unknown)
+int blk_regs(int S, int WC, int cpl);  // the same for a k_blk instance
 }  // namespace ttlg

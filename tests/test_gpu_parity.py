@@ -653,3 +653,62 @@ def test_phase_forced_odd_extents(eb):
                 continue
             got, exp, _ = _run(ext, perm, eb, 1500, plan_kwargs={"variant": 8, **tiles}, canary=32)
             _assert_equal(got, exp, f"phase {ext} {perm} {tiles}")
+
+
+def _blk_cases():
+    """Closed leading blocks: 2-D and 3-D inner perms, 16 / 8 / 4-byte chunks,
+    1-16 chunks per lane, outer perms of every shape, a single block, blocks
+    whose outer strides are odd element counts."""
+    return [
+        ([16, 16, 6, 5, 7], [1, 0, 2, 4, 3]),
+        ([16, 16, 16, 16, 16, 16], [1, 0, 3, 5, 2, 4]),
+        ([24, 24, 5, 7, 3], [1, 0, 4, 3, 2]),
+        ([15, 15, 9, 11], [1, 0, 3, 2]),
+        ([17, 17, 4, 9], [1, 0, 2, 3]),
+        ([8, 8, 8, 33], [2, 1, 0, 3]),
+        ([8, 4, 8, 20, 3], [2, 0, 1, 4, 3]),
+        ([4, 8, 16, 2, 9], [1, 2, 0, 4, 3]),
+        ([32, 32, 7, 3], [1, 0, 3, 2]),
+        ([6, 12, 11, 13], [1, 0, 3, 2]),
+        ([45, 45, 8], [1, 0, 2]),
+        ([16, 16], [1, 0]),
+        ([20, 12, 3, 7, 2], [1, 0, 4, 2, 3]),
+    ]
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+@pytest.mark.parametrize("ext,perm", _blk_cases(), ids=lambda v: "x".join(map(str, v)))
+def test_blk_forced(ext, perm, eb):
+    """k_blk (one warp per closed leading block, chunk loads, gathered chunk
+    stores, padded per-warp staging) forced, against the oracle; also on a
+    misaligned-by-one-element view (its element-width twin)."""
+    try:
+        ttlg.plan(_dt(eb), ext, perm, variant=9)
+    except ttlg.TtlgError:
+        pytest.skip("k_blk not applicable (block > 8 KB or < 32 chunks)")
+    got, exp, info = _run(ext, perm, eb, 1700 + len(ext), plan_kwargs={"variant": 9}, canary=64)
+    assert info["kernel"] == "blk"
+    _assert_equal(got, exp, f"blk {ext} {perm} {info}")
+    n = int(np.prod(ext))
+    A = gen_tensor_torch(1799, n + 1, eb, device=DEV)
+    B = torch.zeros(n + 3, dtype=A.dtype, device=DEV)
+    p = ttlg.plan(_dt(eb), ext, perm, variant=9)
+    p.execute(A[1:].data_ptr(), B[3:].data_ptr(), torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    _assert_equal(_bits(B[3:]), oracle.transpose(_bits(A[1:n + 1]), ext, perm),
+                  f"blk misaligned {ext} {perm}")
+
+
+def test_blk_batch():
+    """k_blk through ttlg_execute_batch (grid.y); strided sub-boxes:
+    tests/test_strided.py variant 9."""
+    ext, perm = [16, 16, 5, 9], [1, 0, 3, 2]
+    n = int(np.prod(ext))
+    p = ttlg.plan("f64", ext, perm, variant=9)
+    As = [gen_tensor_torch(1800 + i, n, 8, device=DEV) for i in range(3)]
+    Bs = [torch.empty_like(a) for a in As]
+    p.execute_batch([a.data_ptr() for a in As], [b.data_ptr() for b in Bs],
+                    torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    for a, b in zip(As, Bs):
+        _assert_equal(_bits(b), oracle.transpose(_bits(a), ext, perm), "blk batch")

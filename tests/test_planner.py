@@ -213,7 +213,7 @@ def test_plan_candidates_every_config_case():
             assert cands, c.label()
             kinds = {d["kernel"] for d in cands}
             # k_bulk only when forced or TTLG_BULK=1
-            assert kinds <= {"direct", "tile", "pipe", "quad", "deint", "vec"}
+            assert kinds <= {"direct", "tile", "pipe", "quad", "deint", "vec", "blk"}
             for d in cands:
                 if d["kernel"] == "vec":   # every listed k_vec slice plans as itself
                     assert d["access_bytes"] in (4, 8)
@@ -257,8 +257,9 @@ def test_bench_reference_arm_contract():
 def test_deep_tiles_only_for_closed_leading_blocks():
     """Input runs one dim past 4 KB (k_pipe only) are enumerated only when the
     leading input block is also the leading output block (1 0 2 4 3 5 family)."""
-    d = ttlg.plan("f64", [24] * 6, [1, 0, 2, 4, 3, 5]).describe()
-    assert d["kernel"] == "pipe" and d["in_dim"] == 2 and d["tile_extents"][2] > 1
+    cands = ttlg.plan_candidates("f64", [24] * 6, [1, 0, 2, 4, 3, 5])
+    assert any(c["kernel"] == "pipe" and c["in_dim"] == 2 and c["tile_extents"][2] > 1
+               for c in cands)
     # not closed (perm[0..1] = 2 0): no deep candidate may appear
     for c in ttlg.plan_candidates("f64", [16, 4, 16, 20, 16, 80], [2, 0, 4, 1, 5, 3]):
         fe, te = c["fused_extents"], c["tile_extents"]
@@ -310,3 +311,35 @@ def test_execute_batch_validation_without_gpu():
     assert e.value.code == 3                    # valid arguments, no device here
     with pytest.raises(ValueError):
         p.execute_batch([1 << 20], [])
+
+
+def test_blk_applicability():
+    """k_blk needs a closed leading block ({perm[0..c-1]} = {0..c-1}, c >= 2)
+    of 32 chunks .. 8 KB, contiguous in both tensors; the chunk width divides
+    the dim-0 row, the block and every outer stride."""
+    cases = [  # (dtype, extents, perm, applies, chunk bytes)
+        ("f64", [16] * 6, [1, 0, 2, 4, 3, 5], True, 16),
+        ("f64", [24] * 6, [1, 0, 5, 4, 3, 2], True, 16),
+        ("f64", [15] * 6, [1, 0, 2, 4, 3, 5], True, 8),   # odd rows: 8-byte chunks
+        ("f32", [15, 15, 40], [1, 0, 2], True, 4),
+        ("f64", [8, 8, 8, 64], [2, 1, 0, 3], True, 16),   # 3-D inner permutation
+        ("f64", [80, 16, 80, 256], [1, 0, 3, 2], False, 0),  # 10 KB block
+        ("f64", [16] * 6, [2, 0, 4, 1, 5, 3], False, 0),    # not closed before dim 5
+        ("f64", [16] * 6, [0, 2, 1, 3, 4, 5], False, 0),    # matching FVI (FML)
+        ("f64", [4, 4, 64], [1, 0, 2], False, 0),           # 16 chunks: lanes idle
+    ]
+    for dt, ext, perm, ok, wc in cases:
+        if ok:
+            d = ttlg.plan(dt, ext, perm, variant=9).describe()
+            assert d["kernel"] == "blk" and d["access_bytes"] == wc, (ext, perm, d)
+            assert d["schema"] == "OA" and d["threads"] == 256
+        else:
+            with pytest.raises(ttlg.TtlgError) as e:
+                ttlg.plan(dt, ext, perm, variant=9)
+            assert e.value.code == 7
+    # slice hints rule it out; the element-width twin keeps it at element width
+    with pytest.raises(ttlg.TtlgError):
+        ttlg.plan("f64", [16] * 6, [1, 0, 2, 4, 3, 5], variant=9, in_dim=2, in_block=4)
+    d = ttlg.plan("f64", [16] * 6, [1, 0, 2, 4, 3, 5], variant=9,
+                  access_bytes=8).describe()
+    assert d["kernel"] == "blk" and d["access_bytes"] == 8

@@ -59,6 +59,9 @@ STRIDED_CASES = [
     ([4, 33, 17], [0, 2, 1], [1, 5, 5 * 34], [1, 6, 6 * 17]),       # matching FVI, odd strides
     ([8, 6, 5, 7, 2], [1, 4, 0, 3, 2], [1, 9, 9 * 6, 9 * 6 * 5, 9 * 6 * 5 * 8], None),
     ([64, 3, 40], [0, 1, 2], [1, 70, 70 * 4], [1, 64, 64 * 3 * 2]),  # identity with gaps
+    # closed 16 x 16 leading block (k_blk) inside padded outer strides
+    ([16, 16, 5, 6], [1, 0, 3, 2], [1, 16, 16 * 16 * 2, 16 * 16 * 2 * 7], [1, 16, 16 * 16 * 8,
+                                                                         16 * 16 * 8 * 6]),
 ]
 
 
@@ -192,7 +195,7 @@ def _torch_bits(t):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("variant", [None, 1, 2, 3])
+@pytest.mark.parametrize("variant", [None, 1, 2, 3, 9])
 @pytest.mark.parametrize("eb", [4, 8])
 @pytest.mark.parametrize("case", STRIDED_CASES, ids=lambda c: "x".join(map(str, c[0])) + "-" +
                          "".join(map(str, c[1])))

@@ -36,7 +36,11 @@ def main():
         ([8, 30, 50], [0, 2, 1], 4, {"variant": 6}),
         ([256, 24, 6], [1, 0, 2], 8, {"variant": 5, "in_dim": 0, "in_block": 256,
                                       "out_dim": 0, "out_block": 24}),  # TMA rows (2 KB)
-        ([24, 24, 12, 4, 3, 2], [1, 0, 2, 4, 3, 5], 8, {}),   # deep k_pipe tiles
+        ([24, 24, 12, 4, 3, 2], [1, 0, 2, 4, 3, 5], 8, {"variant": 2}),  # deep k_pipe tiles
+        ([16, 16, 5, 7], [1, 0, 3, 2], 8, {"variant": 9}),   # k_blk, 16-byte chunks
+        ([15, 15, 6, 5], [1, 0, 3, 2], 8, {"variant": 9}),   # k_blk, 8-byte chunks
+        ([8, 8, 8, 9], [2, 1, 0, 3], 4, {"variant": 9}),     # k_blk, 3-D inner perm
+        ([24, 24, 12, 4, 3, 2], [1, 0, 2, 4, 3, 5], 8, {}),  # auto (k_blk)
     ]
     for ext, perm, eb, hints in cases:
         n = 1
