@@ -104,10 +104,18 @@ typedef struct {
                                             cp.async loads, 16-byte stores gathered from
                                             16/s element reads); 5-7 need every A-row
                                             (6, 7: and B-row) 16-byte aligned and whole
-                                            16-byte chunks, else TTLG_ERR_UNSUPPORTED.
-                                            The automatic choice considers 0-4 and 7
-                                            (env TTLG_VEC=0 drops 7; TTLG_BULK=1 adds
-                                            5, 6)                                          */
+                                            16-byte chunks, else TTLG_ERR_UNSUPPORTED;
+                                            8 = k_phase (k_tile's slice with 16-byte
+                                            loads at any row alignment); 9 = k_blk (the
+                                            fused perm's leading dims 0..c-1, c >= 2,
+                                            map onto output positions 0..c-1 and form a
+                                            block of 32 chunks .. 8 KB contiguous in A
+                                            and B: one warp per block, chunk loads and
+                                            gathered chunk stores), else
+                                            TTLG_ERR_UNSUPPORTED.  The automatic choice
+                                            considers 0-4, 7 and 9 (env TTLG_VEC=0 drops
+                                            7; TTLG_BULK=1 adds 5, 6; TTLG_PHASE=1 adds
+                                            8)                                             */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */
@@ -132,7 +140,8 @@ typedef struct {
   int32_t kernel;                         /* 0 k_direct (FML/COPY), 1 k_tile, 2 k_pipe,
                                              3 k_quad, 4 k_deint / k_inter, 5 k_bulk
                                              (quad consumers), 6 k_bulk (gather
-                                             consumers), 7 k_vec                         */
+                                             consumers), 7 k_vec, 8 k_phase, 9 k_blk
+                                             (closed leading block, one warp per block)  */
   int32_t occupancy;                      /* resident CTAs per SM assumed by the model   */
   int32_t num_features;                   /* model feature vector (§V features, B200)    */
   double features[12];

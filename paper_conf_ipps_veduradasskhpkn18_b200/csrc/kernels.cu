@@ -35,6 +35,9 @@
 //            drain with k_quad's transposes or k_vec's gathers.
 //  k_deint / k_inter (OA with a tiny FVI: AoS <-> SoA): 16-byte accesses
 //            both ways through per-warp swizzled staging buffers.
+//  k_blk     (OA with a closed leading block <= 8 KB, e.g. 16^6 `1 0 2 ...`):
+//            one warp per block, chunk loads, per-warp staging, gathered
+//            chunk stores in output order.
 //
 // Every staged CTA builds its row tables in shared memory (the paper's
 // texture-mapped offset arrays, L737-745) and decodes its tile index with

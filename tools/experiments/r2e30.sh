@@ -1,5 +1,5 @@
 #!/bin/bash
-# round 2, call 31: k_blk with XOR-swizzled staging (gather-conflict search over padding and swizzles)
+# round 2, call 30: k_blk with NB blocks per warp iteration (>= 8 chunks per lane in flight, registers)
 O=gpurun_out/r2e30
 mkdir -p $O
 python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
