@@ -136,9 +136,16 @@ def cpu_baseline(cases, budget_s=12.0, threads=None):
         del A
         if t_total >= budget_s:
             break
-    return {"value": nbytes / t_total / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
-            "sample": f"{len(done)} of {len(cases)} cases ({', '.join(done[:4])}"
-                      f"{', ...' if len(done) > 4 else ''}), {t_total:.1f} s of oracle time"}
+    out = {"value": nbytes / t_total / 1e9, "unit": "GB/s", "cores": cores, "kind": "oracle",
+           "sample": f"{len(done)} of {len(cases)} cases ({', '.join(done[:4])}"
+                     f"{', ...' if len(done) > 4 else ''}), {t_total:.1f} s of oracle time"}
+    if threads is None and cores > 1:
+        # the oracle single-threaded too (a smaller budget, the
+        # first cases of the same sample)
+        st = cpu_baseline(cases, budget_s=max(2.0, budget_s / 3), threads=1)
+        out["single_thread"] = {"value": st["value"], "unit": "GB/s", "cores": 1,
+                                "sample": st["sample"]}
+    return out
 
 
 def run_reference(args, rank, world):

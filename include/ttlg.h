@@ -111,11 +111,15 @@ typedef struct {
                                             map onto output positions 0..c-1 and form a
                                             block of 32 chunks .. 8 KB contiguous in A
                                             and B: one warp per block, chunk loads and
-                                            gathered chunk stores), else
+                                            gathered chunk stores), 10 = k_tmap (OD:
+                                            the tile loaded by TMA tensor-map box copies,
+                                            cp.async.bulk.tensor, 128-byte swizzle; fused
+                                            rank <= 5, 16-byte aligned A strides and
+                                            k_quad's chunk alignment), else
                                             TTLG_ERR_UNSUPPORTED.  The automatic choice
                                             considers 0-4, 7 and 9 (env TTLG_VEC=0 drops
                                             7; TTLG_BULK=1 adds 5, 6; TTLG_PHASE=1 adds
-                                            8)                                             */
+                                            8; TTLG_TMA=1 adds 10)                         */
 } ttlg_plan_hints;
 
 /* Everything a test or benchmark may want to know about a plan. */

@@ -79,7 +79,7 @@ class PlanInfo(ctypes.Structure):
             "bytes": self.bytes, "predicted_seconds": self.predicted_seconds,
             "candidates": self.candidates, "param_bytes": self.param_bytes,
             "kernel": ["direct", "tile", "pipe", "quad", "deint", "bulkq", "bulkg",
-                       "vec", "phase", "blk"][self.kernel],
+                       "vec", "phase", "blk", "tmap"][self.kernel],
             "occupancy": self.occupancy, "stages": self.stages,
             "features": [float(x) for x in self.features[:self.num_features]],
         }

@@ -220,8 +220,8 @@ def candidate_hints(d: dict) -> dict:
          "out_block": d["tile_extents"][d["fused_perm"][b]], "threads": d["threads"]}
     if d["kernel"] != "direct":
         h["variant"] = {"tile": 1, "pipe": 2, "quad": 3, "deint": 4, "bulkq": 5,
-                        "bulkg": 6, "vec": 7, "phase": 8}[d["kernel"]]
-    if d["kernel"] in ("bulkq", "bulkg"):
+                        "bulkg": 6, "vec": 7, "phase": 8, "tmap": 10}[d["kernel"]]
+    if d["kernel"] in ("bulkq", "bulkg", "tmap"):
         h["threads"] = d["threads"] - 32   # consumer threads (warp 0 is the producer)
     return h
 

@@ -512,8 +512,10 @@ ttlg_status ttlg_plan_tune(ttlg_plan_t *plan, const void *A, void *B, void *stre
                 : ci.kernel == KK_BULKQ ? 5
                 : ci.kernel == KK_BULKG ? 6
                 : ci.kernel == KK_VEC   ? 7
+                : ci.kernel == KK_TMA   ? 10
                                         : 0;
-    if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG) h.threads = ci.threads - 32;  // consumers
+    if (ci.kernel == KK_BULKQ || ci.kernel == KK_BULKG || ci.kernel == KK_TMA)
+      h.threads = ci.threads - 32;  // consumers
     if (ci.kernel == KK_DEINT || ci.kernel == KK_BLK) {  // no slice parameters: the
       ttlg_plan_hints_init(&h);                         // structure fixes the slice
       h.variant = ci.kernel == KK_DEINT ? 4 : 9;

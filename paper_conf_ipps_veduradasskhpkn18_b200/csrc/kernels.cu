@@ -42,6 +42,8 @@
 // Every staged CTA builds its row tables in shared memory (the paper's
 // texture-mapped offset arrays, L737-745) and decodes its tile index with
 // fast-divmod (the paper's decode/compute_base, L725-737).
+#include <cuda.h>  // CUtensorMap and its enums (the encoder is fetched at run time)
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 
 #include <atomic>
@@ -1800,6 +1802,200 @@ __global__ void __launch_bounds__(544, 1) k_bulk(const __grid_constant__ TilePar
   }
 }
 
+// ---------------------------------------------------------------------------
+// k_tmap: k_bulk's warp-specialised ring with the A side moved by the Tensor
+// Memory Accelerator's TILED mode -- the north star's "TMA tiled tensor-map
+// loads" (VERDICT r1 "Next round" 10).  The OD tile (k_quad's slice with
+// 16-byte chunks) is a box of a CUtensorMap over A's fused dims in map order
+// (input-run dims 0..a, output-run dims in output order, the rest; rank <=
+// 5; encoded per launch with the operand's address, launch()).  Lane 0 of
+// warp 0 waits for a free stage (mbarrier empty[s]), arms full[s] with the
+// box bytes and issues ONE cp.async.bulk.tensor (SASS UTMALDG) per panel --
+// no per-row or per-chunk load instructions, the hardware walks the box and
+// zero-fills past the tensor's edge (partial tiles).  The box lands dense
+// with the 128-byte swizzle (16-byte slot bits 4-6 XOR address bits 7-9, per
+// 1024-byte atom), which spreads the consumers' column reads -- 8 output
+// positions at one input position, rows pw <= 128 bytes apart -- over all
+// banks, the job the padded layouts of the other kernels do by hand.
+// Consumers: as k_bulk MODE 0 (K x K shuffle transposes, 16-byte stores) with
+// the shared-memory address of chunk (input position x, output position j)
+// = swizzle(panel(x) * pbytes + (x * S mod pw) + j * pw).
+struct __align__(64) TmaMaps {
+  CUtensorMap m[kMaxBatch];
+};
+
+template <int R>
+__device__ __forceinline__ void tma_box_g2s(uint32_t dst, const CUtensorMap *map, const int *c,
+                                            uint32_t bar) {
+  const uint64_t mp = reinterpret_cast<uint64_t>(map);
+  if constexpr (R == 1)
+    asm volatile("cp.async.bulk.tensor.1d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                 " [%0], [%1, {%2}], [%3];\n" ::"r"(dst), "l"(mp), "r"(c[0]), "r"(bar) : "memory");
+  else if constexpr (R == 2)
+    asm volatile("cp.async.bulk.tensor.2d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                 " [%0], [%1, {%2, %3}], [%4];\n" ::"r"(dst), "l"(mp), "r"(c[0]), "r"(c[1]),
+                 "r"(bar) : "memory");
+  else if constexpr (R == 3)
+    asm volatile("cp.async.bulk.tensor.3d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                 " [%0], [%1, {%2, %3, %4}], [%5];\n" ::"r"(dst), "l"(mp), "r"(c[0]), "r"(c[1]),
+                 "r"(c[2]), "r"(bar) : "memory");
+  else if constexpr (R == 4)
+    asm volatile("cp.async.bulk.tensor.4d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                 " [%0], [%1, {%2, %3, %4, %5}], [%6];\n" ::"r"(dst), "l"(mp), "r"(c[0]),
+                 "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(bar) : "memory");
+  else
+    asm volatile("cp.async.bulk.tensor.5d.shared::cluster.global.tile.mbarrier::complete_tx::bytes"
+                 " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];\n" ::"r"(dst), "l"(mp), "r"(c[0]),
+                 "r"(c[1]), "r"(c[2]), "r"(c[3]), "r"(c[4]), "r"(bar) : "memory");
+}
+
+template <int S, int R>
+__global__ void __launch_bounds__(544, 1) k_tmap(const __grid_constant__ TileParams P,
+                                                 const __grid_constant__ BatchPtrs X,
+                                                 const __grid_constant__ TmaMaps M) {
+  constexpr int K = 16 / S;
+  constexpr int LGK = K == 4 ? 2 : 1;
+  using C = typename Chunk<16>::T;
+  unsigned char *B = reinterpret_cast<unsigned char *>(X.B[blockIdx.y]);
+  extern __shared__ __align__(128) unsigned char smem[];
+  const uint32_t s0 = (uint32_t)__cvta_generic_to_shared(smem);
+  const uint32_t s_tabB = s0 + P.off_tabB, s_digA = s0 + P.off_digA;
+  const uint32_t s_bar = s0 + P.off_bar;
+  const uint32_t s_data = (s0 + P.off_data + 1023u) & ~1023u;  // swizzle atoms
+  CtxS *ctx = reinterpret_cast<CtxS *>(smem + P.off_ctx);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int NS = P.nstage, NC = (int)(blockDim.x >> 5) - 1;  // consumer warps
+  auto full_bar = [&](int st) { return s_bar + 16u * st; };
+  auto empty_bar = [&](int st) { return s_bar + 16u * st + 8u; };
+  const int pw = P.tm_pw, pbytes = P.tm_pbytes;
+
+  if (tid == 0) {
+    asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&M.m[blockIdx.y]))
+                 : "memory");
+    for (int st = 0; st < NS; st++) {
+      mbar_init(full_bar(st), 1);
+      mbar_init(empty_bar(st), NC);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  // B-row table: (global offset in B, dense input-run byte offset x * S ->
+  // the panel layout), blocked-digit table for partial tiles
+  build_rows(P.RB, P.nrb, P.rb_div, P.rb_sG, P.rb_sS, P.rb_blk,
+             reinterpret_cast<int2 *>(smem + P.off_tabB),
+             reinterpret_cast<int *>(smem + P.off_digA), S);
+  __syncthreads();
+  if (P.tm_np > 1) {
+    int2 *tb = reinterpret_cast<int2 *>(smem + P.off_tabB);
+    for (int i = tid; i < P.RB; i += blockDim.x) {
+      const int y = tb[i].y;
+      tb[i].y = (y / pw) * pbytes + (y % pw);
+    }
+  }
+  __syncthreads();
+
+  if (warp == 0) {
+    // ---- producer: one elected lane, one TMA box per panel per tile
+    if (lane == 0) {
+      const CUtensorMap *map = &M.m[blockIdx.y];
+      int st = 0;
+      uint32_t ph = 0;
+      for (uint32_t tile = blockIdx.x, k = 0; tile < P.num_tiles; tile += gridDim.x, k++) {
+        if (k >= (uint32_t)NS) mbar_wait(empty_bar(st), ph ^ 1u);
+        const TileCtx c = decode_tile(P, tile);
+        ctx[st].bA = c.bA;
+        ctx[st].bB = c.bB;
+        ctx[st].limA = c.limA;
+        ctx[st].limB = c.limB;
+        int co[5] = {0, 0, 0, 0, 0};
+        uint32_t rem = tile;
+#pragma unroll
+        for (int g = 0; g < TTLG_MAXD; g++) {
+          if (g < P.ng) {
+            const uint32_t q = fdiv(rem, P.gdiv[g]);
+            const int cg = (int)(rem - q * P.gdiv[g].div);
+            rem = q;
+#pragma unroll
+            for (int m = 0; m < 5; m++)
+              if (m == P.tm_gmap[g]) co[m] = cg * P.tm_gt[g];
+          }
+        }
+        mbar_expect_tx(full_bar(st), (uint32_t)(P.tm_np * pbytes));
+        const uint32_t dst = s_data + (uint32_t)st * P.stage_bytes;
+        for (int p = 0; p < P.tm_np; p++) {
+          int cp[5] = {co[0], co[1], co[2], co[3], co[4]};
+#pragma unroll
+          for (int m = 0; m < 5; m++)
+            if (m == P.tm_adim) cp[m] += p * P.tm_pa;
+          tma_box_g2s<R>(dst + (uint32_t)(p * pbytes), map, cp, full_bar(st));
+        }
+        if (++st == NS) {
+          st = 0;
+          ph ^= 1u;
+        }
+      }
+    }
+    return;
+  }
+
+  // ---- consumers (k_bulk MODE 0 on the swizzled panel layout)
+  const int ct = tid - 32, LB = P.LB, RB = P.RB;
+  const int m0 = (int)fdiv1(ct, P.fd_LB), j0 = ct - m0 * LB, rs = P.rsB;
+  const int RBq = RB / K;
+  const int nB = (m0 < rs && m0 < RBq) ? (int)fdiv1(RBq - 1 - m0, P.fd_rsB) + 1 : 0;
+  const uint32_t jc = (uint32_t)((j0 < LB ? j0 : 0) * pw);
+  const int q = j0 & (K - 1);
+  const int nBw = __reduce_max_sync(0xffffffffu, nB);
+  int st = 0;
+  uint32_t ph = 0;
+  for (uint32_t tile = blockIdx.x; tile < P.num_tiles; tile += gridDim.x) {
+    mbar_wait(full_bar(st), ph);
+    TileCtx c;
+    c.bA = ctx[st].bA;
+    c.bB = ctx[st].bB;
+    c.limA = ctx[st].limA;
+    c.limB = ctx[st].limB;
+    const bool full = (c.limA == P.blkA_t) && (c.limB == P.blkB_t);
+    const int lim = full ? LB : P.LBunit * c.limB;
+    const uint32_t sbuf = s_data + (uint32_t)st * P.stage_bytes;
+    int m = m0;
+#pragma unroll 4
+    for (int k = 0; k < nBw; k++) {
+      const bool act = k < nB;
+      const int row = K * (act ? m : 0) + q;  // own B-row x+q after the transpose
+      const int2 t = lds_int2(s_tabB + 8 * row);
+      const bool rok = act && j0 < LB && (full || lds_int(s_digA + 4 * row) < c.limA);
+      const uint32_t o = (uint32_t)(t.y - q * S) + jc;  // chunk x..x+K-1 at position j0
+      C v = lds_T<C>(sbuf + (o ^ ((o >> 3) & 0x70u)));
+      quad_transpose<S, 16>(v, q);
+      const int jb = j0 - q;
+      C *dst = reinterpret_cast<C *>(B + (c.bB + jb) * S);
+      stcs_p(wadd(dst, (uint32_t)t.x >> LGK), v, rok && (full || jb < lim));
+      m += rs;
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(empty_bar(st));
+    if (++st == NS) {
+      st = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
+template <int S>
+static const void *tmap_ptr_s(int rank) {
+  switch (rank) {
+    case 1: return (const void *)k_tmap<S, 1>;
+    case 2: return (const void *)k_tmap<S, 2>;
+    case 3: return (const void *)k_tmap<S, 3>;
+    case 4: return (const void *)k_tmap<S, 4>;
+    case 5: return (const void *)k_tmap<S, 5>;
+  }
+  return nullptr;
+}
+static const void *tmap_ptr(int W, int rank) {
+  return W == 8 ? tmap_ptr_s<8>(rank) : (W == 4 ? tmap_ptr_s<4>(rank) : nullptr);
+}
+
 template <int S>
 static const void *bulk_ptr_s(int mode) {
   return mode == 0 ? (const void *)k_bulk<S, 0> : (const void *)k_bulk<S, 1>;
@@ -1939,7 +2135,8 @@ int kernel_regs(int kind, int W) {
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
                                              {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
-                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}}};
+                                             {{-1}, {-1}, {-1}}, {{-1}, {-1}, {-1}},
+                                             {{-1}, {-1}, {-1}}};
   std::atomic<int> &slot = regs[kind][widx(W)];
   int r = slot.load(std::memory_order_acquire);
   if (r >= 0) return r;
@@ -1949,6 +2146,7 @@ int kernel_regs(int kind, int W) {
   if (r < 0) {
     cudaFuncAttributes attr;
     const void *fn = kind == KK_QUAD    ? quad_ptr(W, 16, 1)
+                     : kind == KK_TMA   ? tmap_ptr(W == 8 ? 8 : 4, 2)
                      : kind == KK_DEINT ? deint_ptr(W == 8 ? 8 : 4, 4)
                      : (kind == KK_BULKQ || kind == KK_BULKG)
                          ? bulk_ptr(W, kind)
@@ -1964,6 +2162,38 @@ int kernel_regs(int kind, int W) {
     slot.store(r, std::memory_order_release);
   }
   return r;
+}
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda
+// link): k_tmap's box over A in map order, 128-byte swizzle, zero fill
+static ttlg_status encode_tmap(CUtensorMap *m, const TileParams &kp, int W, const void *A) {
+  static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *fp = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fp, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      enc = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fp);
+    else
+      cudaGetLastError();
+  });
+  if (!enc) return TTLG_ERR_CUDA;
+  const int r = kp.tm_rank;
+  cuuint64_t dim[5], str[4];
+  cuuint32_t box[5], es[5];
+  for (int m = 0; m < r; m++) {
+    dim[m] = (cuuint64_t)kp.tm_dim[m];
+    box[m] = (cuuint32_t)kp.tm_box[m];
+    es[m] = 1;
+    if (m > 0) str[m - 1] = (cuuint64_t)kp.tm_stride[m];
+  }
+  const CUresult e = enc(m, W == 8 ? CU_TENSOR_MAP_DATA_TYPE_UINT64 : CU_TENSOR_MAP_DATA_TYPE_UINT32,
+                         (cuuint32_t)r, const_cast<void *>(A), dim, str, box, es,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return e == CUDA_SUCCESS ? TTLG_OK : TTLG_ERR_CUDA;
 }
 
 // Programmatic dependent launch is opt-in (TTLG_PDL=1): measured on B200
@@ -1983,7 +2213,8 @@ static bool pdl_enabled() {
 ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *const *B,
                    void *stream) {
   if (n < 1 || n > kMaxBatch) return TTLG_ERR_INVALID_VALUE;
-  const void *fn = plan->kind == KK_BLK ? blk_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.blk_cpl)
+  const void *fn = plan->kind == KK_TMA ? tmap_ptr(plan->W, plan->kp.tm_rank)
+                   : plan->kind == KK_BLK ? blk_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.blk_cpl)
                    : plan->kind == KK_QUAD
                        ? quad_ptr(plan->W, plan->kp.qk * plan->W, plan->kp.qnj)
                        : (plan->kind == KK_BULKQ || plan->kind == KK_BULKG)
@@ -2025,7 +2256,17 @@ ttlg_status launch(const ttlg_plan_s *plan, int n, const void *const *A, void *c
     X.A[i] = A[i < n ? i : 0];
     X.B[i] = B[i < n ? i : 0];
   }
-  void *args[] = {(void *)&kp, (void *)&X};
+  TmaMaps *maps = nullptr;
+  void *args[] = {(void *)&kp, (void *)&X, nullptr};
+  if (plan->kind == KK_TMA) {
+    // the tensor map carries the operand's address: encoded per launch (host
+    // only, ~1 us), one per (A, B) pair of the batch
+    static thread_local TmaMaps tls_maps;
+    maps = &tls_maps;
+    for (int i = 0; i < n; i++)
+      if (encode_tmap(&maps->m[i], kp, plan->W, A[i]) != TTLG_OK) return TTLG_ERR_CUDA;
+    args[2] = (void *)maps;
+  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(plan->grid, n);
   cfg.blockDim = dim3(plan->threads);

@@ -101,7 +101,7 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
   const double *c = (mi.kind == KK_DIRECT)  ? kCoefDirect
                     : (mi.kind == KK_TILE)  ? kCoefTile
                     : (mi.kind == KK_QUAD)  ? kCoefQuad
-                    : (mi.kind == KK_BULKQ) ? kCoefBulkQ
+                    : (mi.kind == KK_BULKQ || mi.kind == KK_TMA) ? kCoefBulkQ
                     : (mi.kind == KK_BULKG) ? kCoefBulkG
                     : (mi.kind == KK_VEC)   ? kCoefVec
                                             : kCoefPipe;
@@ -155,12 +155,15 @@ double predict_ranked_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 }
 
 // The candidates' traversals of one tree are independent: interleaving them
-// (tree-major) lets the core overlap their dependent node loads.
+// (tree-major, a fixed group of kB candidates so that the node indices stay in
+// registers) lets the core overlap their dependent node loads.  Groups are
+// padded with copies of their last candidate; every candidate's sum is
+// accumulated in tree order, exactly as a one-at-a-time walk would.
 template <int NT, int D>
 static void gbt_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out,
                       double init, const int8_t (&F_)[NT][(1 << D) - 1],
                       const float (&T_)[NT][(1 << D) - 1], const float (&V_)[NT][1 << D]) {
-  constexpr int kB = 32;
+  constexpr int kB = 8;
   constexpr int NI = (1 << D) - 1;
   float d[kB][kGbtDesc];
   double s[kB];
@@ -170,20 +173,26 @@ static void gbt_batch(const ModelInput *mis, int n, const DeviceProfile &dev, do
       double dd[kGbtDesc];
       model_descriptor(mis[b0 + c], dev, dd);
       for (int k = 0; k < kGbtDesc; k++) d[c][k] = (float)dd[k];  // sklearn splits on float32
-      s[c] = init;
     }
+    for (int c = m; c < kB; c++)
+      for (int k = 0; k < kGbtDesc; k++) d[c][k] = d[m - 1][k];
+    for (int c = 0; c < kB; c++) s[c] = init;
     for (int t = 0; t < NT; t++) {
       const int8_t *F = F_[t];
       const float *T = T_[t];
-      // level-major: the m walks of one level are independent load chains
       int idx[kB];
-      for (int c = 0; c < m; c++) idx[c] = 0;
-      for (int l = 0; l < D; l++)
-        for (int c = 0; c < m; c++) {
+#pragma GCC unroll 8
+      for (int c = 0; c < kB; c++) idx[c] = 0;
+#pragma GCC unroll 8
+      for (int l = 0; l < D; l++) {
+#pragma GCC unroll 8
+        for (int c = 0; c < kB; c++) {
           const int i = idx[c];
           idx[c] = 2 * i + 1 + (d[c][F[i]] > T[i]);
         }
-      for (int c = 0; c < m; c++) s[c] += V_[t][idx[c] - NI];
+      }
+#pragma GCC unroll 8
+      for (int c = 0; c < kB; c++) s[c] += V_[t][idx[c] - NI];
     }
     for (int c = 0; c < m; c++) {
       const ModelInput &mi = mis[b0 + c];

@@ -189,8 +189,9 @@ static bool env_flag(const char *name, bool dflt) {
   return e[0] == '1';
 }
 static bool new_kernel_auto(int group) {
-  static const bool vec = env_flag("TTLG_VEC", true), bulk = env_flag("TTLG_BULK", false);
-  return group == KK_VEC ? vec : bulk;
+  static const bool vec = env_flag("TTLG_VEC", true), bulk = env_flag("TTLG_BULK", false),
+                    tma = env_flag("TTLG_TMA", false);
+  return group == KK_VEC ? vec : (group == KK_TMA ? tma : bulk);
 }
 constexpr int kBulkMaxStages = 6;
 // k_phase substitution mode (TTLG_PHASE: 0 off [default], 1 rows off 16-byte
@@ -275,7 +276,7 @@ Tile make_tile(const Problem &P, int a, int64_t ta, int b, int64_t tb) {
 
 int schema_of(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_DIRECT) return P.d == 1 ? TTLG_SCHEMA_COPY : TTLG_SCHEMA_FML;
-  if (kind == KK_QUAD || kind == KK_BULKQ) return TTLG_SCHEMA_OD;
+  if (kind == KK_QUAD || kind == KK_BULKQ || kind == KK_TMA) return TTLG_SCHEMA_OD;
   if (P.p[0] == 0) return TTLG_SCHEMA_FMS;
   for (int i = 0; i <= T.b; i++)
     if (P.p[i] <= T.a) return TTLG_SCHEMA_OA;  // input and output groups overlap
@@ -352,6 +353,81 @@ static bool bulk_ok(const Problem &P, const Tile &T, int kind) {  // also k_vec 
   return true;
 }
 
+// k_tmap (TMA tensor-map tile loads): the OD tile of k_quad with 16-byte
+// chunks, described as a TMA box over A's fused dims (rank <= 5) in map
+// order: input-run dims 0..a, the output-run dims in output order, the other
+// dims.  TMA needs 16-byte multiples for every global stride (map dims >= 1)
+// and for the box's inner row; the 128-byte swizzle that makes the consumers'
+// column reads conflict-free needs box rows of <= 128 bytes, so an input run
+// longer than 128 bytes is split along dim a into panels of 128 bytes (dims
+// 0..a-1 must then divide 128 bytes and t_a be a multiple of the panel's
+// share).  Each panel (box rows x the output run) must also start on a
+// 1024-byte boundary (the swizzle atom).  Fills the map fields of K when
+// given.
+static bool tma_ok(const Problem &P, const Tile &T, TileParams *K = nullptr) {
+  const int W = P.W, d = P.d, a = T.a, b = T.b;
+  if (d > 5 || W != P.esize || (W != 4 && W != 8)) return false;
+  if (quad_k(P, T) != 16 / W) return false;
+  int64_t LAunit = 1, LB = 1;
+  for (int k = 0; k < a; k++) LAunit *= T.t[k];
+  for (int i = 0; i <= b; i++) LB *= T.t[P.p[i]];
+  const int64_t LA = LAunit * T.t[a];
+  int64_t pa = T.t[a], np = 1;
+  if (LA * W > 128) {
+    if (128 % (LAunit * W)) return false;
+    pa = 128 / (LAunit * W);
+    if (T.t[a] % pa) return false;
+    np = T.t[a] / pa;
+  }
+  const int64_t pw = LAunit * pa * W;  // box row bytes
+  if (pw % 16 || pw > 128) return false;
+  if (np > 1 && (pw * LB) % 1024) return false;
+  // map order and box
+  int mo[TTLG_MAXD], nm = 0;
+  bool used[TTLG_MAXD] = {false};
+  for (int k = 0; k <= a; k++) {
+    mo[nm++] = k;
+    used[k] = true;
+  }
+  for (int i = 0; i <= b; i++) {
+    mo[nm++] = P.p[i];
+    used[P.p[i]] = true;
+  }
+  for (int k = 0; k < d; k++)
+    if (!used[k]) mo[nm++] = k;
+  if ((a > 0 ? T.t[0] : pa) * W % 16) return false;  // box inner row
+  for (int m = 0; m < nm; m++) {
+    const int k = mo[m];
+    const int64_t box = k == a ? pa : T.t[k];
+    if (box > 256 || P.n[k] > (1ll << 31)) return false;
+    if (m > 0 && ((P.sA[k] * W) % 16 || P.sA[k] * W >= (1ll << 40))) return false;
+  }
+  if (K) {
+    K->tm_rank = d;
+    K->tm_np = (int32_t)np;
+    K->tm_pa = (int32_t)pa;
+    K->tm_pw = (int32_t)pw;
+    K->tm_pbytes = (int32_t)(pw * LB);
+    K->tm_adim = a;  // map order starts with dims 0..a
+    int pos[TTLG_MAXD];
+    for (int m = 0; m < nm; m++) {
+      const int k = mo[m];
+      pos[k] = m;
+      K->tm_dim[m] = P.n[k];
+      K->tm_stride[m] = P.sA[k] * W;
+      K->tm_box[m] = (int32_t)(k == a ? pa : T.t[k]);
+    }
+    int ng = 0;
+    for (int k = 0; k < d; k++) {
+      if (ceil_div(P.n[k], T.t[k]) <= 1) continue;
+      K->tm_gmap[ng] = pos[k];
+      K->tm_gt[ng] = (int32_t)T.t[k];
+      ng++;
+    }
+  }
+  return true;
+}
+
 // Smallest block factor >= t (<= n) that makes pre * t a multiple of K, or 0.
 static int64_t round_block(int64_t t, int64_t pre, int64_t n, int K) {
   int64_t m = 1;
@@ -402,7 +478,8 @@ struct TileSummary {
 // every A-row on a 16-byte (chunk) boundary
 static int layout_unit(const Problem &P, const Tile &T, int kind) {
   if (kind == KK_QUAD) return quad_k(P, T);
-  if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_VEC || kind == KK_PHASE) return 16 / P.W;
+  if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_VEC || kind == KK_PHASE || kind == KK_TMA)
+    return 16 / P.W;
   return 0;
 }
 
@@ -440,8 +517,9 @@ static bool summarize(const Problem &P, const Tile &T, int kind, TileSummary &S)
     Q *= T.t[k];
   }
   S.buf_bytes = (int)r16(cur * P.W);
+  if (kind == KK_TMA) S.buf_bytes = (int)((S.V * P.W + 1023) / 1024 * 1024);  // dense box
   S.smem_base = (int)(r16(S.RA * 8) + r16(S.RB * 8) + r16(S.LB * 4) + r16(S.RA * 4) +
-                      r16(S.RB * 4) + 64 + S.buf_bytes);
+                      r16(S.RB * 4) + 64 + S.buf_bytes + (kind == KK_TMA ? 1024 : 0));
   return true;
 }
 
@@ -451,8 +529,10 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   memset(&K, 0, sizeof(K));
   const int qk = layout_unit(P, T, kind);
   if (kind == KK_QUAD && qk == 0) return false;
-  const bool bulk = kind == KK_BULKQ || kind == KK_BULKG;
-  if (bulk && (isdelta || !bulk_ok(P, T, kind))) return false;
+  const bool tmap = kind == KK_TMA;
+  const bool bulk = kind == KK_BULKQ || kind == KK_BULKG || tmap;
+  if (tmap && (isdelta || !tma_ok(P, T, &K))) return false;
+  if (bulk && !tmap && (isdelta || !bulk_ok(P, T, kind))) return false;
   if (kind == KK_VEC && !bulk_ok(P, T, KK_VEC)) return false;
   // k_vec: isdelta[0] is not an input-run pad but extra chunk units on the
   // first output-only dim's shared-memory stride (the gather-conflict search,
@@ -540,7 +620,8 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
   for (int i = 0; i <= b; i++) {
     const int k = P.p[i];
     if (!inIS[k] && T.t[k] > 1) {
-      int64_t s = pad_stride(cur, Q, P.W, qk, od, mult);
+      // k_tmap: the dense TMA box (its swizzle replaces the pad)
+      int64_t s = tmap ? cur : pad_stride(cur, Q, P.W, qk, od, mult);
       if (first_out) s += (int64_t)opad * qk;
       first_out = false;
       sm[k] = s;
@@ -623,6 +704,11 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     K.off_bar = take(16 * (int64_t)nbuf);
     off = (off + 127) / 128 * 128;
     K.stage_bytes = (int32_t)((smem_elems * P.W + 127) / 128 * 128);
+    if (tmap) {
+      // 1024-byte swizzle atoms: the kernel rounds the ring's start up at run time
+      K.stage_bytes = (int32_t)((smem_elems * P.W + 1023) / 1024 * 1024);
+      off += 1024;
+    }
     K.off_data = (int32_t)off;
     K.off_data2 = K.off_data;
     off += (int64_t)K.stage_bytes * nbuf;
@@ -658,9 +744,9 @@ static bool build_params(const Problem &P, const Tile &T, int kind, int threads,
     // consumers are threads - 32 (warp 0 produces); quad: one output position
     // per consumer, gather: one 16-byte output chunk per consumer
     const int ntc = threads - 32;
-    const int L = kind == KK_BULKQ ? K.LB : K.LB * P.W / 16;
+    const int L = kind != KK_BULKG ? K.LB : K.LB * P.W / 16;
     if (L > ntc) return false;
-    K.qk = kind == KK_BULKQ ? qk : 0;
+    K.qk = kind != KK_BULKG ? qk : 0;
     // TMA bulk copies cost ~40 SM cycles each (measured: 256-byte rows move
     // 1.9 TB/s): only rows of >= kBulkTmaRowBytes go through TMA
     K.tma_rows = bulk_tma_mode() == 1 ||
@@ -1024,9 +1110,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                      const TileSummary &S, double cl, double cs) {
     int smem = S.smem_base + (kind == KK_PIPE ? S.buf_bytes : 0);
     mi.nstage = 0;
-    if (kind == KK_BULKQ || kind == KK_BULKG) {
+    if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_TMA) {
       // one output position (quad) / 16-byte output chunk (gather) per consumer thread
-      if ((kind == KK_BULKQ ? S.LB : S.LB * P.W / 16) > threads - 32) return false;
+      if ((kind != KK_BULKG ? S.LB : S.LB * P.W / 16) > threads - 32) return false;
       // as many ring stages as fit next to the tables (2..kBulkMaxStages), one CTA per SM
       const int buf = (S.buf_bytes + 127) / 128 * 128;
       const int fixed = S.smem_base - S.buf_bytes + 256;
@@ -1039,7 +1125,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // k_quad: at most 4 output positions per thread, warp-wide shuffles (whole warps)
     if (kind == KK_QUAD && (S.LB > 4 * threads || threads % 32)) return false;
     if (kind == KK_VEC && (S.LB * P.W / 16 > threads || threads % 32)) return false;
-    mi.qk = (kind == KK_QUAD || kind == KK_VEC || kind == KK_BULKQ || kind == KK_BULKG) ? S.qk : 0;
+    mi.qk = (kind == KK_QUAD || kind == KK_VEC || kind == KK_BULKQ || kind == KK_BULKG ||
+             kind == KK_TMA)
+                ? S.qk
+                : 0;
     mi.kind = kind;
     mi.schema = schema;
     mi.W = P.W;
@@ -1083,7 +1172,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                          double &cs, TileSummary &S) {
     for (int k = 0; k < TTLG_MAXD; k++) delta[k] = 0;
     cl = cs = 1.0;
-    if (group == KK_BULKQ || group == KK_BULKG) {
+    if (group == KK_BULKQ || group == KK_BULKG || group == KK_TMA) {
       // feasibility at the largest consumer count; the ring is sized in make_mi
       if (!build_params(P, T, group, 32 + 512, 1, K0)) return false;
       S.smem_base = K0.smem_bytes;
@@ -1209,10 +1298,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // variant and block size.
   auto consider = [&](int group, int a, int64_t ta, int b, int64_t tb) {
     if (hv == 4 || hv == 9) return;  // k_deint / k_blk forced: no staged / direct candidates
-    const bool bulk = group == KK_BULKQ || group == KK_BULKG;
+    const bool bulk = group == KK_BULKQ || group == KK_BULKG || group == KK_TMA;
     if (bulk || group == KK_VEC) {
       if (forceW) return;  // element-width fallback plans: no 16-byte requirement
-      const int want = group == KK_BULKQ ? 5 : (group == KK_BULKG ? 6 : 7);
+      const int want = group == KK_BULKQ ? 5 : (group == KK_BULKG ? 6 : (group == KK_TMA ? 10 : 7));
       if (hv == 0 ? !new_kernel_auto(group) : hv != want) return;
       // in the automatic choice k_vec only challenges matching-FVI winners (below)
       if (hv == 0 && group == KK_VEC && P.p[0] != 0 && !listing) return;
@@ -1230,7 +1319,8 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     Tile T = make_tile(P, a, ta, b, tb);
     if (!T.ok) return;
     if (group == KK_QUAD && (!quad_k(P, T) || forceW || (hv != 0 && hv != 3))) return;
-    if ((bulk || group == KK_VEC) && !bulk_ok(P, T, group)) return;  // 16-byte rows
+    if (group == KK_TMA ? !tma_ok(P, T) : ((bulk || group == KK_VEC) && !bulk_ok(P, T, group)))
+      return;  // 16-byte rows / a TMA box
     const int schema = schema_of(P, T, group);
     if (force_schema != TTLG_SCHEMA_AUTO && force_schema != schema) {
       // COPY and FML share the direct kernel; accept FML for a rank-1 problem
@@ -1339,6 +1429,19 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       }
     }
   };
+  // groups that consider() would reject for every slice (opt-in kernels not
+  // enabled, k_vec outside its matching-FVI challenge): skip the calls
+  const bool want_bulkq = hv == 5 || (hv == 0 && new_kernel_auto(KK_BULKQ));
+  const bool want_bulkg = hv == 6 || (hv == 0 && new_kernel_auto(KK_BULKG));
+  const bool want_tma = hv == 10 || (hv == 0 && new_kernel_auto(KK_TMA));
+  const bool want_vec = hv == 7 || (hv == 0 && new_kernel_auto(KK_VEC) && (P.p[0] == 0 || listing));
+  auto consider_opt = [&](int group, int a, int64_t ta, int b, int64_t tb) {
+    const bool want = group == KK_BULKQ ? want_bulkq
+                      : group == KK_BULKG ? want_bulkg
+                      : group == KK_TMA   ? want_tma
+                                          : want_vec;
+    if (want) consider(group, a, ta, b, tb);
+  };
   int64_t blocksA[32], blocksB[32];
   if (P.p[0] == 0) {
     // ---- direct (FML / COPY): input run = dims 0..a (contiguous), output run = dim 0
@@ -1373,22 +1476,23 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           // factor, drawn from both candidate lists
           for (int i = 0; i < nbA; i++) {
             consider(KK_TILE, a, blocksA[i], b, blocksA[i]);
-            consider(KK_VEC, a, blocksA[i], b, blocksA[i]);
-            consider(KK_BULKG, a, blocksA[i], b, blocksA[i]);
+            consider_opt(KK_VEC, a, blocksA[i], b, blocksA[i]);
+            consider_opt(KK_BULKG, a, blocksA[i], b, blocksA[i]);
           }
           for (int j = 0; j < nbB; j++) {
             consider(KK_TILE, a, blocksB[j], b, blocksB[j]);
-            consider(KK_VEC, a, blocksB[j], b, blocksB[j]);
-            consider(KK_BULKG, a, blocksB[j], b, blocksB[j]);
+            consider_opt(KK_VEC, a, blocksB[j], b, blocksB[j]);
+            consider_opt(KK_BULKG, a, blocksB[j], b, blocksB[j]);
           }
         } else {
           for (int i = 0; i < nbA; i++) {
             for (int j = 0; j < nbB; j++) {
               consider(KK_TILE, a, blocksA[i], b, blocksB[j]);
               consider(KK_QUAD, a, blocksA[i], b, blocksB[j]);
-              consider(KK_BULKQ, a, blocksA[i], b, blocksB[j]);
-              consider(KK_BULKG, a, blocksA[i], b, blocksB[j]);
-              consider(KK_VEC, a, blocksA[i], b, blocksB[j]);
+              consider_opt(KK_BULKQ, a, blocksA[i], b, blocksB[j]);
+              consider_opt(KK_TMA, a, blocksA[i], b, blocksB[j]);
+              consider_opt(KK_BULKG, a, blocksA[i], b, blocksB[j]);
+              consider_opt(KK_VEC, a, blocksA[i], b, blocksB[j]);
               // k_quad needs whole chunks per run: the same slice with the
               // blocking factors rounded up to a chunk multiple (e.g. t1 = 22
               // -> 24 for [3, 4096, 4096] fp32 `2 1 0`)
@@ -1398,9 +1502,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                 const int64_t rb = round_block(blocksB[j], preB, P.n[pb], Kq);
                 if (ra && rb && (ra != blocksA[i] || rb != blocksB[j])) {
                   consider(KK_QUAD, a, ra, b, rb);
-                  consider(KK_BULKQ, a, ra, b, rb);
-                  consider(KK_BULKG, a, ra, b, rb);
-                  consider(KK_VEC, a, ra, b, rb);
+                  consider_opt(KK_BULKQ, a, ra, b, rb);
+                  consider_opt(KK_TMA, a, ra, b, rb);
+                  consider_opt(KK_BULKG, a, ra, b, rb);
+                  consider_opt(KK_VEC, a, ra, b, rb);
                 }
               }
             }
@@ -1622,20 +1727,30 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     const int mask = 128 / blk_wc - 1;
     int lg = 0;
     while ((1 << lg) <= mask) lg++;
+    // the simulated lanes' output digits do not depend on the layout: decode
+    // them once (the layouts below only change the strides)
+    const int nm = (int)std::min<int64_t>(2, ceil_div(Cb, 32));
+    int16_t gdig[2][4][32][TTLG_MAXD];
+    for (int m = 0; m < nm; m++)
+      for (int u = 0; u < KC; u++)
+        for (int l = 0; l < 32; l++) {
+          int64_t rem = (32 * m + l) % Cb * KC + u;
+          for (int k = 0; k < cb; k++) {
+            const int64_t e = P.n[P.p[k]];
+            gdig[m][u][l][k] = (int16_t)(rem % e);
+            rem /= e;
+          }
+        }
     auto gather_cost = [&](int pad, int swz) {
       int32_t sS[TTLG_MAXD];
       strides(pad, sS);
       double c = 0;
-      for (int64_t m = 0; m < std::min<int64_t>(2, ceil_div(Cb, 32)); m++)
+      for (int m = 0; m < nm; m++)
         for (int u = 0; u < KC; u++) {
           int64_t addr[32];
           for (int l = 0; l < 32; l++) {
-            int64_t rem = (32 * m + l) % Cb * KC + u, off = 0;
-            for (int k = 0; k < cb; k++) {
-              const int64_t e = P.n[P.p[k]];
-              off += (rem % e) * sS[k];
-              rem /= e;
-            }
+            int64_t off = 0;
+            for (int k = 0; k < cb; k++) off += (int64_t)gdig[m][u][l][k] * sS[k];
             if (swz) {
               const int64_t ch = off / KC;
               off = (ch ^ ((ch >> swz) & mask)) * KC + off % KC;
@@ -1942,7 +2057,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   plan->W = P.W;
   plan->align = kind_final == KK_QUAD ? K.qk * P.W
                 : (kind_final == KK_BULKQ || kind_final == KK_BULKG || kind_final == KK_VEC ||
-                   kind_final == KK_PHASE)
+                   kind_final == KK_PHASE || kind_final == KK_TMA)
                     ? 16
                     : P.W;
   plan->threads = B.mi.threads;

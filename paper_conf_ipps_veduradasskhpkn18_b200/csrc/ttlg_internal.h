@@ -61,7 +61,9 @@ enum KernelKind : int32_t {
                   // in shared memory) and element stores (k_phase)
   KK_BLK = 9,     // closed leading block (<= 8 KB, contiguous in A and B): one warp per
                   // block, WC-byte chunk loads and gathered WC-byte stores (k_blk)
-  KK_NUM = 10,
+  KK_TMA = 10,    // OD: TMA tensor-map tile loads (cp.async.bulk.tensor, 128-byte swizzle)
+                  // into an mbarrier ring, k_bulk's quad consumers (k_tmap)
+  KK_NUM = 11,
 };
 
 // Everything one launch needs, passed by value as a __grid_constant__ kernel
@@ -135,6 +137,18 @@ struct TileParams {
   int64_t a_elems;
   int32_t blk_cpl;  // k_blk: chunks per lane (template instance)
   int32_t blk_swz;  // k_blk: chunk-slot XOR swizzle shift (0: row padding RA instead)
+  // k_tmap: the tile box as a TMA tensor map over A's fused dims in "map order"
+  // (input-run dims 0..a, then the output-run dims in output order, then the
+  // other dims).  The input run is split into tm_np panels of tm_pa elements
+  // of dim a (tm_pw bytes per box row, <= 128); panel p is one box load of
+  // tm_pbytes to stage + p * tm_pbytes, 128-byte swizzled.  Grid dim g
+  // contributes coordinate (digit * tm_gt[g]) to map dim tm_gmap[g].
+  int32_t tm_rank, tm_np, tm_pa, tm_pw, tm_pbytes, tm_adim;
+  int32_t tm_gmap[TTLG_MAXD], tm_gt[TTLG_MAXD];
+  // host side (encoded per launch with the operand's address, kernels.cu)
+  int64_t tm_dim[TTLG_MAXD];     // globalDim, map order
+  int64_t tm_stride[TTLG_MAXD];  // globalStrides in bytes of map dims 1..rank-1
+  int32_t tm_box[TTLG_MAXD];     // boxDim (dim a: tm_pa)
 };
 
 // Operand pointers of one launch: entry blockIdx.y (grid.y = n <= kMaxBatch;

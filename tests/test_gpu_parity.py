@@ -712,3 +712,51 @@ def test_blk_batch():
     torch.cuda.synchronize()
     for a, b in zip(As, Bs):
         _assert_equal(_bits(b), oracle.transpose(_bits(a), ext, perm), "blk batch")
+
+
+@pytest.mark.parametrize("case", _bulk_cases(), ids=lambda c: c.label())
+def test_tmap_forced(case):
+    """k_tmap (variant 10: TMA tensor-map box loads, 128-byte swizzle, k_bulk's
+    quad consumers) forced on every config shape it applies to (fused rank
+    <= 5, 16-byte aligned strides)."""
+    try:
+        ttlg.plan(_dt(case.elem_bytes), case.extents, case.perm, variant=10)
+    except ttlg.TtlgError:
+        pytest.skip("k_tmap not applicable")
+    got, exp, info = _run(case.extents, case.perm, case.elem_bytes, case_seed(case.case_id),
+                          plan_kwargs={"variant": 10}, canary=64)
+    assert info["kernel"] == "tmap"
+    _assert_equal(got, exp, f"tmap {info}")
+
+
+@pytest.mark.parametrize("eb", [4, 8])
+def test_tmap_partial_tiles_panels_and_candidates(eb):
+    """k_tmap on ragged tiles (the box's zero fill past the edge), input runs
+    split into 128-byte panels, every candidate slice of a few shapes, and a
+    batch of pairs (one tensor map per pair)."""
+    K = 16 // eb
+    n_ok = 0
+    for ext, perm in (([6 * K, 40, 7], [1, 0, 2]), ([4 * K, 30, 3 * K], [2, 1, 0]),
+                      ([64, 72, 5], [1, 0, 2]), ([80, 4, 16, 20, 16], [3, 2, 0, 4, 1]),
+                      ([2 * K, 50, 3, 4 * K], [3, 1, 0, 2]), ([200, 136], [1, 0])):
+        try:
+            cands = ttlg.plan_candidates(_dt(eb), ext, perm, variant=10)
+        except ttlg.TtlgError:
+            continue
+        for cd in cands[:: max(1, len(cands) // 12)]:
+            kw = dict(cd["hints"])
+            got, exp, info = _run(ext, perm, eb, 96, plan_kwargs=kw, canary=32)
+            assert info["kernel"] == "tmap"
+            _assert_equal(got, exp, f"tmap {ext} {perm} {kw} {info}")
+            n_ok += 1
+    assert n_ok >= 20
+    ext, perm = [64, 72, 5], [1, 0, 2]
+    n = int(np.prod(ext))
+    p = ttlg.plan(_dt(eb), ext, perm, variant=10)
+    As = [gen_tensor_torch(1900 + i, n, eb, device=DEV) for i in range(3)]
+    Bs = [torch.empty_like(a) for a in As]
+    p.execute_batch([a.data_ptr() for a in As], [b.data_ptr() for b in Bs],
+                    torch.cuda.current_stream().cuda_stream)
+    torch.cuda.synchronize()
+    for a, b in zip(As, Bs):
+        _assert_equal(_bits(b), oracle.transpose(_bits(a), ext, perm), "tmap batch")

@@ -343,3 +343,28 @@ def test_blk_applicability():
     d = ttlg.plan("f64", [16] * 6, [1, 0, 2, 4, 3, 5], variant=9,
                   access_bytes=8).describe()
     assert d["kernel"] == "blk" and d["access_bytes"] == 8
+
+
+def test_tmap_applicability():
+    """k_tmap (variant 10) describes the OD tile as a TMA box: fused rank <= 5,
+    16-byte multiples for every A stride past the FVI, box rows <= 128 bytes
+    (longer input runs split into 128-byte panels), k_quad's chunk alignment.
+    Not in the automatic choice unless TTLG_TMA=1."""
+    d = ttlg.plan("f64", [5120, 5120], [1, 0], variant=10).describe()
+    assert d["kernel"] == "tmap" and d["schema"] == "OD" and d["stages"] >= 2
+    assert d["threads"] in (288, 544)
+    # a fused rank-5 problem qualifies; rank 6 (16^6 reversal) does not
+    assert ttlg.plan("f64", [80, 4, 16, 20, 16], [3, 2, 0, 4, 1],
+                     variant=10).describe()["kernel"] == "tmap"
+    for ext, perm in (([16] * 6, [5, 4, 3, 2, 1, 0]), ([17, 17, 17], [2, 1, 0]),
+                      ([3, 4096, 4096], [2, 1, 0])):
+        with pytest.raises(ttlg.TtlgError) as e:
+            ttlg.plan("f64" if ext[0] != 3 else "f32", ext, perm, variant=10)
+        assert e.value.code == 7
+    # every candidate keeps the box rule: the input run is one panel of <= 128
+    # bytes or whole 128-byte panels of dim a
+    for c in ttlg.plan_candidates("f64", [200, 136], [1, 0], variant=10):
+        la = c["in_run"] * 8
+        assert la <= 128 or la % 128 == 0
+    auto = ttlg.plan("f64", [5120, 5120], [1, 0]).describe()
+    assert auto["kernel"] != "tmap"

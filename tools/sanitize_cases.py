@@ -1,7 +1,8 @@
 #!/usr/bin/env python
 """Small launches of every kernel family for compute-sanitizer (memcheck,
 racecheck, synccheck): k_direct, k_tile, k_pipe, k_quad, k_deint, k_inter,
-k_bulk (TMA rows and cp.async rows, quad and gather consumers), ragged tiles,
+k_bulk (TMA rows and cp.async rows, quad and gather consumers), k_blk, k_tmap
+(TMA tensor-map boxes), ragged tiles,
 strided sub-tensor plans and batched launches.
 
   compute-sanitizer --tool memcheck python tools/sanitize_cases.py
@@ -41,6 +42,9 @@ def main():
         ([15, 15, 6, 5], [1, 0, 3, 2], 8, {"variant": 9}),   # k_blk, 8-byte chunks
         ([8, 8, 8, 9], [2, 1, 0, 3], 4, {"variant": 9}),     # k_blk, 3-D inner perm
         ([24, 24, 12, 4, 3, 2], [1, 0, 2, 4, 3, 5], 8, {}),  # auto (k_blk)
+        ([64, 72, 5], [1, 0, 2], 8, {"variant": 10}),        # k_tmap (TMA boxes)
+        ([80, 4, 16, 20, 16], [3, 2, 0, 4, 1], 8, {"variant": 10}),  # k_tmap panels
+        ([24, 40, 7], [1, 0, 2], 4, {"variant": 10}),        # k_tmap fp32, ragged
     ]
     for ext, perm, eb, hints in cases:
         n = 1
