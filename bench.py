@@ -609,15 +609,36 @@ def main():
                         if kname(infos[i]) == k:
                             p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
                 kev[k][s][1].record(stream)
-    # per-case durations (model error, per-case table): an event pair per launch
-    for s in range(args.steps):
-        one_step(evs[s])
+    # per-case durations (model error, per-case table): in graph mode each case
+    # as its own graph of K back-to-back launches between one event pair (the
+    # kernel time the step sees; an event pair per launch also times the host's
+    # launch rate, which dominates sub-10-us kernels); else an event pair per launch
+    if graph is not None:
+        per_case_ms = []
+        for i, p in enumerate(plans):
+            cg = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(cg, stream=stream):
+                for _ in range(args.steps):
+                    p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
+            with torch.cuda.stream(stream):
+                cg.replay()
+                ms = []
+                for _ in range(3):
+                    evs[0][i][0].record(stream)
+                    cg.replay()
+                    evs[0][i][1].record(stream)
+                    evs[0][i][1].synchronize()
+                    ms.append(evs[0][i][0].elapsed_time(evs[0][i][1]) / args.steps)
+            per_case_ms.append(ms)
+            del cg
+    else:
+        for s in range(args.steps):
+            one_step(evs[s])
+        torch.cuda.synchronize()
+        per_case_ms = [[evs[s][i][0].elapsed_time(evs[s][i][1]) for s in range(args.steps)]
+                       for i in range(len(plans))]
     torch.cuda.synchronize()
     clk = clocks.stop()
-
-    # per-launch durations -> per-kernel shares, model error, per-case table
-    per_case_ms = [[evs[s][i][0].elapsed_time(evs[s][i][1]) for s in range(args.steps)]
-                   for i in range(len(plans))]
     groups = {}
     for i, info in enumerate(infos):
         k = kname(info)
@@ -760,8 +781,9 @@ def main():
                        "timing": "value: K steps between two events (no per-launch events); "
                                  "roofline/kernels: a second pass of K steps, each kernel's "
                                  "launches grouped (as one graph in graph mode) between one "
-                                 "event pair per step; cases / model error: a third pass "
-                                 "with an event pair per launch",
+                                 "event pair per step; cases / model error: a third pass, "
+                                 + ("each case as a graph of K launches between one event pair"
+                                    if graph is not None else "an event pair per launch"),
                        "l2": l2_label},
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,

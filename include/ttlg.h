@@ -113,7 +113,7 @@ typedef struct {
                                             and B: one warp per block, chunk loads and
                                             gathered chunk stores), 10 = k_tmap (OD:
                                             the tile loaded by TMA tensor-map box copies,
-                                            cp.async.bulk.tensor, 128-byte swizzle; fused
+                                            cp.async.bulk.tensor, swizzled; fused
                                             rank <= 5, 16-byte aligned A strides and
                                             k_quad's chunk alignment), else
                                             TTLG_ERR_UNSUPPORTED.  The automatic choice

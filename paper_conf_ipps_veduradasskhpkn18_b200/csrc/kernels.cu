@@ -1813,10 +1813,11 @@ __global__ void __launch_bounds__(544, 1) k_bulk(const __grid_constant__ TilePar
 // box bytes and issues ONE cp.async.bulk.tensor (SASS UTMALDG) per panel --
 // no per-row or per-chunk load instructions, the hardware walks the box and
 // zero-fills past the tensor's edge (partial tiles).  The box lands dense
-// with the 128-byte swizzle (16-byte slot bits 4-6 XOR address bits 7-9, per
-// 1024-byte atom), which spreads the consumers' column reads -- 8 output
-// positions at one input position, rows pw <= 128 bytes apart -- over all
-// banks, the job the padded layouts of the other kernels do by hand.
+// with the swizzle whose span is one box row (pw = 128 / 64 / 32 bytes:
+// 16-byte slot bits 4-6 / 4-5 / 4 XOR address bits 7-9 / 7-8 / 7; 16-byte
+// rows need none), which spreads the consumers' column reads -- 8 output
+// positions at one input position, rows pw bytes apart -- over all banks,
+// the job the padded layouts of the other kernels do by hand.
 // Consumers: as k_bulk MODE 0 (K x K shuffle transposes, 16-byte stores) with
 // the shared-memory address of chunk (input position x, output position j)
 // = swizzle(panel(x) * pbytes + (x * S mod pw) + j * pw).
@@ -1868,6 +1869,7 @@ __global__ void __launch_bounds__(544, 1) k_tmap(const __grid_constant__ TilePar
   auto full_bar = [&](int st) { return s_bar + 16u * st; };
   auto empty_bar = [&](int st) { return s_bar + 16u * st + 8u; };
   const int pw = P.tm_pw, pbytes = P.tm_pbytes;
+  const uint32_t swz = (uint32_t)P.tm_swz;
 
   if (tid == 0) {
     asm volatile("prefetch.tensormap [%0];\n" ::"l"(reinterpret_cast<uint64_t>(&M.m[blockIdx.y]))
@@ -1965,7 +1967,7 @@ __global__ void __launch_bounds__(544, 1) k_tmap(const __grid_constant__ TilePar
       const int2 t = lds_int2(s_tabB + 8 * row);
       const bool rok = act && j0 < LB && (full || lds_int(s_digA + 4 * row) < c.limA);
       const uint32_t o = (uint32_t)(t.y - q * S) + jc;  // chunk x..x+K-1 at position j0
-      C v = lds_T<C>(sbuf + (o ^ ((o >> 3) & 0x70u)));
+      C v = lds_T<C>(sbuf + (o ^ ((o >> 3) & swz)));
       quad_transpose<S, 16>(v, q);
       const int jb = j0 - q;
       C *dst = reinterpret_cast<C *>(B + (c.bB + jb) * S);
@@ -2165,7 +2167,7 @@ int kernel_regs(int kind, int W) {
 }
 
 // cuTensorMapEncodeTiled through the runtime's driver entry point (no libcuda
-// link): k_tmap's box over A in map order, 128-byte swizzle, zero fill
+// link): k_tmap's box over A in map order, the row's swizzle span, zero fill
 static ttlg_status encode_tmap(CUtensorMap *m, const TileParams &kp, int W, const void *A) {
   static PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
   static std::once_flag once;
@@ -2191,7 +2193,11 @@ static ttlg_status encode_tmap(CUtensorMap *m, const TileParams &kp, int W, cons
   }
   const CUresult e = enc(m, W == 8 ? CU_TENSOR_MAP_DATA_TYPE_UINT64 : CU_TENSOR_MAP_DATA_TYPE_UINT32,
                          (cuuint32_t)r, const_cast<void *>(A), dim, str, box, es,
-                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                         CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         kp.tm_pw == 128  ? CU_TENSOR_MAP_SWIZZLE_128B
+                         : kp.tm_pw == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                         : kp.tm_pw == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                          : CU_TENSOR_MAP_SWIZZLE_NONE,
                          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return e == CUDA_SUCCESS ? TTLG_OK : TTLG_ERR_CUDA;
 }

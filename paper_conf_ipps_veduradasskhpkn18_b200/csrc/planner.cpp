@@ -356,14 +356,14 @@ static bool bulk_ok(const Problem &P, const Tile &T, int kind) {  // also k_vec 
 // k_tmap (TMA tensor-map tile loads): the OD tile of k_quad with 16-byte
 // chunks, described as a TMA box over A's fused dims (rank <= 5) in map
 // order: input-run dims 0..a, the output-run dims in output order, the other
-// dims.  TMA needs 16-byte multiples for every global stride (map dims >= 1)
-// and for the box's inner row; the 128-byte swizzle that makes the consumers'
-// column reads conflict-free needs box rows of <= 128 bytes, so an input run
-// longer than 128 bytes is split along dim a into panels of 128 bytes (dims
-// 0..a-1 must then divide 128 bytes and t_a be a multiple of the panel's
-// share).  Each panel (box rows x the output run) must also start on a
-// 1024-byte boundary (the swizzle atom).  Fills the map fields of K when
-// given.
+// dims.  TMA needs 16-byte multiples for every global stride (map dims >= 1).
+// The swizzle that makes the consumers' column reads conflict-free lays box
+// rows of exactly its span (16 [none], 32, 64 or 128 bytes) densely (measured:
+// 64-byte rows under the 128-byte swizzle land elsewhere), and the box row is
+// dim 0's box: so the input run lies in dim 0 (a = 0) and is 16, 32, 64 or
+// 128 bytes, or a multiple of 128 bytes split into 128-byte panels (one box
+// load each, every panel on a 1024-byte swizzle-atom boundary).  Fills the
+// map fields of K when given.
 static bool tma_ok(const Problem &P, const Tile &T, TileParams *K = nullptr) {
   const int W = P.W, d = P.d, a = T.a, b = T.b;
   if (d > 5 || W != P.esize || (W != 4 && W != 8)) return false;
@@ -379,8 +379,8 @@ static bool tma_ok(const Problem &P, const Tile &T, TileParams *K = nullptr) {
     if (T.t[a] % pa) return false;
     np = T.t[a] / pa;
   }
-  const int64_t pw = LAunit * pa * W;  // box row bytes
-  if (pw % 16 || pw > 128) return false;
+  const int64_t pw = LAunit * pa * W;  // box row bytes = the swizzle span (16 / 32 / 64 / 128)
+  if (pw != 16 && pw != 32 && pw != 64 && pw != 128) return false;
   if (np > 1 && (pw * LB) % 1024) return false;
   // map order and box
   int mo[TTLG_MAXD], nm = 0;
@@ -395,7 +395,9 @@ static bool tma_ok(const Problem &P, const Tile &T, TileParams *K = nullptr) {
   }
   for (int k = 0; k < d; k++)
     if (!used[k]) mo[nm++] = k;
-  if ((a > 0 ? T.t[0] : pa) * W % 16) return false;  // box inner row
+  // the swizzle lays box rows of its span densely: the box's inner row (dim
+  // 0) must be the whole row, so the input run lies in dim 0 (a = 0)
+  if (a != 0) return false;
   for (int m = 0; m < nm; m++) {
     const int k = mo[m];
     const int64_t box = k == a ? pa : T.t[k];
@@ -409,6 +411,7 @@ static bool tma_ok(const Problem &P, const Tile &T, TileParams *K = nullptr) {
     K->tm_pw = (int32_t)pw;
     K->tm_pbytes = (int32_t)(pw * LB);
     K->tm_adim = a;  // map order starts with dims 0..a
+    K->tm_swz = pw == 128 ? 0x70 : (pw == 64 ? 0x30 : (pw == 32 ? 0x10 : 0));
     int pos[TTLG_MAXD];
     for (int m = 0; m < nm; m++) {
       const int k = mo[m];
@@ -818,21 +821,35 @@ static double wavefront_ratio(const int64_t *addr, int W) {
   const int per_phase = 128 / W, phases = 32 / per_phase, wpl = W / 4;
   int total = 0;
   for (int ph = 0; ph < phases; ph++) {
-    // distinct words per bank (a repeated word is a broadcast); degree capped at 8
-    uint32_t bw[32][8];
-    uint8_t cnt[32] = {0};
+    // a phase touches 32 words; distinct words per bank (a repeated word is a
+    // broadcast), degree capped at 8
+    uint32_t w[32];
+    int n = 0;
+    for (int l = ph * per_phase; l < (ph + 1) * per_phase; l++)
+      for (int k = 0; k < wpl; k++) w[n++] = (uint32_t)(addr[l] * wpl + k);
+    uint32_t lanes[32] = {0}, seen = 0;
+    for (int i = 0; i < n; i++) {
+      lanes[w[i] & 31] |= 1u << i;
+      seen |= 1u << (w[i] & 31);
+    }
+    if (n == 32 && seen == 0xffffffffu) {  // one word per bank: conflict-free
+      total += 1;
+      continue;
+    }
     int worst = 1;
-    for (int l = ph * per_phase; l < (ph + 1) * per_phase; l++) {
-      for (int k = 0; k < wpl; k++) {
-        const uint32_t w = (uint32_t)(addr[l] * wpl + k);
-        const int b = (int)(w & 31);
+    for (int b = 0; b < 32; b++) {
+      uint32_t m = lanes[b];
+      if (__builtin_popcount(m) <= worst) continue;  // cannot exceed the incumbent
+      uint32_t vals[8];
+      int c = 0;
+      while (m && c < 8) {
+        const int i = __builtin_ctz(m);
+        m &= m - 1;
         bool dup = false;
-        for (int s = 0; s < cnt[b]; s++) dup |= bw[b][s] == w;
-        if (!dup && cnt[b] < 8) {
-          bw[b][cnt[b]++] = w;
-          if (cnt[b] > worst) worst = cnt[b];
-        }
+        for (int t = 0; t < c; t++) dup |= vals[t] == w[i];
+        if (!dup) vals[c++] = w[i];
       }
+      if (c > worst) worst = c;
     }
     total += worst;
   }
@@ -1741,12 +1758,18 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
             rem /= e;
           }
         }
+    // (a layout's cost only grows over its chunk sets, and a later layout must
+    // be strictly cheaper to win: stop a layout at the incumbent's cost, and
+    // the whole search at the conflict-free bound of one wavefront per set)
+    double best_c = 1e300;
+    const double floor_c = (double)nm * KC;
     auto gather_cost = [&](int pad, int swz) {
       int32_t sS[TTLG_MAXD];
       strides(pad, sS);
       double c = 0;
       for (int m = 0; m < nm; m++)
         for (int u = 0; u < KC; u++) {
+          if (c >= best_c) return c;
           int64_t addr[32];
           for (int l = 0; l < 32; l++) {
             int64_t off = 0;
@@ -1762,8 +1785,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       return c;
     };
     int best_pad = 0, best_swz = 0;
-    double best_c = 1e300;
-    for (int pad = 0; pad <= 8 * KC; pad += KC) {
+    for (int pad = 0; pad <= 8 * KC && best_c > floor_c; pad += KC) {
       const double c = gather_cost(pad, 0);
       if (c < best_c - 1e-9) {
         best_c = c;
@@ -1773,7 +1795,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     // a swizzle permutes whole groups of 128 bytes; 16-byte chunks only
     // (measured, r2e31: 8-byte chunk swizzles lose to padding on 15^6)
     if (Cb % (mask + 1) == 0 && blk_wc == 16)
-      for (int swz = lg; swz <= lg + 6; swz++) {
+      for (int swz = lg; swz <= lg + 6 && best_c > floor_c; swz++) {
         const double c = gather_cost(0, swz);
         if (c < best_c - 1e-9) {
           best_c = c;

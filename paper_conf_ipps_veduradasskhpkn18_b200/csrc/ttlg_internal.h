@@ -141,9 +141,11 @@ struct TileParams {
   // (input-run dims 0..a, then the output-run dims in output order, then the
   // other dims).  The input run is split into tm_np panels of tm_pa elements
   // of dim a (tm_pw bytes per box row, <= 128); panel p is one box load of
-  // tm_pbytes to stage + p * tm_pbytes, 128-byte swizzled.  Grid dim g
+  // tm_pbytes to stage + p * tm_pbytes, swizzled with the span of one row.  Grid dim g
   // contributes coordinate (digit * tm_gt[g]) to map dim tm_gmap[g].
   int32_t tm_rank, tm_np, tm_pa, tm_pw, tm_pbytes, tm_adim;
+  int32_t tm_swz;  // XOR mask the swizzle applies to (byte offset >> 3): 0x70 / 0x30 / 0x10 / 0
+                   // for box rows of 128 / 64 / 32 / 16 bytes (SWIZZLE_128B / 64B / 32B / none)
   int32_t tm_gmap[TTLG_MAXD], tm_gt[TTLG_MAXD];
   // host side (encoded per launch with the operand's address, kernels.cu)
   int64_t tm_dim[TTLG_MAXD];     // globalDim, map order

@@ -716,7 +716,7 @@ def test_blk_batch():
 
 @pytest.mark.parametrize("case", _bulk_cases(), ids=lambda c: c.label())
 def test_tmap_forced(case):
-    """k_tmap (variant 10: TMA tensor-map box loads, 128-byte swizzle, k_bulk's
+    """k_tmap (variant 10: TMA tensor-map box loads, swizzled box rows, k_bulk's
     quad consumers) forced on every config shape it applies to (fused rank
     <= 5, 16-byte aligned strides)."""
     try:

@@ -361,10 +361,10 @@ def test_tmap_applicability():
         with pytest.raises(ttlg.TtlgError) as e:
             ttlg.plan("f64" if ext[0] != 3 else "f32", ext, perm, variant=10)
         assert e.value.code == 7
-    # every candidate keeps the box rule: the input run is one panel of <= 128
-    # bytes or whole 128-byte panels of dim a
+    # every candidate keeps the box rule: the input run is one box row of a
+    # swizzle span (16 / 32 / 64 / 128 bytes) or whole 128-byte panels of dim a
     for c in ttlg.plan_candidates("f64", [200, 136], [1, 0], variant=10):
         la = c["in_run"] * 8
-        assert la <= 128 or la % 128 == 0
+        assert la in (16, 32, 64, 128) or la % 128 == 0
     auto = ttlg.plan("f64", [5120, 5120], [1, 0]).describe()
     assert auto["kernel"] != "tmap"

@@ -62,6 +62,9 @@ def main():
     ap.add_argument("--log-size", action="store_true", help="tensor sizes log-uniform")
     ap.add_argument("--max-cand", type=int, default=40)
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--graph", type=int, default=0,
+                    help="time R back-to-back launches captured as one CUDA graph (per-launch "
+                         "time = replay / R) instead of an event pair around one launch")
     ap.add_argument("--stride", type=int, default=1)
     ap.add_argument("--ids", default="", help="comma list of case ids to keep")
     ap.add_argument("--threads", default="", help="comma list of block sizes to try per candidate")
@@ -84,6 +87,7 @@ def main():
     dev = torch.device("cuda:0")
     stream = torch.cuda.current_stream()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    gs = torch.cuda.Stream()
     for c in cases:
         dt = "f64" if c.elem_bytes == 8 else "f32"
         cands = ttlg.plan_candidates(dt, c.extents, c.perm)
@@ -112,12 +116,32 @@ def main():
             for _ in range(2):
                 p.execute(A.data_ptr(), B.data_ptr(), stream.cuda_stream)
             ts = []
-            for _ in range(args.reps):
-                e0.record()
-                p.execute(A.data_ptr(), B.data_ptr(), stream.cuda_stream)
-                e1.record()
-                e1.synchronize()
-                ts.append(e0.elapsed_time(e1) * 1e-3)
+            if args.graph:
+                # back-to-back launches as one CUDA graph (no launch gaps: the
+                # kernel time a bench step sees; an event pair around ONE launch
+                # after a sync also times the host's launch latency, which
+                # dominates tensors below a few MB)
+                torch.cuda.synchronize()
+                g = torch.cuda.CUDAGraph()
+                with torch.cuda.graph(g, stream=gs):
+                    for _ in range(args.graph):
+                        p.execute(A.data_ptr(), B.data_ptr(), gs.cuda_stream)
+                with torch.cuda.stream(gs):
+                    g.replay()
+                    for _ in range(args.reps):
+                        e0.record(gs)
+                        g.replay()
+                        e1.record(gs)
+                        e1.synchronize()
+                        ts.append(e0.elapsed_time(e1) * 1e-3 / args.graph)
+                del g
+            else:
+                for _ in range(args.reps):
+                    e0.record()
+                    p.execute(A.data_ptr(), B.data_ptr(), stream.cuda_stream)
+                    e1.record()
+                    e1.synchronize()
+                    ts.append(e0.elapsed_time(e1) * 1e-3)
             t = statistics.median(ts)
             print(json.dumps({
                 "case": c.label(), "group": c.group, "bytes": c.alg_bytes, "W": info["access_bytes"],
@@ -127,6 +151,7 @@ def main():
                 "V": info["tile_volume"], "tiles": info["num_tiles"], "grid": info["grid"],
                 "occ": info["occupancy"], "nstage": info["stages"], "features": info["features"],
                 "pred": info["predicted_seconds"], "meas": t, "gbs": c.alg_bytes / t / 1e9,
+                "timing": f"graph{args.graph}" if args.graph else "event",
                 "is_auto": info["tile_extents"] == auto["tile_extents"]
                 and info["schema"] == auto["schema"]}), flush=True)
         del A, B

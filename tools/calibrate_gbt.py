@@ -15,6 +15,7 @@ from __future__ import annotations
 
 import argparse
 import collections
+import gzip
 import json
 import math
 import os
@@ -74,7 +75,9 @@ def main():
     ap.add_argument("--sym", default="kGbt", help="C symbol prefix of the tree set")
     ap.add_argument("--out", default="model_gbt.h", help="header name under csrc/")
     args = ap.parse_args()
-    rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
+    def lines(f):
+        return gzip.open(f, "rt") if f.endswith(".gz") else open(f)
+    rows = [json.loads(l) for f in args.files for l in lines(f) if l.startswith("{")]
     # k_deint is not ranked by the trees (its time is a measured factor, model.h)
     rows = [r for r in rows if r["kernel"] in KID]
     co = linear_coefs()
