@@ -609,13 +609,22 @@ def main():
                         if kname(infos[i]) == k:
                             p.execute(As[i].data_ptr(), Bs[i].data_ptr(), sptr)
                 kev[k][s][1].record(stream)
-    # per-case durations (model error, per-case table): in graph mode each case
-    # as its own graph of K back-to-back launches between one event pair (the
-    # kernel time the step sees; an event pair per launch also times the host's
-    # launch rate, which dominates sub-10-us kernels); else an event pair per launch
-    if graph is not None:
-        per_case_ms = []
+    # per-case durations (model error, per-case table): an event pair per
+    # launch; in graph mode, cases moving < 32 MB (tensors < 16 MB, kernels of a few
+    # us: an event pair per launch times the host's launch rate there) as
+    # their own graph of K back-to-back launches between one event pair --
+    # the two timings the model was calibrated with (cal35 / cal33; the third
+    # and second tree sets report the predictions on either side)
+    for s in range(args.steps):
+        one_step(evs[s])
+    torch.cuda.synchronize()
+    per_case_ms = [[evs[s][i][0].elapsed_time(evs[s][i][1]) for s in range(args.steps)]
+                   for i in range(len(plans))]
+    small_case = [c.alg_bytes < 32 * 2 ** 20 for c in cases]  # model.h kSmallTraffic
+    if graph is not None and any(small_case):
         for i, p in enumerate(plans):
+            if not small_case[i]:
+                continue
             cg = torch.cuda.CUDAGraph()
             with torch.cuda.graph(cg, stream=stream):
                 for _ in range(args.steps):
@@ -629,14 +638,8 @@ def main():
                     evs[0][i][1].record(stream)
                     evs[0][i][1].synchronize()
                     ms.append(evs[0][i][0].elapsed_time(evs[0][i][1]) / args.steps)
-            per_case_ms.append(ms)
+            per_case_ms[i] = ms
             del cg
-    else:
-        for s in range(args.steps):
-            one_step(evs[s])
-        torch.cuda.synchronize()
-        per_case_ms = [[evs[s][i][0].elapsed_time(evs[s][i][1]) for s in range(args.steps)]
-                       for i in range(len(plans))]
     torch.cuda.synchronize()
     clk = clocks.stop()
     groups = {}
@@ -781,9 +784,10 @@ def main():
                        "timing": "value: K steps between two events (no per-launch events); "
                                  "roofline/kernels: a second pass of K steps, each kernel's "
                                  "launches grouped (as one graph in graph mode) between one "
-                                 "event pair per step; cases / model error: a third pass, "
-                                 + ("each case as a graph of K launches between one event pair"
-                                    if graph is not None else "an event pair per launch"),
+                                 "event pair per step; cases / model error: a third pass "
+                                 "with an event pair per launch"
+                                 + ("; cases moving < 32 MB each as a graph of K launches "
+                                    "between one event pair" if graph is not None else ""),
                        "l2": l2_label},
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": peak,

@@ -10,7 +10,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libttlg.so")
 SOURCES = ["api.cpp", "planner.cpp", "model.cpp", "kernels.cu"]
-HEADERS = ["ttlg_internal.h", "model.h", "model_coeffs.h", "model_gbt.h", "model_gbt2.h"]
+HEADERS = ["ttlg_internal.h", "model.h", "model_coeffs.h", "model_gbt.h", "model_gbt2.h",
+           "model_gbt3.h"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

@@ -117,6 +117,7 @@ double predict_seconds(const ModelInput &mi, const DeviceProfile &dev) {
 // ---- ranking stage: boosted regression trees (model_gbt.h) --------------------
 #include "model_gbt.h"
 #include "model_gbt2.h"
+#include "model_gbt3.h"
 
 namespace ttlg {
 
@@ -208,6 +209,10 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
 
 void predict_ranked2_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
   gbt_batch<kGbt2Trees, kGbt2Depth>(mis, n, dev, out, kGbt2Init, kGbt2F, kGbt2T, kGbt2V);
+}
+
+void predict_ranked3_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out) {
+  gbt_batch<kGbt3Trees, kGbt3Depth>(mis, n, dev, out, kGbt3Init, kGbt3F, kGbt3T, kGbt3V);
 }
 
 }  // namespace ttlg

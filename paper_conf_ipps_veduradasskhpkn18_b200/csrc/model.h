@@ -43,6 +43,11 @@ void predict_ranked_batch(const ModelInput *mis, int n, const DeviceProfile &dev
 // second tree set (model_gbt2.h: refit with k_vec / k_bulk and small tensors in the
 // data): decides whether a k_vec candidate beats the first set's winner
 void predict_ranked2_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
+// third tree set (model_gbt3.h: the second set's data with the tensors below
+// 32 MB re-timed as CUDA graphs of back-to-back launches, cal35 -- an event
+// pair around one launch after a sync also times the host's launch latency):
+// ranks and reports plans moving less than kSmallTraffic bytes
+void predict_ranked3_batch(const ModelInput *mis, int n, const DeviceProfile &dev, double *out);
 // k_vec replaces the winner only when predicted this much faster by the second set
 constexpr double kVecMargin = 0.95;
 // ... and is considered only when the first set predicts its winner below this
