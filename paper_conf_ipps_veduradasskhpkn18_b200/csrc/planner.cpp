@@ -194,6 +194,15 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : (group == KK_TMA ? tma : bulk);
 }
 constexpr int kBulkMaxStages = 6;
+// k_tmap CTAs per SM (TTLG_TMA_CTAS, 1..4; default 1: one ring per SM as k_bulk)
+static int tma_ctas() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_TMA_CTAS");
+    v = (e && e[0] >= '1' && e[0] <= '4') ? e[0] - '0' : 1;
+  }
+  return v;
+}
 // k_phase substitution mode (TTLG_PHASE: 0 off [default], 1 rows off 16-byte
 // boundaries, 2 always).  Measured on the 720-perm sweeps (r2e22): halving
 // the load instructions does not pay for the phase arithmetic and the
@@ -1131,10 +1140,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     if (kind == KK_BULKQ || kind == KK_BULKG || kind == KK_TMA) {
       // one output position (quad) / 16-byte output chunk (gather) per consumer thread
       if ((kind != KK_BULKG ? S.LB : S.LB * P.W / 16) > threads - 32) return false;
-      // as many ring stages as fit next to the tables (2..kBulkMaxStages), one CTA per SM
+      // as many ring stages as fit next to the tables (2..kBulkMaxStages), one CTA
+      // per SM (k_tmap: TTLG_TMA_CTAS per SM, each ring in its share)
       const int buf = (S.buf_bytes + 127) / 128 * 128;
       const int fixed = S.smem_base - S.buf_bytes + 256;
-      const int ns = std::min(kBulkMaxStages, (dev.smem_per_block_optin - fixed) / std::max(buf, 1));
+      const int cps = kind == KK_TMA ? tma_ctas() : 1;
+      const int room = cps == 1 ? dev.smem_per_block_optin
+                                : std::min(dev.smem_per_block_optin, dev.smem_per_sm / cps - 1024);
+      const int ns = std::min(kBulkMaxStages, (room - fixed) / std::max(buf, 1));
       if (ns < 2) return false;
       mi.nstage = ns;
       smem = fixed + ns * buf;
@@ -1161,7 +1174,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     mi.smem_bytes = smem;
     mi.occ = occupancy(dev, threads, smem, kernel_regs(kind, P.W));
     if (mi.occ < 1) return false;
-    if (mi.nstage) mi.occ = 1;  // __launch_bounds__(544, 1)
+    if (mi.nstage) mi.occ = kind == KK_TMA ? std::min(mi.occ, tma_ctas()) : 1;  // k_bulk: 1 per SM
     const int64_t slots = (int64_t)dev.sms * mi.occ;
     tpc = 1;
     if (mi.nstage) {

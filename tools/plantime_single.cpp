@@ -1,7 +1,8 @@
 // plantime_single.cpp -- host-only timing of the single-use planning path
 // (ttlg_transpose's plan at the effort level it picks; no GPU needed: with no
 // device the call plans, then returns TTLG_ERR_DEVICE at execute).  Prints
-// per shape: min / median microseconds over N calls.
+// per shape: min / median microseconds over N calls.  HOST-ONLY: on a machine
+// with a GPU the fake operand pointers would be launched on -- never run it there.
 //   g++ -O2 -std=c++17 -I include tools/plantime_single.cpp -L paper_conf_ipps_veduradasskhpkn18_b200 \
 //       -lttlg -Wl,-rpath,$PWD/paper_conf_ipps_veduradasskhpkn18_b200 -o tools/plantime_single
 //   tools/plantime_single [N] < tools/c3_shapes.txt
