@@ -10,6 +10,7 @@ from __future__ import annotations
 
 import argparse
 import collections
+import gzip
 import json
 import math
 import os
@@ -64,7 +65,7 @@ def main():
     ap.add_argument("--exclude", default="", help="comma list of kernels the trees do not rank")
     args = ap.parse_args()
     trees = load_trees(os.path.join(cg.CSRC, args.header), args.sym)
-    rows = [json.loads(l) for f in args.files for l in open(f) if l.startswith("{")]
+    rows = [json.loads(l) for f in args.files for l in (gzip.open(f, "rt") if f.endswith(".gz") else open(f)) if l.startswith("{")]
     rows = [r for r in rows if r["kernel"] in cg.KID
             and r["kernel"] not in args.exclude.split(",")]
     co = cg.linear_coefs()
