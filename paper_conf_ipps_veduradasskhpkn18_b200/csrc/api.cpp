@@ -1,5 +1,7 @@
 // api.cpp -- the C ABI declared in include/ttlg.h.
 #include <cuda_runtime.h>
+
+#include <cstdlib>
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
@@ -440,7 +442,12 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
   double bytes = 2.0 * (dt == TTLG_F64 ? 8 : 4);
   for (int k = 0; k < rank; k++) bytes *= (double)extents[k];
   const double pass = bytes / (device_profile(current_device()).hbm_gbs * 1e9);
-  const int fast = pass < kFast2PlanSeconds ? 2 : (pass < kFastPlanSeconds ? 1 : 0);
+  int fast = pass < kFast2PlanSeconds ? 2 : (pass < kFastPlanSeconds ? 1 : 0);
+  static const int forced = [] {  // TTLG_FAST_LEVEL=0/1/2 pins the level (experiments)
+    const char *e = getenv("TTLG_FAST_LEVEL");
+    return (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : -1;
+  }();
+  if (forced >= 0) fast = forced;
   st = plan_into(&p, dt, rank, extents, perm, nullptr, fast);
   if (st != TTLG_OK) return st;
   return execute(&p, A, B, stream);
