@@ -1110,8 +1110,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     Tile T;
     int kind, schema, tpc, group;
     int8_t delta[TTLG_MAXD];  // input-run padding chosen by the conflict search
+    uint64_t key;             // hash of the tile box (dedupe pre-check)
   };
   constexpr int kShort = 2 * kGbtTopK;
+  auto box_key = [&](const Tile &T) {
+    uint64_t h = 1469598103934665603ull;
+    for (int k = 0; k < P.d; k++) h = (h ^ (uint64_t)T.t[k]) * 1099511628211ull;
+    return h;
+  };
   // sink modes: full candidate listing (calibration) or the ranked short list
   // (measure-mode tuning, ttlg_plan_tune)
   const bool listing = sink && !sink->shortlist;
@@ -1278,9 +1284,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
                     int tpc, int group, const int *delta) {
     // different (a, ta, b, tb) can describe the same tile box: keep one entry
     // per (box, kernel, block size) so the short list stays diverse
+    const uint64_t key = box_key(T);
     for (int i = 0; i < ntop; i++) {
       const Entry &o = pool[i];
-      if (o.kind != kind || o.mi.threads != mi.threads) continue;
+      if (o.key != key || o.kind != kind || o.mi.threads != mi.threads) continue;
       bool same = true;
       for (int k = 0; k < P.d && same; k++) same = o.T.t[k] == T.t[k];
       if (same) {
@@ -1320,6 +1327,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     e.schema = schema;
     e.tpc = tpc;
     e.group = group;
+    e.key = key;
     for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
     if (ntop == kShort) admit = pool[order[kShort - 1]].lin;
   };
@@ -1453,6 +1461,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           e.schema = schema;
           e.tpc = tpc;
           e.group = group;
+          e.key = box_key(T);
           for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = 0;
           continue;
         }
