@@ -85,7 +85,14 @@ static int current_device() {
 }
 
 constexpr double kFastPlanSeconds = 150e-6;
-constexpr double kFast2PlanSeconds = 35e-6;  // shorter than a fast-effort plan
+// passes shorter than a fast-effort plan: the second fast level (refine 8 /
+// rank 6) below 35 us, and below 45 us for rank >= 4 problems, whose level-1
+// plans take ~40 us on the GPU box's CPU: 16^6 fp64 (41-us passes) measured
+// single/repeated mean 1.034, max 1.08 on level 2 vs 1.042 / 1.51 on level 1
+// (r2e40); rank-3 problems of the same size plan fast enough on level 1 and
+// lose on level 2 (r2e41: [2, 4096, 4096] fp32 `2 1 0` 1.01 -> 1.18)
+constexpr double kFast2PlanSeconds = 35e-6;
+constexpr double kFast2PlanSecondsHighRank = 45e-6;
 
 static ttlg_status plan_into(ttlg_plan_s *p, ttlg_dtype dt, int rank, const int64_t *ext,
                              const int32_t *perm, const ttlg_plan_hints *hints,
@@ -442,7 +449,8 @@ ttlg_status ttlg_transpose(ttlg_dtype dt, int rank, const int64_t *extents, cons
   double bytes = 2.0 * (dt == TTLG_F64 ? 8 : 4);
   for (int k = 0; k < rank; k++) bytes *= (double)extents[k];
   const double pass = bytes / (device_profile(current_device()).hbm_gbs * 1e9);
-  int fast = pass < kFast2PlanSeconds ? 2 : (pass < kFastPlanSeconds ? 1 : 0);
+  const double fast2 = rank >= 4 ? kFast2PlanSecondsHighRank : kFast2PlanSeconds;
+  int fast = pass < fast2 ? 2 : (pass < kFastPlanSeconds ? 1 : 0);
   static const int forced = [] {  // TTLG_FAST_LEVEL=0/1/2 pins the level (experiments)
     const char *e = getenv("TTLG_FAST_LEVEL");
     return (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : -1;
