@@ -1983,7 +1983,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (!listing && pool[win].lin < 1e299 && win_t > ideal_t / kVecChallenge && nv > 0 &&
       P.p[0] == 0) {
     const bool use_vec = true;
-    if (fast >= 2) nv = std::min(nv, 4);  // level 1 keeps the full k_vec list (r2e41: [3, 4096, 4096] `0 2 1` 65.7 -> 85.7 us on 4)
+    // single use: 4 k_vec slices (the full list's gather-conflict padding
+    // searches cost ~190 us of planning, r2e42; on 4 [3, 4096, 4096] `0 2 1`
+    // runs an 86-us slice instead of the 66-us one, r2e41)
+    if (fast) nv = std::min(nv, 4);
     ModelInput cm[1 + kVecShort];
     const Entry *ce[1 + kVecShort];
     int m = 0;
