@@ -919,7 +919,9 @@ static void smem_conflicts(const TileParams &K, int W, double &load, double &sto
 // k_vec's gather: lane l of the first warp owns output chunk q = l mod LBc of
 // B-row l / LBc and reads positions K q + u (u < K): the worst wavefront ratio
 // over the K reads (1 = conflict-free)
-static double vec_conflicts(const TileParams &K, int W) {
+// (stop: return as soon as the ratio reaches it -- the padding search only
+// needs to know that a layout is not better than its incumbent)
+static double vec_conflicts(const TileParams &K, int W, double stop = 1e300) {
   const int Kc = 16 / W, LBc = K.LB / Kc;
   auto offsets = [](int cnt, int n, const int32_t *ext, const int32_t *sS, int64_t *out) {
     int dig[TTLG_MAXD] = {0};
@@ -945,6 +947,7 @@ static double vec_conflicts(const TileParams &K, int W) {
       addr[l] = rows[r] + cols[j];
     }
     worst = std::max(worst, wavefront_ratio(addr, W));
+    if (worst >= stop) break;
   }
   return worst;
 }
@@ -1228,7 +1231,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         d2[0] = m;
         TileParams Kt;
         if (!build_params(P, T, group, thr_list[0], 1, Kt, d2)) continue;
-        const double c2 = vec_conflicts(Kt, P.W);
+        const double c2 = vec_conflicts(Kt, P.W, best);
         if (c2 < best - 1e-9) {
           best = c2;
           bp = m;
@@ -1983,10 +1986,26 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   if (!listing && pool[win].lin < 1e299 && win_t > ideal_t / kVecChallenge && nv > 0 &&
       P.p[0] == 0) {
     const bool use_vec = true;
-    // single use: 4 k_vec slices (the full list's gather-conflict padding
-    // searches cost ~190 us of planning, r2e42; on 4 [3, 4096, 4096] `0 2 1`
-    // runs an 86-us slice instead of the 66-us one, r2e41)
-    if (fast) nv = std::min(nv, 4);
+    // single use: refine 4 k_vec slices, not all (the full list's
+    // gather-conflict padding searches cost ~190 us of planning, r2e42) --
+    // the 4 the second tree set ranks best on their screen features (the
+    // linear screen's best 4 ran an 86-us slice on [3, 4096, 4096] `0 2 1`
+    // where the full plan runs 66 us, r2e41)
+    if (fast && nv > 4) {
+      ModelInput pm[kVecShort];
+      double pt[kVecShort];
+      int idx[kVecShort];
+      for (int i = 0; i < nv; i++) {
+        pm[i] = vpool[i].mi;
+        idx[i] = i;
+      }
+      predict_ranked2_batch(pm, nv, dev, pt);
+      std::partial_sort(idx, idx + 4, idx + nv, [&](int x, int y) { return pt[x] < pt[y]; });
+      Entry keep[4];
+      for (int j = 0; j < 4; j++) keep[j] = vpool[idx[j]];
+      for (int j = 0; j < 4; j++) vpool[j] = keep[j];
+      nv = 4;
+    }
     ModelInput cm[1 + kVecShort];
     const Entry *ce[1 + kVecShort];
     int m = 0;
