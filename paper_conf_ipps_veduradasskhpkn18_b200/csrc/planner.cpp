@@ -194,6 +194,12 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : (group == KK_TMA ? tma : bulk);
 }
 constexpr int kBulkMaxStages = 6;
+// k_direct cap for odd-length output rows (TTLG_FML_CAP=0 disables it)
+constexpr int64_t kFmlOddTileBytes = 34 * 1024;
+static bool fml_cap() {
+  static const bool v = env_flag("TTLG_FML_CAP", true);
+  return v;
+}
 // k_tmap CTAs per SM (TTLG_TMA_CTAS, 1..4; default 1: one ring per SM as k_bulk)
 static int tma_ctas() {
   static int v = -1;
@@ -1384,6 +1390,16 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       }
       if (LBc > 512 && ndig > 1) return;
     } else if (V * P.W > 256 * 1024) {
+      return;
+    } else if (fml_cap() && V * P.W > kFmlOddTileBytes && (P.n[0] * P.W) % 32 != 0 &&
+               P.n[0] * P.W < 2048 && V / T.t[0] >= 32) {
+      // k_direct tiles of >= 32 output rows that are not 32-byte multiples
+      // and shorter than 2 KB (odd fp64 extents) lose beyond ~34 KB although
+      // the model sees no difference: 127^4 `0 2 1 3` [127, 127] 4.6 TB/s vs
+      // [127, 33] 6.5, 63^4 [63, 63, 2] 5.9 vs [63, 63, 1] 6.3 (r2e45).  A/B
+      // (r2e46, per-case graph timing): Fig. 13 sizes 5457 -> 6233 GB/s, the
+      // 33 changed 15^6 plans +3.9 % (0.94-1.38); 17^6's 2312-byte rows lost
+      // 10 % under the cap, hence the 2 KB bound
       return;
     }
     TileSummary S;
