@@ -368,3 +368,27 @@ def test_tmap_applicability():
         assert la in (16, 32, 64, 128) or la % 128 == 0
     auto = ttlg.plan("f64", [5120, 5120], [1, 0]).describe()
     assert auto["kernel"] != "tmap"
+
+
+def test_direct_cap_for_odd_short_rows():
+    """k_direct tiles of >= 32 output rows that are not 32-byte multiples and
+    shorter than 2 KB stay <= 34 KB (r2e45-47: 127^4 `0 2 1 3`
+    [127, 127] ran 4.6 TB/s, [127, 33] 6.5); 2312-byte rows (17^6) are not
+    capped; TTLG_FML_CAP=0 lifts the cap (checked in a child process: the
+    flag is read once)."""
+    for ext in ([127] * 4, [63] * 4, [31] * 4):
+        for c in ttlg.plan_candidates("f64", ext, [0, 2, 1, 3]):
+            if c["kernel"] == "direct" and c["tile_volume"] // c["tile_extents"][0] >= 32:
+                assert c["tile_volume"] * 8 <= 34 * 1024, c
+    big = [c for c in ttlg.plan_candidates("f64", [17] * 6, [0, 1, 4, 3, 2, 5])
+           if c["kernel"] == "direct" and c["tile_volume"] * 8 > 34 * 1024]
+    assert big
+    import subprocess
+    import sys
+    code = ("import paper_conf_ipps_veduradasskhpkn18_b200 as t\n"
+            "c = t.plan_candidates('f64', [127] * 4, [0, 2, 1, 3])\n"
+            "print(max(x['tile_volume'] for x in c if x['kernel'] == 'direct') * 8)\n")
+    env = dict(os.environ, TTLG_FML_CAP="0")
+    out = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True,
+                         cwd=os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    assert int(out.stdout.strip()) > 34 * 1024, out.stderr
