@@ -15,6 +15,7 @@
 #include <string.h>
 
 #include <algorithm>
+#include <vector>
 #include <cmath>
 
 #include "model.h"
@@ -194,6 +195,18 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : (group == KK_TMA ? tma : bulk);
 }
 constexpr int kBulkMaxStages = 6;
+// tree pre-screen for repeated-use plans (option, TTLG_TREE_SCREEN=1): the
+// ranking trees also score every screened candidate and their best
+// kTreeScreen join the linear screen's best kTreeScreen in the short list.
+// A/B on every workload (r2e50, per-case graph timing): configs 2 / 3 / 4
+// +0.1 / +0.5 / +0.2 %, 720-16 / 720-15 +0.3 / +0.5 %, config 1 +1.6 %, but
+// 720-17 -0.6 % with single perms down to 0.74 and Fig. 13 -0.2 %; TTC cases
+// below 0.9 of D2D 3 -> 1, CCSD(T) 2 -> 3 -- mixed, so off by default
+constexpr int kTreeScreen = 16;
+static bool tree_screen() {
+  static const bool v = env_flag("TTLG_TREE_SCREEN", false);
+  return v;
+}
 // k_direct cap for odd-length output rows (TTLG_FML_CAP=0 disables it)
 constexpr int64_t kFmlOddTileBytes = 34 * 1024;
 static bool fml_cap() {
@@ -1130,6 +1143,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // sink modes: full candidate listing (calibration) or the ranked short list
   // (measure-mode tuning, ttlg_plan_tune)
   const bool listing = sink && !sink->shortlist;
+  // repeated-use plans: every screened candidate, for the tree pre-screen
+  const bool tscreen = !listing && !fast && tree_screen() && !(hints && hints->variant);
+  std::vector<Entry> allc;
   Entry pool[kShort];
   int order[kShort];  // pool slots sorted by the linear prediction
   // k_vec candidates of the automatic choice rank in their own short list and
@@ -1483,6 +1499,19 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           e.key = box_key(T);
           for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = 0;
           continue;
+        }
+        if (tscreen) {
+          Entry e;
+          e.lin = tm;
+          e.mi = mi;
+          e.T = T;
+          e.kind = kind;
+          e.schema = schema;
+          e.tpc = tpc;
+          e.group = group;
+          e.key = box_key(T);
+          for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
+          allc.push_back(e);
         }
         if (tm < admit) insert(tm, mi, T, kind, schema, tpc, group, delta);
       }
@@ -1912,6 +1941,50 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     return forced ? TTLG_ERR_UNSUPPORTED : TTLG_ERR_INTERNAL;
   }
 
+  // tree pre-screen: the short list becomes the linear screen's best
+  // kTreeScreen plus the trees' best kTreeScreen of every screened candidate
+  // (the linear screen alone dropped e.g. TTC `3 2 5 1 0 4`'s fastest slice,
+  // a 512-thread k_tile at linear rank 281 of 1004 that the trees rank first)
+  bool merged = false;
+  if (tscreen && (int)allc.size() > kTreeScreen) {
+    const int n = (int)allc.size();
+    std::vector<ModelInput> mis(n);
+    std::vector<double> tp(n);
+    std::vector<int> idx(n);
+    for (int i = 0; i < n; i++) {
+      mis[i] = allc[i].mi;
+      idx[i] = i;
+    }
+    if (2.0 * (double)N * P.W < kSmallTraffic)
+      predict_ranked3_batch(mis.data(), n, dev, tp.data());
+    else
+      predict_ranked_batch(mis.data(), n, dev, tp.data());
+    std::partial_sort(idx.begin(), idx.begin() + kTreeScreen, idx.end(),
+                      [&](int x, int y) { return tp[x] < tp[y]; });
+    Entry nb[kShort];
+    int nn = 0;
+    for (int i = 0; i < std::min(ntop, kTreeScreen); i++) nb[nn++] = pool[order[i]];
+    for (int j = 0; j < kTreeScreen && nn < kShort; j++) {
+      const Entry &c = allc[idx[j]];
+      bool dup = false;
+      for (int i = 0; i < nn && !dup; i++) {
+        const Entry &o = nb[i];
+        if (o.key != c.key || o.kind != c.kind || o.mi.threads != c.mi.threads) continue;
+        bool same = true;
+        for (int k = 0; k < P.d && same; k++) same = o.T.t[k] == c.T.t[k];
+        dup = same;
+      }
+      if (!dup) nb[nn++] = c;
+    }
+    for (int i = 0; i < nn; i++) {
+      pool[i] = nb[i];
+      order[i] = i;
+    }
+    ntop = nn;
+    std::sort(order, order + ntop, [&](int x, int y) { return pool[x].lin < pool[y].lin; });
+    merged = true;
+  }
+
   // refine the short list: exact blocks, conflicts and padding (cached per geometry)
   if (!listing) {
     struct Done {
@@ -1965,10 +2038,12 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // ranking stage: boosted trees over the kGbtTopK best
   int win = order[0];
   double win_t = 1e300;
-  ModelInput rk[kGbtTopK];
-  int rid[kGbtTopK], nrk = 0;
-  double rt[kGbtTopK];
-  const int topk = fast >= 2 ? kFast2TopK : (fast ? kFastTopK : kGbtTopK);
+  ModelInput rk[kShort];
+  int rid[kShort], nrk = 0;
+  double rt[kShort];
+  // (after the tree pre-screen every short-list entry is ranked: the trees'
+  // picks need not be among the refined linear best kGbtTopK)
+  const int topk = fast >= 2 ? kFast2TopK : (fast ? kFastTopK : (merged ? kShort : kGbtTopK));
   for (int i = 0; i < std::min(ntop, topk); i++) {
     const Entry &e = pool[order[i]];
     if (e.lin >= 1e299) continue;
