@@ -203,8 +203,24 @@ constexpr int kBulkMaxStages = 6;
 // 720-17 -0.6 % with single perms down to 0.74 and Fig. 13 -0.2 %; TTC cases
 // below 0.9 of D2D 3 -> 1, CCSD(T) 2 -> 3 -- mixed, so off by default
 constexpr int kTreeScreen = 16;
-static bool tree_screen() {
-  static const bool v = env_flag("TTLG_TREE_SCREEN", false);
+// TTLG_TREE_SCREEN=1: merged short list (r2e50); =2: the trees' picks only
+// challenge the normal winner and replace it when predicted TTLG_TREE_MARGIN
+// percent faster (default 5)
+static int tree_screen_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_TREE_SCREEN");
+    v = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 0;
+  }
+  return v;
+}
+static bool tree_screen() { return tree_screen_mode() != 0; }
+static double tree_margin() {
+  static double v = -1;
+  if (v < 0) {
+    const char *e = getenv("TTLG_TREE_MARGIN");
+    v = (e && e[0]) ? atof(e) / 100.0 : 0.05;
+  }
   return v;
 }
 // k_direct cap for odd-length output rows (TTLG_FML_CAP=0 disables it)
@@ -1133,6 +1149,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     int kind, schema, tpc, group;
     int8_t delta[TTLG_MAXD];  // input-run padding chosen by the conflict search
     uint64_t key;             // hash of the tile box (dedupe pre-check)
+    bool ts;                  // a challenger from the tree pre-screen (mode 2)
   };
   constexpr int kShort = 2 * kGbtTopK;
   auto box_key = [&](const Tile &T) {
@@ -1146,8 +1163,9 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // repeated-use plans: every screened candidate, for the tree pre-screen
   const bool tscreen = !listing && !fast && tree_screen() && !(hints && hints->variant);
   std::vector<Entry> allc;
-  Entry pool[kShort];
-  int order[kShort];  // pool slots sorted by the linear prediction
+  constexpr int kPool = kShort + kTreeScreen;  // mode 2: linear short list + challengers
+  Entry pool[kPool];
+  int order[kPool];  // pool slots sorted by the linear prediction
   // k_vec candidates of the automatic choice rank in their own short list and
   // must beat the main winner under the second tree set (model_gbt2.h)
   constexpr int kVecShort = 16;
@@ -1353,6 +1371,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     e.tpc = tpc;
     e.group = group;
     e.key = key;
+    e.ts = false;
     for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
     if (ntop == kShort) admit = pool[order[kShort - 1]].lin;
   };
@@ -1497,6 +1516,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           e.tpc = tpc;
           e.group = group;
           e.key = box_key(T);
+          e.ts = false;
           for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = 0;
           continue;
         }
@@ -1510,6 +1530,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
           e.tpc = tpc;
           e.group = group;
           e.key = box_key(T);
+          e.ts = true;
           for (int k = 0; k < TTLG_MAXD; k++) e.delta[k] = (int8_t)delta[k];
           allc.push_back(e);
         }
@@ -1961,10 +1982,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       predict_ranked_batch(mis.data(), n, dev, tp.data());
     std::partial_sort(idx.begin(), idx.begin() + kTreeScreen, idx.end(),
                       [&](int x, int y) { return tp[x] < tp[y]; });
-    Entry nb[kShort];
+    Entry nb[kPool];
     int nn = 0;
-    for (int i = 0; i < std::min(ntop, kTreeScreen); i++) nb[nn++] = pool[order[i]];
-    for (int j = 0; j < kTreeScreen && nn < kShort; j++) {
+    const bool chall = tree_screen_mode() == 2;
+    for (int i = 0; i < (chall ? ntop : std::min(ntop, kTreeScreen)); i++) {
+      nb[nn] = pool[order[i]];
+      nb[nn++].ts = false;
+    }
+    for (int j = 0; j < kTreeScreen && nn < kPool; j++) {
       const Entry &c = allc[idx[j]];
       bool dup = false;
       for (int i = 0; i < nn && !dup; i++) {
@@ -1974,7 +1999,10 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
         for (int k = 0; k < P.d && same; k++) same = o.T.t[k] == c.T.t[k];
         dup = same;
       }
-      if (!dup) nb[nn++] = c;
+      if (!dup) {
+        nb[nn] = c;
+        nb[nn++].ts = chall;
+      }
     }
     for (int i = 0; i < nn; i++) {
       pool[i] = nb[i];
@@ -1995,7 +2023,7 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
       TileSummary S;
       bool ok;
     };
-    Done done[kShort];
+    Done done[kPool];
     int nd = 0;
     // fast planning (single-use calls on small tensors): refine only the
     // linear screen's best few; the rest drop out
@@ -2038,15 +2066,28 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
   // ranking stage: boosted trees over the kGbtTopK best
   int win = order[0];
   double win_t = 1e300;
-  ModelInput rk[kShort];
-  int rid[kShort], nrk = 0;
-  double rt[kShort];
-  // (after the tree pre-screen every short-list entry is ranked: the trees'
-  // picks need not be among the refined linear best kGbtTopK)
-  const int topk = fast >= 2 ? kFast2TopK : (fast ? kFastTopK : (merged ? kShort : kGbtTopK));
-  for (int i = 0; i < std::min(ntop, topk); i++) {
+  ModelInput rk[kPool];
+  int rid[kPool], nrk = 0;
+  double rt[kPool];
+  // (mode 1: every merged short-list entry is ranked -- the trees' picks need
+  // not be among the refined linear best kGbtTopK; mode 2: the refined linear
+  // best kGbtTopK of the linear short list as without the pre-screen, then
+  // the challengers)
+  const bool mode1 = merged && tree_screen_mode() == 1;
+  const int topk = fast >= 2 ? kFast2TopK : (fast ? kFastTopK : (mode1 ? kShort : kGbtTopK));
+  int nnorm = 0;
+  for (int i = 0; i < ntop && nnorm < topk; i++) {
     const Entry &e = pool[order[i]];
+    if (e.ts) continue;
+    nnorm++;
     if (e.lin >= 1e299) continue;
+    rk[nrk] = e.mi;
+    rid[nrk++] = order[i];
+  }
+  const int nfirst = nrk;
+  for (int i = 0; merged && i < ntop; i++) {
+    const Entry &e = pool[order[i]];
+    if (!e.ts || e.lin >= 1e299) continue;
     rk[nrk] = e.mi;
     rid[nrk++] = order[i];
   }
@@ -2058,8 +2099,14 @@ ttlg_status make_plan(ttlg_plan_s *plan, ttlg_dtype dt, int rank, const int64_t 
     predict_ranked3_batch(rk, nrk, dev, rt);
   else
     predict_ranked_batch(rk, nrk, dev, rt);
-  for (int i = 0; i < nrk; i++) {
+  for (int i = 0; i < nfirst; i++) {
     if (rt[i] < win_t) {
+      win_t = rt[i];
+      win = rid[i];
+    }
+  }
+  for (int i = nfirst; i < nrk; i++) {
+    if (rt[i] < win_t * (1.0 - tree_margin())) {
       win_t = rt[i];
       win = rid[i];
     }
