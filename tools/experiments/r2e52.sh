@@ -9,4 +9,4 @@ for w in c2 c3 c4 fig13 720-16 720-15 720-17 c1; do
     TTLG_TREE_SCREEN=$c timeout 900 python tools/cases.py --workload $w --out $O/cases_${w}_ts$c.json > /dev/null 2> $O/cases_${w}_ts$c.err
   done
 done
-timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "config1 or scaled or odd or rank6 or 720" > $O/t_sel.log 2>&1; tail -1 $O/t_sel.log
+TTLG_TREE_SCREEN=2 timeout 900 python -m pytest tests/test_gpu_parity.py -x -q -k "config1 or scaled or odd or rank6 or 720" > $O/t_sel.log 2>&1; tail -1 $O/t_sel.log
