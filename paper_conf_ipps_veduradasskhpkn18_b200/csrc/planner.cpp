@@ -195,13 +195,16 @@ static bool new_kernel_auto(int group) {
   return group == KK_VEC ? vec : (group == KK_TMA ? tma : bulk);
 }
 constexpr int kBulkMaxStages = 6;
-// tree pre-screen for repeated-use plans (option, TTLG_TREE_SCREEN=1): the
-// ranking trees also score every screened candidate and their best
-// kTreeScreen join the linear screen's best kTreeScreen in the short list.
-// A/B on every workload (r2e50, per-case graph timing): configs 2 / 3 / 4
-// +0.1 / +0.5 / +0.2 %, 720-16 / 720-15 +0.3 / +0.5 %, config 1 +1.6 %, but
-// 720-17 -0.6 % with single perms down to 0.74 and Fig. 13 -0.2 %; TTC cases
-// below 0.9 of D2D 3 -> 1, CCSD(T) 2 -> 3 -- mixed, so off by default
+// tree pre-screen for repeated-use plans: the ranking trees also score
+// every screened candidate (the linear screen alone dropped e.g. TTC
+// `3 2 5 1 0 4`'s fastest slice at linear rank 281 of 1004, which the trees
+// rank first).  Mode 2 (default): the trees' best kTreeScreen challenge the
+// normal winner and replace it when predicted TTLG_TREE_MARGIN (5) % faster --
+// A/B on every workload (r2e52, per-case graph timing): configs 2 / 3 / 4
+// +0.4 / +0.9 / +1.1 %, 720-17 +1.0 %, 720-15 +0.1 %, 720-16 / Fig. 13 /
+// config 1 unchanged plans.  Mode 1 merges the trees' picks into the short
+// list and ranks them all without a margin (r2e50: configs +0.1-0.5 % but
+// 720-17 -0.6 %, perms to 0.74); mode 0 turns the pre-screen off.
 constexpr int kTreeScreen = 16;
 // TTLG_TREE_SCREEN=1: merged short list (r2e50); =2: the trees' picks only
 // challenge the normal winner and replace it when predicted TTLG_TREE_MARGIN
@@ -210,7 +213,7 @@ static int tree_screen_mode() {
   static int v = -1;
   if (v < 0) {
     const char *e = getenv("TTLG_TREE_SCREEN");
-    v = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 0;
+    v = (e && e[0] >= '0' && e[0] <= '2') ? e[0] - '0' : 2;
   }
   return v;
 }
