@@ -199,16 +199,17 @@ constexpr int kBulkMaxStages = 6;
 // every screened candidate (the linear screen alone dropped e.g. TTC
 // `3 2 5 1 0 4`'s fastest slice at linear rank 281 of 1004, which the trees
 // rank first).  Mode 2 (default): the trees' best kTreeScreen challenge the
-// normal winner and replace it when predicted TTLG_TREE_MARGIN (5) % faster --
-// A/B on every workload (r2e52, per-case graph timing): configs 2 / 3 / 4
-// +0.4 / +0.9 / +1.1 %, 720-17 +1.0 %, 720-15 +0.1 %, 720-16 / Fig. 13 /
-// config 1 unchanged plans.  Mode 1 merges the trees' picks into the short
+// normal winner and replace it when predicted TTLG_TREE_MARGIN (8) % faster --
+// A/B on every workload at 5 % (r2e52, per-case graph timing): configs 2 / 3
+// / 4 +0.4 / +0.9 / +1.1 %, 720-17 +1.0 %, 720-15 +0.1 %, 720-16 / Fig. 13 /
+// config 1 unchanged plans; the 24^6 reversal swapped at a < 8 % predicted
+// gain and lost 11 % (r2e53), the TTC / config-4 wins carry > 8 %.  Mode 1 merges the trees' picks into the short
 // list and ranks them all without a margin (r2e50: configs +0.1-0.5 % but
 // 720-17 -0.6 %, perms to 0.74); mode 0 turns the pre-screen off.
 constexpr int kTreeScreen = 16;
 // TTLG_TREE_SCREEN=1: merged short list (r2e50); =2: the trees' picks only
 // challenge the normal winner and replace it when predicted TTLG_TREE_MARGIN
-// percent faster (default 5)
+// percent faster (default 8)
 static int tree_screen_mode() {
   static int v = -1;
   if (v < 0) {
@@ -222,7 +223,7 @@ static double tree_margin() {
   static double v = -1;
   if (v < 0) {
     const char *e = getenv("TTLG_TREE_MARGIN");
-    v = (e && e[0]) ? atof(e) / 100.0 : 0.05;
+    v = (e && e[0]) ? atof(e) / 100.0 : 0.08;
   }
   return v;
 }
